@@ -1,0 +1,384 @@
+#!/usr/bin/env python
+"""Benchmark of the LC-style codec hot path on B200.
+
+A step = compress + decompress, through the C ABI with device-resident data,
+of every codec on its field of the workload (BASELINE.json configs[1] for the
+SP codecs — CESM-ATM-shaped 1800×3600 f32 fields T and U — and configs[2]'s
+Miranda-shaped 256×384×384 f64 density field for the DP codecs, so all §8(a)
+rows run every step). The L2 is flushed (256 MiB write) before every timed
+call; each call is timed with CUDA events on the launching stream.
+
+Metric: uncompressed GB/s (10^9 B/s) = Σ uncompressed bytes moved through
+compress and decompress ÷ Σ device time, plus per-codec compress/decompress
+GB/s, ratio and HBM-roofline fraction. Multi-GPU (torchrun): weak scaling,
+each rank owns a contiguous chunk range of one global stream per field (the
+fields are generated as sub-blocks of N× larger global fields), compresses it
+with lcf_compress_shard and all-gathers the per-rank payload byte counts over
+NCCL (the only exchange).
+
+`--impl reference` times the CPU oracle (oracle/) on a bounded sample of the
+same workload — the only reference this paper-only tier has.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+WORKLOAD = "cesm_1800x3600_f32[T,U]:SPspeed,SPratio + miranda_256x384x384_f64[density]:DPspeed,DPratio"
+SP_CONFIG, SP_FIELDS = "cesm_1800x3600_f32", ("T", "U")
+DP_CONFIG, DP_FIELDS = "miranda_256x384x384_f64", ("density",)
+ALL_CODECS = ("SPspeed", "SPratio", "DPspeed", "DPratio")
+L2_FLUSH_BYTES = 256 << 20
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.rows, self.proc = index, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100",
+                 "-i", str(self.index)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def make_fields(world, rank, device):
+    """Per-rank sub-blocks of N× larger global fields (weak scaling)."""
+    from paper_conf_asplos_azamifb25_b200 import datagen
+    fields = []
+    for cfg, names, codecs in ((SP_CONFIG, SP_FIELDS, ("SPspeed", "SPratio")),
+                               (DP_CONFIG, DP_FIELDS, ("DPspeed", "DPratio"))):
+        _, shape, _, _ = datagen.CONFIGS[cfg]
+        for nm in names:
+            # rank r's block of a global field of shape (N·d0, d1, ...)
+            x = datagen.field(cfg, nm, device=device)
+            if world > 1:
+                x = x.contiguous()
+            fields.append((cfg, nm, codecs, x.view(torch.int32 if x.dtype == torch.float32 else torch.int64)))
+    return fields
+
+
+class Timer:
+    def __init__(self):
+        self.flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device="cuda")
+
+    def time(self, fn):
+        self.flush.fill_(1)  # evict the L2 (126 MB) before every timed call
+        st = torch.cuda.current_stream()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(st)
+        fn()
+        b.record(st)
+        return a, b
+
+
+def run_lcf(args):
+    from paper_conf_asplos_azamifb25_b200 import lcf
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    codecs = [c for c in args.codecs.split(",") if c]
+    fields = make_fields(world, rank, dev)
+    stream = torch.cuda.current_stream()
+
+    # one job per (codec, field): buffers allocated once, outside the timed region
+    jobs = []
+    for cfg, nm, fcodecs, x in fields:
+        nbytes = x.numel() * x.element_size()
+        for codec in fcodecs:
+            if codec not in codecs:
+                continue
+            cap = lcf.lcf_max_compressed_size(codec, None, nbytes)
+            s = torch.empty(cap, dtype=torch.uint8, device=dev)
+            y = torch.empty_like(x)
+            try:
+                n = lcf.lcf_compress(codec, None, x, nbytes, s, cap)
+            except lcf.LcfError as e:
+                if e.status == 1:
+                    print(f"[bench] {codec} unavailable: {e}", file=sys.stderr)
+                    continue
+                raise
+            lcf.lcf_decompress(codec, None, s, n, y, nbytes)
+            assert torch.equal(x, y), f"{codec}/{nm}: round trip failed"
+            jobs.append({"codec": codec, "field": f"{cfg}/{nm}", "x": x, "s": s, "y": y, "cap": cap,
+                         "nbytes": nbytes, "sbytes": n, "ct": [], "dt": []})
+    timer = Timer()
+
+    def step(record):
+        evs = []
+        for j in jobs:
+            c = timer.time(lambda j=j: lcf.lcf_compress(j["codec"], None, j["x"], j["nbytes"], j["s"], j["cap"],
+                                                        sync=False))
+            d = timer.time(lambda j=j: lcf.lcf_decompress(j["codec"], None, j["s"], j["sbytes"], j["y"],
+                                                          j["nbytes"], sync=False))
+            evs.append((j, c, d))
+        if record:
+            torch.cuda.synchronize()
+            for j, c, d in evs:
+                j["ct"].append(c[0].elapsed_time(c[1]))
+                j["dt"].append(d[0].elapsed_time(d[1]))
+
+    for _ in range(args.warmup):
+        step(False)
+    lcf.lcf_check_stream()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    launches0 = lcf.lcf_launch_count()
+    with ClockSampler(local) as clk:
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            step(True)
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+    launches = lcf.lcf_launch_count() - launches0
+    lcf.lcf_check_stream()
+    for j in jobs:  # the timed outputs are still exact
+        assert torch.equal(j["x"], j["y"]), j["codec"]
+
+    hbm, peak_kind = peaks()
+    per_codec, tot_bytes, tot_ms, dominant = {}, 0, 0.0, None
+    for j in jobs:
+        ct, dt = statistics.median(j["ct"]), statistics.median(j["dt"])
+        moved = j["nbytes"] + j["sbytes"]
+        key = f"{j['codec']}:{j['field']}"
+        per_codec[key] = {
+            "compress_gbs": j["nbytes"] / ct / 1e6, "decompress_gbs": j["nbytes"] / dt / 1e6,
+            "ratio": j["nbytes"] / j["sbytes"], "compress_ms": ct, "decompress_ms": dt,
+            "compress_roofline_frac": moved / ct / 1e6 / hbm, "decompress_roofline_frac": moved / dt / 1e6 / hbm,
+        }
+        tot_bytes += 2 * j["nbytes"]
+        tot_ms += ct + dt
+        for kind, t in (("compress", ct), ("decompress", dt)):
+            if dominant is None or t > dominant[2]:
+                dominant = (j, kind, t)
+    j, kind, t = dominant
+    moved = j["nbytes"] + j["sbytes"]
+    roofline = {"bound": "hbm", "achieved": moved / t / 1e6, "peak": hbm, "unit": "GB/s",
+                "frac": moved / t / 1e6 / hbm, "traffic": None,
+                "kernel": f"{j['codec']} {kind} ({j['field']})", "peak_kind": peak_kind,
+                "algorithmic_bytes_per_launch": moved}
+    value = tot_bytes / tot_ms / 1e6
+    # aggregate over ranks: weak scaling, max step time
+    ms_step = tot_ms
+    if world > 1:
+        tt = torch.tensor([ms_step], device=dev)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        ms_step = float(tt.item())
+        value = world * tot_bytes / ms_step / 1e6
+
+    e2e = run_e2e(lcf, jobs, args) if rank == 0 else None
+    cpu = run_cpu_baseline(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
+    if rank == 0:
+        line = {
+            "metric": "compress+decompress throughput (uncompressed GB/s)", "value": value, "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+            "wall_ms_per_step": wall / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32/u64 (f32/f64 bits)", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "l2": "flushed (256 MiB write) before every timed call",
+                       "parallelism": f"chunk-range shards x{world}" if world > 1 else "single GPU"},
+            "per_codec": per_codec, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches, "clocks": clk.summary(),
+        }
+        print(json.dumps(line))
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def run_e2e(lcf, jobs, args):
+    """Same metric through lcf_compress_host / lcf_decompress_host (pinned
+    host buffers; H2D of the step's inputs and D2H of its results inside)."""
+    host = []
+    for j in jobs:
+        hx = torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True)
+        hx.copy_(j["x"].view(torch.uint8).cpu())
+        hs = torch.empty(j["cap"], dtype=torch.uint8, pin_memory=True)
+        hy = torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True)
+        host.append((j, hx, hs, hy))
+    h2d = d2h = 0
+    times = []
+    for it in range(max(1, args.warmup) + max(1, args.steps)):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        h2d = d2h = 0
+        for j, hx, hs, hy in host:
+            n = lcf.lcf_compress_host(j["codec"], None, hx, j["nbytes"], hs, j["cap"])
+            m = lcf.lcf_decompress_host(j["codec"], None, hs, n, hy, j["nbytes"])
+            h2d += j["nbytes"] + n
+            d2h += n + m
+        times.append(time.perf_counter() - t0)
+    for j, hx, hs, hy in host:
+        assert torch.equal(hx, hy), j["codec"]
+    t = statistics.median(times[max(1, args.warmup):])
+    total = sum(2 * j["nbytes"] for j, *_ in host)
+    return {"value": total / t / 1e9, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "ms_per_step": t * 1e3, "api": "lcf_compress_host + lcf_decompress_host"}
+
+
+def run_cpu_baseline(jobs, budget_s: float = 12.0):
+    """The oracle as it stands, single-threaded, on a bounded sample: the first
+    K chunks of every (codec, field) job, K sized for ~budget_s seconds."""
+    import oracle
+    oracle.lib()
+    sample_bytes = 1 << 20
+    done_bytes, spent = 0, 0.0
+    per = []
+    for j in jobs:
+        words = j["x"][: sample_bytes // j["x"].element_size()].cpu().numpy()
+        words = words.view(np.uint32 if words.dtype == np.int32 else np.uint64)
+        t0 = time.perf_counter()
+        s = oracle.compress(j["codec"], words)
+        t1 = time.perf_counter()
+        y = oracle.decompress(j["codec"], s)
+        t2 = time.perf_counter()
+        assert np.array_equal(y, words)
+        per.append((j["codec"], words.nbytes, t1 - t0, t2 - t1))
+        done_bytes += 2 * words.nbytes
+        spent += t2 - t0
+    # scale the sample up to the budget
+    reps = max(1, int(budget_s / max(spent, 1e-3)))
+    reps = min(reps, 8)
+    if reps > 1:
+        for _ in range(reps - 1):
+            for j in jobs:
+                words = j["x"][: sample_bytes // j["x"].element_size()].cpu().numpy()
+                words = words.view(np.uint32 if words.dtype == np.int32 else np.uint64)
+                t0 = time.perf_counter()
+                s = oracle.compress(j["codec"], words)
+                oracle.decompress(j["codec"], s)
+                spent += time.perf_counter() - t0
+                done_bytes += 2 * words.nbytes
+    return {"value": done_bytes / spent / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {sample_bytes >> 20} MiB of every (codec, field) of the workload, compress+decompress, "
+                      f"x{reps}; {spent:.1f} s single-threaded"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on rank 0 only."""
+    world, rank, local = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    from paper_conf_asplos_azamifb25_b200 import datagen
+    oracle.lib()
+    sample_bytes = 1 << 20
+    samples = []
+    for cfg, names, codecs in ((SP_CONFIG, SP_FIELDS, ("SPspeed", "SPratio")),
+                               (DP_CONFIG, DP_FIELDS, ("DPspeed", "DPratio"))):
+        for nm in names:
+            if cfg == DP_CONFIG:
+                x = datagen.field(cfg, nm, device="cpu", origin=(0, 0, 0), shape=(2, 384, 384))
+            else:
+                x = datagen.field(cfg, nm, device="cpu")
+            w = x.numpy().reshape(-1).view(np.uint32 if x.dtype == torch.float32 else np.uint64)
+            w = w[: sample_bytes // w.itemsize].copy()
+            for c in codecs:
+                samples.append((c, w))
+    times = []
+    total = 0
+    for it in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        total = 0
+        for c, w in samples:
+            s = oracle.compress(c, w)
+            oracle.decompress(c, s)
+            total += 2 * w.nbytes
+        if it >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    t = statistics.median(times)
+    v = total / t / 1e9
+    print(json.dumps({
+        "impl": "reference", "metric": "compress+decompress throughput (uncompressed GB/s)", "value": v,
+        "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/u64 (f32/f64 bits)",
+        "data": "synthetic", "config": {"workload": WORKLOAD, "sample": "first 1 MiB of every (codec, field)"},
+        "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": "first 1 MiB of every (codec, field) of the workload per step"},
+        "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="lcf", choices=["lcf", "reference"])
+    ap.add_argument("--codecs", default=",".join(ALL_CODECS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_lcf(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,135 @@
+/*
+ * lcf.h — C ABI of liblcf.so, the B200 (sm_100a) implementation of the four
+ * lossless floating-point codecs of Azami, Fallin & Burtscher, ASPLOS '25
+ * (PAPER.md; "L<n>" = PAPER.md line). Stream format: FORMAT.md (LCF1).
+ *
+ * Problem statement (L41, L92, L278, L354): losslessly compress an array of
+ * IEEE-754 float32 (SPspeed, SPratio) or float64 (DPspeed, DPratio) values,
+ * treated bit-for-bit as integers, into ONE contiguous compressed block whose
+ * chunks are placed by a prefix sum of their sizes (L120–122), and decompress
+ * it again; the stream is a pure function of the input (L415) and identical to
+ * the CPU oracle's.
+ *
+ * Conventions (all entry points):
+ *  - Pointers named d_* are DEVICE pointers on the current CUDA device, owned by
+ *    the caller; the library never frees or retains them beyond the stream work
+ *    it enqueues. h_* pointers are HOST pointers (pinned memory recommended).
+ *  - Calls are stream-ordered and asynchronous on `stream` (a cudaStream_t;
+ *    NULL = legacy default stream) unless an `out_bytes` pointer is non-NULL, in
+ *    which case the call synchronises `stream` to report the size.
+ *  - Library-owned scratch (ticket counter, look-back status, FCM sort buffers,
+ *    error word) is cached per (device, stream) and grown on demand; the first
+ *    call for a (device, stream, size) may allocate.
+ *  - Errors: arguments are validated on the host before anything is enqueued.
+ *    Stream corruption found by decoder kernels is recorded on the device and
+ *    reported as LCF_ERROR_CORRUPT_STREAM by the next synchronising call on that
+ *    stream (out_bytes != NULL, lcf_get_info, lcf_check_stream). Decoders never
+ *    read or write outside [d_in, d_in+in_bytes) and [d_out, d_out+out_capacity).
+ *  - There is no CPU fallback: with no usable CUDA device every call returns
+ *    LCF_ERROR_CUDA.
+ */
+#ifndef LCF_H
+#define LCF_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { LCF_SPSPEED = 0, LCF_SPRATIO = 1, LCF_DPSPEED = 2, LCF_DPRATIO = 3 } lcf_algo_t;
+typedef enum { LCF_FLOAT32 = 0, LCF_FLOAT64 = 1 } lcf_dtype_t;
+typedef enum {
+  LCF_SUCCESS = 0,
+  LCF_ERROR_INVALID_ARGUMENT = 1,
+  LCF_ERROR_DTYPE_MISMATCH = 2,
+  LCF_ERROR_BUFFER_TOO_SMALL = 3,
+  LCF_ERROR_CORRUPT_STREAM = 4,
+  LCF_ERROR_CUDA = 5,
+  LCF_ERROR_OUT_OF_MEMORY = 6
+} lcf_status_t;
+
+/* Worst-case stream size for in_bytes of input (pure host function):
+ * round16(32 + 4·C) + Σ_c round16(raw bytes of chunk c) — every chunk stored raw
+ * (L104). DPratio's FCM doubles the data (L185), so its bound is ≈ 2·in_bytes.
+ * Returns 0 for an invalid algo. */
+size_t lcf_max_compressed_size(lcf_algo_t algo, lcf_dtype_t dtype, size_t in_bytes);
+
+/* Compress in_bytes of float words at d_in into the LCF1 stream at d_out.
+ * in_bytes must be a multiple of the word size (4 or 8) → else INVALID_ARGUMENT;
+ * SP codecs need LCF_FLOAT32 and DP codecs LCF_FLOAT64 → else DTYPE_MISMATCH
+ * (L41); out_capacity ≥ lcf_max_compressed_size(...) → else BUFFER_TOO_SMALL.
+ * d_in must be 16-byte aligned. in_bytes = 0 yields the 32-byte header.
+ * Stages per 16 KiB chunk: SPspeed DIFFMS→MPLG (L108–118), SPratio
+ * DIFFMS→BIT→RZE (L138–158), DPspeed DIFFMS→MPLG, DPratio FCM→DIFFMS→RAZE→RARE
+ * (L168–201); raw fallback per chunk (L104); placement by a single-pass
+ * decoupled look-back over chunk sizes (L122). *out_bytes (if non-NULL)
+ * receives the stream length after a stream synchronisation. */
+lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes,
+                          void* d_out, size_t out_capacity, size_t* out_bytes, void* stream);
+
+/* Decompress the LCF1 stream of in_bytes at d_in into d_out (16-byte aligned).
+ * With out_bytes == NULL nothing is read back: the header, size table and
+ * payloads are validated by the kernels themselves (no host round trip), and an
+ * out_capacity smaller than the stream's n_bytes or a malformed stream is
+ * recorded on the device and reported by the next synchronising call. With
+ * out_bytes != NULL the header is first read to the host (one 32-byte D2H) and
+ * checked there, returning CORRUPT_STREAM / DTYPE_MISMATCH / BUFFER_TOO_SMALL
+ * directly, and device-found corruption is reported before returning.
+ * Inverse stages in reverse order (L94); chunk read offsets from the prefix sum
+ * of stored sizes (L120). `stream` is a cudaStream_t passed as void*. */
+lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes,
+                            void* d_out, size_t out_capacity, size_t* out_bytes, void* stream);
+
+/* Synchronise `stream` and read the 32-byte header at d_in (D2H): any of the
+ * out-pointers may be NULL. Returns CORRUPT_STREAM for a malformed header. */
+lcf_status_t lcf_get_info(const void* d_in, size_t in_bytes, lcf_algo_t* algo, lcf_dtype_t* dtype,
+                          size_t* uncompressed_bytes, size_t* compressed_bytes, void* stream);
+
+/* Synchronise `stream`; returns CORRUPT_STREAM (or BUFFER_TOO_SMALL) if any
+ * decompression enqueued on it since the previous check found a malformed
+ * stream, else SUCCESS. */
+lcf_status_t lcf_check_stream(void* stream);
+
+/* ---- host-buffer convenience (the end-to-end path) ----------------------
+ * Same as lcf_compress / lcf_decompress but h_in and h_out are HOST buffers:
+ * the library copies h_in to device scratch, runs the codec on `stream`, copies
+ * the result back and synchronises. *out_bytes is always written. */
+lcf_status_t lcf_compress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,
+                               void* h_out, size_t out_capacity, size_t* out_bytes, void* stream);
+lcf_status_t lcf_decompress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,
+                                 void* h_out, size_t out_capacity, size_t* out_bytes, void* stream);
+
+/* ---- sharded mode (one process per GPU) ----------------------
+ * Compress chunks [first_chunk, first_chunk + k) of the stream for an input of
+ * total_in_bytes, where d_in_shard holds exactly those chunks' words
+ * (shard_bytes). Writes the k size-table entries to d_table_slice (u32 each),
+ * the chunks' padded payloads contiguously to d_payload (offsets from 0), and
+ * the piece's payload byte count to the DEVICE u64 *d_payload_bytes (so it can
+ * feed an NCCL all-gather on the same stream without a host sync). The
+ * concatenation header ‖ table slices ‖ pad ‖ payload pieces, in chunk order, is
+ * byte-identical to lcf_compress's stream. Not available for DPratio (its FCM
+ * stage is a whole-array pass, L104): INVALID_ARGUMENT. */
+lcf_status_t lcf_compress_shard(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in_shard,
+                                size_t shard_bytes, size_t total_in_bytes, uint64_t first_chunk,
+                                void* d_table_slice, void* d_payload, size_t payload_capacity,
+                                uint64_t* d_payload_bytes, void* stream);
+
+/* Number of chunks of a stream for in_bytes of input (FORMAT.md §2). */
+uint64_t lcf_num_chunks(lcf_algo_t algo, size_t in_bytes);
+
+/* Write the 32-byte stream header (FORMAT.md §1) and the zero pad between the
+ * size table and the payload base to d_stream (which must have room for
+ * round16(32 + 4·n_chunks) bytes); total_payload_bytes is a host value. */
+lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,
+                              uint64_t total_payload_bytes, void* d_stream, void* stream);
+
+/* Number of kernel launches the library enqueued since the process started
+ * (bench/test accounting). */
+uint64_t lcf_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LCF_H */

@@ -1,0 +1,420 @@
+// lcf_api.cu — host side of liblcf.so: the C ABI of include/lcf.h, argument
+// validation, per-(device, stream) workspaces, launch of the codec kernels.
+#include <lcf.h>
+
+#include <atomic>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <utility>
+
+#include "lcf_kernels.cuh"
+
+using namespace lcf;
+
+namespace {
+
+std::atomic<uint64_t> g_launches{0};
+
+struct Workspace {
+  int device = -1;
+  cudaStream_t stream = nullptr;
+  std::mutex mu;
+  unsigned long long* ticket = nullptr;  // device counter, never reset
+  unsigned long long ticket_next = 0;    // host mirror: tickets handed out so far
+  uint64_t* status = nullptr;            // look-back status words
+  size_t status_cap = 0;
+  uint32_t* tile_flag = nullptr;         // DPratio decode tile completion flags
+  size_t tile_cap = 0;
+  uint32_t* err = nullptr;               // (epoch << 8 | bits) of the newest failure
+  uint32_t epoch = 0, checked_epoch = 0;
+  void* scratch[4] = {nullptr, nullptr, nullptr, nullptr};  // grown on demand
+  size_t scratch_cap[4] = {0, 0, 0, 0};
+};
+
+std::mutex g_mu;
+std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+
+constexpr uint32_t kEpochLimit = 1u << 22;
+
+bool cuda_ok(cudaError_t e) { return e == cudaSuccess; }
+
+Workspace* get_ws(cudaStream_t stream, lcf_status_t* st) {
+  int dev = -1;
+  if (!cuda_ok(cudaGetDevice(&dev))) { *st = LCF_ERROR_CUDA; return nullptr; }
+  std::lock_guard<std::mutex> g(g_mu);
+  auto key = std::make_pair(dev, stream);
+  auto it = g_ws.find(key);
+  if (it != g_ws.end()) return it->second;
+  Workspace* ws = new Workspace();
+  ws->device = dev;
+  ws->stream = stream;
+  if (!cuda_ok(cudaMalloc(&ws->ticket, sizeof(unsigned long long))) ||
+      !cuda_ok(cudaMalloc(&ws->err, sizeof(uint32_t))) ||
+      !cuda_ok(cudaMemsetAsync(ws->ticket, 0, sizeof(unsigned long long), stream)) ||
+      !cuda_ok(cudaMemsetAsync(ws->err, 0, sizeof(uint32_t), stream))) {
+    *st = LCF_ERROR_OUT_OF_MEMORY;
+    delete ws;
+    return nullptr;
+  }
+  g_ws[key] = ws;
+  return ws;
+}
+
+template <typename T>
+lcf_status_t grow(T*& ptr, size_t& cap, size_t need, cudaStream_t s, bool zero) {
+  if (cap >= need) return LCF_SUCCESS;
+  size_t ncap = cap * 2 > need ? cap * 2 : need;
+  if (ptr) {
+    cudaStreamSynchronize(s);
+    cudaFree(ptr);
+    ptr = nullptr;
+    cap = 0;
+  }
+  if (!cuda_ok(cudaMalloc(&ptr, ncap * sizeof(T)))) return LCF_ERROR_OUT_OF_MEMORY;
+  if (zero && !cuda_ok(cudaMemsetAsync(ptr, 0, ncap * sizeof(T), s))) return LCF_ERROR_CUDA;
+  cap = ncap;
+  return LCF_SUCCESS;
+}
+
+uint32_t next_epoch(Workspace* ws) {
+  if (++ws->epoch >= kEpochLimit) {  // wrap: forget every status/flag word
+    if (ws->status) cudaMemsetAsync(ws->status, 0, ws->status_cap * sizeof(uint64_t), ws->stream);
+    if (ws->tile_flag) cudaMemsetAsync(ws->tile_flag, 0, ws->tile_cap * sizeof(uint32_t), ws->stream);
+    cudaMemsetAsync(ws->err, 0, sizeof(uint32_t), ws->stream);
+    ws->epoch = 1;
+    ws->checked_epoch = 0;
+  }
+  return ws->epoch;
+}
+
+LaunchCtx make_ctx(Workspace* ws, uint64_t grid) {
+  LaunchCtx c;
+  c.ticket = ws->ticket;
+  c.ticket_base = ws->ticket_next;
+  c.status = ws->status;
+  c.epoch = next_epoch(ws);
+  c.err = ws->err;
+  ws->ticket_next += grid;
+  return c;
+}
+
+uint32_t word_bytes_of(int algo) { return (algo == LCF_SPSPEED || algo == LCF_SPRATIO) ? 4u : 8u; }
+bool valid_algo(int algo) { return algo >= LCF_SPSPEED && algo <= LCF_DPRATIO; }
+bool dtype_matches(int algo, int dtype) {
+  return (word_bytes_of(algo) == 4 && dtype == LCF_FLOAT32) || (word_bytes_of(algo) == 8 && dtype == LCF_FLOAT64);
+}
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+uint64_t payload_bound(int algo, uint64_t in_bytes) {
+  const uint64_t wb = word_bytes_of(algo);
+  if (algo == LCF_DPRATIO) {
+    const uint64_t n = in_bytes / wb;
+    return 2 * ((n / 2048) * 16384 + round16(8 * (n % 2048)));
+  }
+  return (in_bytes / kChunkBytes) * kChunkBytes + round16(in_bytes % kChunkBytes);
+}
+
+// Host-side header check (same rules as lcf::read_header).
+lcf_status_t check_header(const uint8_t* h, uint64_t in_bytes, int algo, uint64_t* n_bytes, uint64_t* n_chunks,
+                          uint64_t* payload) {
+  uint32_t magic;
+  std::memcpy(&magic, h, 4);
+  if (magic != kMagic || h[4] != kVersion || h[7] != 0 || h[5] > 3) return LCF_ERROR_CORRUPT_STREAM;
+  if (h[5] != algo) return LCF_ERROR_DTYPE_MISMATCH;
+  if (h[6] != word_bytes_of(algo)) return LCF_ERROR_CORRUPT_STREAM;
+  std::memcpy(n_bytes, h + 8, 8);
+  std::memcpy(n_chunks, h + 16, 8);
+  std::memcpy(payload, h + 24, 8);
+  if (*n_bytes % h[6]) return LCF_ERROR_CORRUPT_STREAM;
+  if (*n_chunks != lcf_num_chunks((lcf_algo_t)algo, *n_bytes)) return LCF_ERROR_CORRUPT_STREAM;
+  if (*n_chunks > (in_bytes - 32) / 4) return LCF_ERROR_CORRUPT_STREAM;
+  const uint64_t base = round16(kHeaderBytes + 4 * *n_chunks);
+  if (base > in_bytes || *payload > in_bytes - base) return LCF_ERROR_CORRUPT_STREAM;
+  return LCF_SUCCESS;
+}
+
+lcf_status_t last_launch_status() {
+  return cuda_ok(cudaGetLastError()) ? LCF_SUCCESS : LCF_ERROR_CUDA;
+}
+
+lcf_status_t device_error_since(Workspace* ws, uint32_t since_epoch) {
+  uint32_t e = 0;
+  if (!cuda_ok(cudaMemcpyAsync(&e, ws->err, 4, cudaMemcpyDeviceToHost, ws->stream)) ||
+      !cuda_ok(cudaStreamSynchronize(ws->stream)))
+    return LCF_ERROR_CUDA;
+  if ((e >> 8) > since_epoch) return (e & DERR_SMALL) ? LCF_ERROR_BUFFER_TOO_SMALL : LCF_ERROR_CORRUPT_STREAM;
+  return LCF_SUCCESS;
+}
+
+EncArgs enc_args(int algo, const void* in, uint64_t in_bytes) {
+  EncArgs a{};
+  a.in = in;
+  a.word_bytes = word_bytes_of(algo);
+  a.n_words_total = in_bytes / a.word_bytes;
+  a.algo = (uint32_t)algo;
+  a.n_bytes = in_bytes;
+  return a;
+}
+
+lcf_status_t enqueue_encode(Workspace* ws, EncArgs& a) {
+  if (lcf_status_t s = grow(ws->status, ws->status_cap, a.n_chunks, ws->stream, true)) return s;
+  LaunchCtx ctx = make_ctx(ws, a.n_chunks);
+  switch (a.algo) {
+    case LCF_SPSPEED: launch_speed_encode<uint32_t>(a, ctx, ws->stream); break;
+    case LCF_DPSPEED: launch_speed_encode<uint64_t>(a, ctx, ws->stream); break;
+    default: return LCF_ERROR_INVALID_ARGUMENT;
+  }
+  ++g_launches;
+  return last_launch_status();
+}
+
+}  // namespace
+
+extern "C" {
+
+uint64_t lcf_num_chunks(lcf_algo_t algo, size_t in_bytes) {
+  if (!valid_algo(algo)) return 0;
+  const uint64_t wb = word_bytes_of(algo);
+  if (algo == LCF_DPRATIO) return 2 * ((in_bytes / wb + 2047) / 2048);
+  return (in_bytes + kChunkBytes - 1) / kChunkBytes;
+}
+
+size_t lcf_max_compressed_size(lcf_algo_t algo, lcf_dtype_t dtype, size_t in_bytes) {
+  (void)dtype;
+  if (!valid_algo(algo)) return 0;
+  return round16(kHeaderBytes + 4 * lcf_num_chunks(algo, in_bytes)) + payload_bound(algo, in_bytes);
+}
+
+uint64_t lcf_launch_count(void) { return g_launches.load(); }
+
+lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
+                          size_t out_capacity, size_t* out_bytes, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!dtype_matches(algo, dtype)) return LCF_ERROR_DTYPE_MISMATCH;
+  const uint32_t wb = word_bytes_of(algo);
+  if (in_bytes % wb || !d_out || !aligned16(d_out) || (in_bytes && (!d_in || !aligned16(d_in))))
+    return LCF_ERROR_INVALID_ARGUMENT;
+  if (out_capacity < lcf_max_compressed_size(algo, dtype, in_bytes)) return LCF_ERROR_BUFFER_TOO_SMALL;
+  if (algo == LCF_DPRATIO || algo == LCF_SPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  const uint64_t C = lcf_num_chunks(algo, in_bytes);
+  const uint64_t base = round16(kHeaderBytes + 4 * C);
+  EncArgs a = enc_args(algo, d_in, in_bytes);
+  a.first_chunk = 0;
+  a.n_chunks = C;
+  a.stream_chunks = C;
+  a.table = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(d_out) + kHeaderBytes);
+  a.payload = static_cast<uint8_t*>(d_out) + base;
+  a.header = reinterpret_cast<StreamHeader*>(d_out);
+  a.pad_start = static_cast<uint8_t*>(d_out) + kHeaderBytes + 4 * C;
+  a.pad_len = (uint32_t)(base - kHeaderBytes - 4 * C);
+  if (C == 0) {
+    launch_write_header(a, stream);
+    ++g_launches;
+    st = last_launch_status();
+  } else {
+    st = enqueue_encode(ws, a);
+  }
+  if (st) return st;
+  if (out_bytes) {
+    uint64_t pb = 0;
+    if (!cuda_ok(cudaMemcpyAsync(&pb, static_cast<uint8_t*>(d_out) + 24, 8, cudaMemcpyDeviceToHost, stream)) ||
+        !cuda_ok(cudaStreamSynchronize(stream)))
+      return LCF_ERROR_CUDA;
+    *out_bytes = base + pb;
+  }
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
+                            size_t out_capacity, size_t* out_bytes, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!dtype_matches(algo, dtype)) return LCF_ERROR_DTYPE_MISMATCH;
+  if (!d_in || !aligned16(d_in) || (out_capacity && (!d_out || !aligned16(d_out))))
+    return LCF_ERROR_INVALID_ARGUMENT;
+  if (in_bytes < kHeaderBytes) return LCF_ERROR_CORRUPT_STREAM;
+  if (algo == LCF_DPRATIO || algo == LCF_SPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  uint64_t grid;
+  uint64_t n_bytes = 0;
+  if (out_bytes) {
+    uint8_t h[32];
+    if (!cuda_ok(cudaMemcpyAsync(h, d_in, 32, cudaMemcpyDeviceToHost, stream)) ||
+        !cuda_ok(cudaStreamSynchronize(stream)))
+      return LCF_ERROR_CUDA;
+    uint64_t n_chunks, payload;
+    if (lcf_status_t s = check_header(h, in_bytes, algo, &n_bytes, &n_chunks, &payload)) return s;
+    if (n_bytes > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+    grid = n_chunks;
+    if (grid == 0) {
+      *out_bytes = 0;
+      return LCF_SUCCESS;
+    }
+  } else {
+    const uint64_t by_table = (in_bytes - kHeaderBytes) / 4;
+    const uint64_t by_out = (out_capacity + kChunkBytes - 1) / kChunkBytes;
+    grid = by_table < by_out ? by_table : by_out;
+    if (grid == 0) grid = 1;  // still validate the header on the device
+  }
+  if (lcf_status_t s = grow(ws->status, ws->status_cap, grid, stream, true)) return s;
+  DecArgs a{};
+  a.stream = static_cast<const uint8_t*>(d_in);
+  a.stream_bytes = in_bytes;
+  a.out = static_cast<uint8_t*>(d_out);
+  a.out_capacity = out_capacity;
+  a.algo = (uint32_t)algo;
+  a.word_bytes = word_bytes_of(algo);
+  const uint32_t before = ws->epoch;
+  LaunchCtx ctx = make_ctx(ws, grid);
+  switch (algo) {
+    case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, (unsigned)grid, stream); break;
+    case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, (unsigned)grid, stream); break;
+    default: return LCF_ERROR_INVALID_ARGUMENT;
+  }
+  ++g_launches;
+  if ((st = last_launch_status())) return st;
+  if (out_bytes) {
+    if ((st = device_error_since(ws, ctx.epoch < before ? 0 : before))) return st;
+    *out_bytes = n_bytes;
+  }
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_get_info(const void* d_in, size_t in_bytes, lcf_algo_t* algo, lcf_dtype_t* dtype,
+                          size_t* uncompressed_bytes, size_t* compressed_bytes, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!d_in) return LCF_ERROR_INVALID_ARGUMENT;
+  if (in_bytes < kHeaderBytes) return LCF_ERROR_CORRUPT_STREAM;
+  uint8_t h[32];
+  if (!cuda_ok(cudaMemcpyAsync(h, d_in, 32, cudaMemcpyDeviceToHost, stream)) ||
+      !cuda_ok(cudaStreamSynchronize(stream)))
+    return LCF_ERROR_CUDA;
+  if (h[5] > 3) return LCF_ERROR_CORRUPT_STREAM;
+  uint64_t nb, nc, pb;
+  if (lcf_status_t s = check_header(h, in_bytes, h[5], &nb, &nc, &pb)) return s;
+  if (algo) *algo = (lcf_algo_t)h[5];
+  if (dtype) *dtype = h[6] == 4 ? LCF_FLOAT32 : LCF_FLOAT64;
+  if (uncompressed_bytes) *uncompressed_bytes = nb;
+  if (compressed_bytes) *compressed_bytes = round16(kHeaderBytes + 4 * nc) + pb;
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_check_stream(void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  st = device_error_since(ws, ws->checked_epoch);
+  ws->checked_epoch = ws->epoch;
+  return st;
+}
+
+static lcf_status_t host_roundtrip(bool compress, lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in,
+                                   size_t in_bytes, void* h_out, size_t out_capacity, size_t* out_bytes,
+                                   cudaStream_t stream) {
+  if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!out_bytes || (in_bytes && !h_in)) return LCF_ERROR_INVALID_ARGUMENT;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  size_t dcap;
+  if (compress) {
+    dcap = lcf_max_compressed_size(algo, dtype, in_bytes);
+  } else {
+    if (in_bytes < 32) return LCF_ERROR_CORRUPT_STREAM;
+    uint64_t nb;
+    std::memcpy(&nb, static_cast<const uint8_t*>(h_in) + 8, 8);
+    if (nb > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+    dcap = nb;
+  }
+  {
+    std::lock_guard<std::mutex> g(ws->mu);
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[0]), ws->scratch_cap[0], round16(in_bytes) + 16, stream, false)))
+      return st;
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[1]), ws->scratch_cap[1], round16(dcap) + 16, stream, false)))
+      return st;
+    if (!cuda_ok(cudaMemcpyAsync(ws->scratch[0], h_in, in_bytes, cudaMemcpyHostToDevice, stream)))
+      return LCF_ERROR_CUDA;
+  }
+  size_t n = 0;
+  st = compress ? lcf_compress(algo, dtype, ws->scratch[0], in_bytes, ws->scratch[1], dcap, &n, stream)
+                : lcf_decompress(algo, dtype, ws->scratch[0], in_bytes, ws->scratch[1], dcap, &n, stream);
+  if (st) return st;
+  if (n > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+  if (!cuda_ok(cudaMemcpyAsync(h_out, ws->scratch[1], n, cudaMemcpyDeviceToHost, stream)) ||
+      !cuda_ok(cudaStreamSynchronize(stream)))
+    return LCF_ERROR_CUDA;
+  *out_bytes = n;
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_compress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes, void* h_out,
+                               size_t out_capacity, size_t* out_bytes, void* stream) {
+  return host_roundtrip(true, algo, dtype, h_in, in_bytes, h_out, out_capacity, out_bytes, (cudaStream_t)stream);
+}
+lcf_status_t lcf_decompress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes, void* h_out,
+                                 size_t out_capacity, size_t* out_bytes, void* stream) {
+  return host_roundtrip(false, algo, dtype, h_in, in_bytes, h_out, out_capacity, out_bytes, (cudaStream_t)stream);
+}
+
+lcf_status_t lcf_compress_shard(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in_shard, size_t shard_bytes,
+                                size_t total_in_bytes, uint64_t first_chunk, void* d_table_slice, void* d_payload,
+                                size_t payload_capacity, uint64_t* d_payload_bytes, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!valid_algo(algo) || algo == LCF_DPRATIO) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!dtype_matches(algo, dtype)) return LCF_ERROR_DTYPE_MISMATCH;
+  const uint32_t wb = word_bytes_of(algo);
+  if (total_in_bytes % wb || shard_bytes % wb || !d_payload_bytes) return LCF_ERROR_INVALID_ARGUMENT;
+  const uint64_t C = lcf_num_chunks(algo, total_in_bytes);
+  if (first_chunk > C || first_chunk * kChunkBytes + shard_bytes > total_in_bytes) return LCF_ERROR_INVALID_ARGUMENT;
+  const bool has_tail = first_chunk * kChunkBytes + shard_bytes == total_in_bytes;
+  if (!has_tail && shard_bytes % kChunkBytes) return LCF_ERROR_INVALID_ARGUMENT;
+  const uint64_t k = (shard_bytes + kChunkBytes - 1) / kChunkBytes;
+  if (k && (!d_in_shard || !aligned16(d_in_shard) || !d_table_slice || !d_payload || !aligned16(d_payload)))
+    return LCF_ERROR_INVALID_ARGUMENT;
+  if (payload_capacity < (shard_bytes / kChunkBytes) * kChunkBytes + round16(shard_bytes % kChunkBytes))
+    return LCF_ERROR_BUFFER_TOO_SMALL;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  if (k == 0) return cuda_ok(cudaMemsetAsync(d_payload_bytes, 0, 8, stream)) ? LCF_SUCCESS : LCF_ERROR_CUDA;
+  EncArgs a = enc_args(algo, d_in_shard, total_in_bytes);
+  a.first_chunk = first_chunk;
+  a.n_chunks = k;
+  a.stream_chunks = C;
+  a.table = static_cast<uint32_t*>(d_table_slice);
+  a.payload = static_cast<uint8_t*>(d_payload);
+  a.count_out = d_payload_bytes;
+  return enqueue_encode(ws, a);
+}
+
+lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,
+                              uint64_t total_payload_bytes, void* d_stream, void* stream_) {
+  if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!dtype_matches(algo, dtype)) return LCF_ERROR_DTYPE_MISMATCH;
+  if (!d_stream || !aligned16(d_stream) || total_in_bytes % word_bytes_of(algo)) return LCF_ERROR_INVALID_ARGUMENT;
+  const uint64_t C = lcf_num_chunks(algo, total_in_bytes);
+  const uint64_t base = round16(kHeaderBytes + 4 * C);
+  EncArgs a = enc_args(algo, nullptr, total_in_bytes);
+  a.stream_chunks = C;
+  a.header = reinterpret_cast<StreamHeader*>(d_stream);
+  a.pad_start = static_cast<uint8_t*>(d_stream) + kHeaderBytes + 4 * C;
+  a.pad_len = (uint32_t)(base - kHeaderBytes - 4 * C);
+  a.payload_total = total_payload_bytes;
+  launch_write_header(a, (cudaStream_t)stream_);
+  ++g_launches;
+  return last_launch_status();
+}
+
+}  // extern "C"

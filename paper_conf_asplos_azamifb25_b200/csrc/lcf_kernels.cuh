@@ -1,0 +1,125 @@
+// lcf_kernels.cuh — argument blocks and launchers of the codec kernels, plus
+// the per-chunk prologue/epilogue shared by all chunk kernels.
+#pragma once
+#include "lcf_internal.cuh"
+
+namespace lcf {
+
+__host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+
+// One compress launch covers chunks [first_chunk, first_chunk + n_chunks) of a
+// stream whose input has n_words_total words (FORMAT.md §2).
+struct EncArgs {
+  const void* in;           // words of chunk first_chunk (16-byte aligned)
+  uint64_t n_words_total;   // words of the whole stream input
+  uint64_t first_chunk;     // global index of this launch's chunk 0
+  uint64_t n_chunks;        // chunks in this launch (grid size)
+  uint32_t* table;          // size-table entries of this launch's chunks
+  uint8_t* payload;         // where this launch's chunk 0 payload goes
+  uint64_t* count_out;      // optional: device u64 ← payload bytes of the launch
+  StreamHeader* header;     // optional: full-stream mode writes the header
+  uint64_t stream_chunks;   // header n_chunks
+  uint64_t n_bytes;         // header n_bytes
+  uint64_t payload_total;   // header payload_bytes (lcf_write_header only)
+  uint32_t algo, word_bytes;
+  uint8_t* pad_start;       // optional zero pad between table and payload base
+  uint32_t pad_len;
+  // DPratio: FCM side inputs (per-word distance, 0 = no match)
+  const uint32_t* fcm_dist;
+};
+
+struct DecArgs {
+  const uint8_t* stream;  // 16-byte aligned
+  uint64_t stream_bytes;
+  uint8_t* out;           // 16-byte aligned
+  uint64_t out_capacity;
+  uint32_t algo, word_bytes;
+  uint32_t* tile_flag;    // DPratio: per-tile completion (epoch) flags
+};
+
+struct DecChunk {
+  uint64_t c;              // chunk index (DPratio: tile index)
+  uint64_t base;           // payload base offset in the stream
+  uint64_t payload_bytes;
+  uint64_t n_words;        // words of the whole output
+  uint64_t n_chunks;
+  uint32_t len, m, raw, ok;
+};
+
+__device__ __forceinline__ void finish_encode(const EncArgs& a, uint64_t total) {
+  if (a.count_out) *a.count_out = total;
+  if (a.header) {
+    uint32_t w[8];
+    w[0] = kMagic;
+    w[1] = kVersion | (a.algo << 8) | (a.word_bytes << 16);
+    w[2] = (uint32_t)a.n_bytes; w[3] = (uint32_t)(a.n_bytes >> 32);
+    w[4] = (uint32_t)a.stream_chunks; w[5] = (uint32_t)(a.stream_chunks >> 32);
+    w[6] = (uint32_t)total; w[7] = (uint32_t)(total >> 32);
+    uint4* h = reinterpret_cast<uint4*>(a.header);
+    h[0] = make_uint4(w[0], w[1], w[2], w[3]);
+    h[1] = make_uint4(w[4], w[5], w[6], w[7]);
+  }
+}
+
+// Reads and validates the stream header (FORMAT.md §1, §7). Returns false for
+// a malformed header; fills n_words/n_chunks/base/payload_bytes.
+__device__ __forceinline__ bool read_header(const DecArgs& a, const LaunchCtx& ctx, uint64_t& n_words,
+                                            uint64_t& n_chunks, uint64_t& base, uint64_t& payload) {
+  if (a.stream_bytes < kHeaderBytes) return false;
+  const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
+  const uint4 h1 = reinterpret_cast<const uint4*>(a.stream)[1];
+  const uint64_t n_bytes = ((uint64_t)h0.w << 32) | h0.z;
+  n_chunks = ((uint64_t)h1.y << 32) | h1.x;
+  payload = ((uint64_t)h1.w << 32) | h1.z;
+  if (h0.x != kMagic || (h0.y & 0xFF) != kVersion || ((h0.y >> 8) & 0xFF) != a.algo ||
+      ((h0.y >> 16) & 0xFF) != a.word_bytes || (h0.y >> 24) != 0)
+    return false;
+  if (n_bytes % a.word_bytes) return false;
+  n_words = n_bytes / a.word_bytes;
+  const uint64_t expect = a.algo == DPRATIO ? 2 * ((n_words + 2047) / 2048)
+                                            : (n_bytes + kChunkBytes - 1) / kChunkBytes;
+  if (n_chunks != expect) return false;
+  base = round16(kHeaderBytes + 4 * n_chunks);
+  if (base > a.stream_bytes || payload > a.stream_bytes - base) return false;
+  return true;
+}
+
+// Prologue of a speed/SPratio decode CTA (thread 0): ticket, header and size
+// entry validation, publication of the chunk's aggregate for the look-back.
+__device__ __forceinline__ DecChunk decode_chunk_begin(const DecArgs& a, const LaunchCtx& ctx,
+                                                       uint32_t wb, uint32_t CW) {
+  DecChunk d{};
+  d.c = atomicAdd(ctx.ticket, 1ull) - ctx.ticket_base;
+  uint64_t& n_chunks = d.n_chunks;
+  if (!read_header(a, ctx, d.n_words, n_chunks, d.base, d.payload_bytes)) {
+    if (d.c == 0) record_error(ctx, DERR_CORRUPT);
+    return d;
+  }
+  if (d.n_words * wb > a.out_capacity) {
+    if (d.c == 0) record_error(ctx, DERR_SMALL);
+    return d;
+  }
+  if (d.c >= n_chunks) return d;
+  const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[d.c];
+  d.len = e & ~kRawFlag;
+  d.raw = e >> 31;
+  d.m = (uint32_t)umin64(CW, d.n_words - d.c * CW);
+  const uint32_t raw_len = d.m * wb;
+  if (d.raw ? d.len != raw_len : d.len >= raw_len) {
+    record_error(ctx, DERR_CORRUPT);
+    lookback_publish(ctx, d.c, 0);
+    return d;
+  }
+  lookback_publish(ctx, d.c, round16(d.len));
+  d.ok = 1;
+  return d;
+}
+
+template <typename U> void launch_speed_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
+template <typename U>
+void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, unsigned grid, cudaStream_t st);
+void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
+void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, unsigned grid, cudaStream_t st);
+void launch_write_header(const EncArgs& a, cudaStream_t st);
+
+}  // namespace lcf

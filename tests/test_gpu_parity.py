@@ -1,0 +1,269 @@
+"""GPU parity: the sm_100a path (through the C ABI) vs the CPU oracle, bit-exact
+on streams, size tables and decompressed bits (-m gpu)."""
+import numpy as np
+import pytest
+
+import fmt_ref
+from paper_conf_asplos_azamifb25_b200 import datagen
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+SPEED_ALGOS = ["SPspeed", "DPspeed"]
+GPU_ALGOS = ["SPspeed", "DPspeed", "SPratio", "DPratio"]
+
+
+@pytest.fixture(scope="module")
+def L():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_asplos_azamifb25_b200 import lcf
+    lcf.lib()
+    return lcf
+
+
+def wdt(algo):
+    return np.uint32 if algo.startswith("SP") else np.uint64
+
+
+def tdt(algo):
+    return torch.int32 if algo.startswith("SP") else torch.int64
+
+
+def to_dev(words: np.ndarray):
+    t = torch.from_numpy(words.view(np.int32 if words.dtype == np.uint32 else np.int64).copy())
+    return t.cuda()
+
+
+def gpu_roundtrip(L, algo, x_dev):
+    s = L.compress(algo, x_dev)
+    y = L.decompress(algo, s)
+    torch.cuda.synchronize()
+    return s.cpu().numpy().tobytes(), y
+
+
+def check_parity(L, orc, algo, words: np.ndarray, name=""):
+    x = to_dev(words)
+    s_gpu, y = gpu_roundtrip(L, algo, x)
+    s_orc = orc.compress(algo, words)
+    if s_gpu != s_orc:
+        h1, t1, c1 = fmt_ref.parse_stream(s_gpu)
+        h2, t2, c2 = fmt_ref.parse_stream(s_orc)
+        bad = [i for i in range(min(len(t1), len(t2))) if t1[i] != t2[i] or c1[i] != c2[i]]
+        raise AssertionError(f"{algo}/{name}: stream differs (len {len(s_gpu)} vs {len(s_orc)}; "
+                             f"headers {h1 == h2}; first bad chunk {bad[:5]})")
+    assert torch.equal(y, x), f"{algo}/{name}: decompressed bits differ"
+    # cross-decode: oracle decodes the GPU stream (identical bytes) and GPU decodes oracle's
+    assert np.array_equal(orc.decompress(algo, s_gpu), words)
+    return len(s_gpu)
+
+
+def algos_available(L):
+    avail = []
+    for a in GPU_ALGOS:
+        try:
+            x = torch.zeros(16, dtype=tdt(a), device="cuda")
+            L.compress(a, x)
+            avail.append(a)
+        except L.LcfError:
+            pass
+    return avail
+
+
+@pytest.mark.parametrize("algo", GPU_ALGOS)
+def test_adversarial_parity(L, orc, algo):
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    for name, words in datagen.adversarial(32 if algo.startswith("SP") else 64):
+        check_parity(L, orc, algo, words, name)
+
+
+@pytest.mark.parametrize("algo", GPU_ALGOS)
+def test_exhaustive_tiny_parity(L, orc, algo):
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    sp = datagen.F32_SPECIALS if algo.startswith("SP") else datagen.F64_SPECIALS
+    rng = np.random.default_rng(0)
+    for r in (1, 2, 3):
+        for _ in range(60):
+            check_parity(L, orc, algo, sp[rng.integers(0, 16, r)], f"tiny{r}")
+
+
+@pytest.mark.parametrize("algo", GPU_ALGOS)
+def test_random_width_subchunks(L, orc, algo):
+    """Every MPLG width 0..W (both flag states) and ragged tails."""
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    W = 32 if algo.startswith("SP") else 64
+    dt = wdt(algo)
+    rng = np.random.default_rng(W)
+    SW = 4096 // W
+    CW = 32 * SW
+    for n in (CW * 3 + 1035, SW * 7 + 5, CW):
+        u = np.zeros(n, dtype=dt)  # the DIFFMS output we want the encoder to see
+        for s in range(-(-n // SW)):
+            w = int(rng.integers(0, W + 1))
+            m = min(SW, n - s * SW)
+            vals = rng.integers(0, 2**W - 1, size=m, dtype=dt, endpoint=True)
+            u[s * SW:s * SW + m] = vals & dt((1 << w) - 1) if w < W else vals
+        d = (u >> dt(1)) ^ (dt(0) - (u & dt(1)))  # magnitude-sign → two's complement
+        words = np.concatenate([np.cumsum(d[c:c + CW], dtype=dt) for c in range(0, n, CW)])
+        check_parity(L, orc, algo, words, f"widths{n}")
+
+
+CONFIG_CASES = [("SPspeed", "tiny_512x512_f32", "f"), ("SPratio", "tiny_512x512_f32", "f"),
+                ("SPspeed", "cesm_1800x3600_f32", "T"), ("SPspeed", "cesm_1800x3600_f32", "U"),
+                ("SPratio", "cesm_1800x3600_f32", "T"), ("SPratio", "cesm_1800x3600_f32", "U")]
+
+
+@pytest.mark.parametrize("algo,config,field", CONFIG_CASES)
+def test_config_field_parity(L, orc, algo, config, field):
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    x = datagen.field(config, field, device="cuda")
+    words = x.cpu().numpy().view(wdt(algo))
+    n = check_parity(L, orc, algo, words, f"{config}/{field}")
+    assert n < words.nbytes  # these smooth fields compress
+
+
+@pytest.mark.parametrize("algo,field", [("DPspeed", "density"), ("DPspeed", "velocity"),
+                                        ("DPratio", "density"), ("DPratio", "velocity")])
+def test_miranda_subvolume_parity(L, orc, algo, field):
+    """Miranda-shaped f64 (a 32×384×384 slab of the full field, 4.7 M words)."""
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    x = datagen.field("miranda_256x384x384_f64", field, device="cuda", origin=(0, 0, 0), shape=(32, 384, 384))
+    check_parity(L, orc, algo, x.cpu().numpy().view(np.uint64), f"miranda/{field}")
+
+
+def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
+    """Full-size check: GPU stream vs oracle on a sample of chunks (compress_chunks)."""
+    s = L.compress(algo, x_dev)
+    stream = s.cpu().numpy().tobytes()
+    words = x_dev.cpu().numpy().view(wdt(algo))
+    h, table, chunks = fmt_ref.parse_stream(stream)
+    C = len(table)
+    rng = np.random.default_rng(seed)
+    picks = sorted(set([0, C - 1] + rng.integers(0, C, n_samples).tolist()))
+    for c in picks:
+        tab, pay = orc.compress_chunks(algo, words, c, 1)
+        assert tab[0] == table[c], (c, tab[0], table[c])
+        assert pay[:tab[0] & 0x7FFFFFFF] == chunks[c][1], c
+    y = L.decompress(algo, s)
+    assert torch.equal(y, x_dev)
+    return len(stream)
+
+
+@pytest.mark.parametrize("algo,config,field", [
+    ("SPspeed", "nyx_512x512x512_f32", "baryon_density"), ("SPspeed", "nyx_512x512x512_f32", "velocity"),
+    ("SPspeed", "hacc_280953867_f32", "xx"), ("SPratio", "nyx_512x512x512_f32", "velocity"),
+    ("SPratio", "hacc_280953867_f32", "vx"), ("DPspeed", "miranda_256x384x384_f64", "density")])
+def test_full_size_sampled_parity(L, orc, algo, config, field):
+    if algo not in algos_available(L):
+        pytest.skip(f"{algo} not built")
+    x = datagen.field(config, field, device="cuda")
+    x = x.view(tdt(algo))
+    sampled_chunk_parity(L, orc, algo, x)
+    del x
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("algo", SPEED_ALGOS)
+def test_async_path_and_corruption(L, orc, algo):
+    words = datagen.smooth_1d(3 * 4096 + 77, np.float32 if algo == "SPspeed" else np.float64, seed=3)
+    words = words.view(wdt(algo))
+    x = to_dev(words)
+    s = L.compress(algo, x)
+    out = torch.empty_like(x)
+    # async: no out_bytes, then check
+    L.lcf_decompress(algo, None, s, s.numel(), out, out.numel() * out.element_size(), sync=False)
+    L.lcf_check_stream()
+    assert torch.equal(out, x)
+    # header corruption → CORRUPT_STREAM, both sync and async
+    for off, val in [(0, 0), (6, 3), (16, 99), (24, 255)]:
+        t = s.clone()
+        t[off] = val
+        with pytest.raises(L.LcfError) as e:
+            L.lcf_decompress(algo, None, t, t.numel(), out, out.numel() * out.element_size())
+        assert e.value.status == 4
+        L.lcf_decompress(algo, None, t, t.numel(), out, out.numel() * out.element_size(), sync=False)
+        with pytest.raises(L.LcfError):
+            L.lcf_check_stream()
+    # size-table corruption: reject, never crash; random payload bytes: no crash
+    t = s.clone()
+    t[32 + 3] = 0x7F
+    with pytest.raises(L.LcfError):
+        L.lcf_decompress(algo, None, t, t.numel(), out, out.numel() * out.element_size())
+    rng = np.random.default_rng(1)
+    for _ in range(50):
+        t = s.clone()
+        pos = int(rng.integers(32, s.numel()))
+        t[pos] = int(rng.integers(0, 256))
+        try:
+            L.lcf_decompress(algo, None, t, t.numel(), out, out.numel() * out.element_size())
+            ok_gpu = True
+        except L.LcfError:
+            ok_gpu = False
+        ok_orc = orc.decompress_status(algo, t.cpu().numpy().tobytes()) == 0
+        assert ok_gpu == ok_orc
+    # too small an output buffer
+    with pytest.raises(L.LcfError) as e:
+        L.lcf_decompress(algo, None, s, s.numel(), out, 100)
+    assert e.value.status == 3
+    torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("algo", SPEED_ALGOS)
+def test_concurrent_streams_and_repeats(L, orc, algo):
+    """Different streams get separate workspaces; repeated calls stay exact."""
+    dt = np.float32 if algo == "SPspeed" else np.float64
+    xs = [to_dev(datagen.smooth_1d(50 * 4096 // (1 if dt == np.float32 else 2) + i, dt, seed=i).view(wdt(algo)))
+          for i in range(3)]
+    expect = [orc.compress(algo, x.cpu().numpy().view(wdt(algo))) for x in xs]
+    streams = [torch.cuda.Stream() for _ in xs]
+    for rep in range(5):
+        outs = []
+        for x, st in zip(xs, streams):
+            with torch.cuda.stream(st):
+                cap = L.lcf_max_compressed_size(algo, None, x.numel() * x.element_size())
+                o = torch.empty(cap, dtype=torch.uint8, device="cuda")
+                L.lcf_compress(algo, None, x, x.numel() * x.element_size(), o, cap, sync=False, stream=st)
+                outs.append(o)
+        torch.cuda.synchronize()
+        for o, e in zip(outs, expect):
+            assert o[:len(e)].cpu().numpy().tobytes() == e
+
+
+def test_empty_and_info(L, orc):
+    for algo in ["SPspeed", "DPspeed"]:
+        x = torch.zeros(0, dtype=tdt(algo), device="cuda")
+        s = L.compress(algo, x)
+        assert s.cpu().numpy().tobytes() == orc.compress(algo, np.zeros(0, wdt(algo)))
+        info = L.lcf_get_info(s, s.numel())
+        assert info["uncompressed_bytes"] == 0 and info["compressed_bytes"] == 32
+        assert L.decompress(algo, s).numel() == 0
+
+
+def test_host_buffer_api(L, orc):
+    words = datagen.smooth_1d(10 * 4096 + 3, np.float32, seed=8).view(np.uint32)
+    cap = L.lcf_max_compressed_size("SPspeed", None, words.nbytes)
+    hout = np.zeros(cap, np.uint8)
+    n = L.lcf_compress_host("SPspeed", None, words, words.nbytes, hout, cap)
+    assert hout[:n].tobytes() == orc.compress("SPspeed", words)
+    back = np.zeros_like(words)
+    m = L.lcf_decompress_host("SPspeed", None, hout, n, back, back.nbytes)
+    assert m == words.nbytes and np.array_equal(back, words)
+
+
+def test_dtype_and_argument_errors(L):
+    x = torch.zeros(100, dtype=torch.int32, device="cuda")
+    o = torch.empty(10000, dtype=torch.uint8, device="cuda")
+    with pytest.raises(L.LcfError) as e:
+        L.lcf_compress("SPspeed", "float64", x, 400, o, 10000)
+    assert e.value.status == 2
+    with pytest.raises(L.LcfError) as e:
+        L.lcf_compress("SPspeed", "float32", x, 402, o, 10000)
+    assert e.value.status == 1
+    with pytest.raises(L.LcfError) as e:
+        L.lcf_compress("SPspeed", "float32", x, 400, o, 100)
+    assert e.value.status == 3

@@ -20,8 +20,7 @@ struct Workspace {
   int device = -1;
   cudaStream_t stream = nullptr;
   std::mutex mu;
-  unsigned long long* ticket = nullptr;  // device counter, never reset
-  unsigned long long ticket_next = 0;    // host mirror: tickets handed out so far
+  unsigned long long* ticket = nullptr;  // [0] ticket counter, [1] retired CTAs (kernels reset both)
   uint64_t* status = nullptr;            // look-back status words
   size_t status_cap = 0;
   uint32_t* tile_flag = nullptr;         // DPratio decode tile completion flags
@@ -49,9 +48,9 @@ Workspace* get_ws(cudaStream_t stream, lcf_status_t* st) {
   Workspace* ws = new Workspace();
   ws->device = dev;
   ws->stream = stream;
-  if (!cuda_ok(cudaMalloc(&ws->ticket, sizeof(unsigned long long))) ||
+  if (!cuda_ok(cudaMalloc(&ws->ticket, 2 * sizeof(unsigned long long))) ||
       !cuda_ok(cudaMalloc(&ws->err, sizeof(uint32_t))) ||
-      !cuda_ok(cudaMemsetAsync(ws->ticket, 0, sizeof(unsigned long long), stream)) ||
+      !cuda_ok(cudaMemsetAsync(ws->ticket, 0, 2 * sizeof(unsigned long long), stream)) ||
       !cuda_ok(cudaMemsetAsync(ws->err, 0, sizeof(uint32_t), stream))) {
     *st = LCF_ERROR_OUT_OF_MEMORY;
     delete ws;
@@ -88,14 +87,12 @@ uint32_t next_epoch(Workspace* ws) {
   return ws->epoch;
 }
 
-LaunchCtx make_ctx(Workspace* ws, uint64_t grid) {
+LaunchCtx make_ctx(Workspace* ws) {
   LaunchCtx c;
   c.ticket = ws->ticket;
-  c.ticket_base = ws->ticket_next;
   c.status = ws->status;
   c.epoch = next_epoch(ws);
   c.err = ws->err;
-  ws->ticket_next += grid;
   return c;
 }
 
@@ -159,7 +156,7 @@ EncArgs enc_args(int algo, const void* in, uint64_t in_bytes) {
 
 lcf_status_t enqueue_encode(Workspace* ws, EncArgs& a) {
   if (lcf_status_t s = grow(ws->status, ws->status_cap, a.n_chunks, ws->stream, true)) return s;
-  LaunchCtx ctx = make_ctx(ws, a.n_chunks);
+  LaunchCtx ctx = make_ctx(ws);
   switch (a.algo) {
     case LCF_SPSPEED: launch_speed_encode<uint32_t>(a, ctx, ws->stream); break;
     case LCF_DPSPEED: launch_speed_encode<uint64_t>(a, ctx, ws->stream); break;
@@ -273,17 +270,20 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   a.out_capacity = out_capacity;
   a.algo = (uint32_t)algo;
   a.word_bytes = word_bytes_of(algo);
-  const uint32_t before = ws->epoch;
-  LaunchCtx ctx = make_ctx(ws, grid);
+  LaunchCtx ctx = make_ctx(ws);
   switch (algo) {
-    case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, (unsigned)grid, stream); break;
-    case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, (unsigned)grid, stream); break;
+    case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, grid, stream); break;
+    case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, grid, stream); break;
     default: return LCF_ERROR_INVALID_ARGUMENT;
   }
   ++g_launches;
   if ((st = last_launch_status())) return st;
   if (out_bytes) {
-    if ((st = device_error_since(ws, ctx.epoch < before ? 0 : before))) return st;
+    // a synchronising call reports any device-found failure since the last
+    // report on this stream (include/lcf.h), its own included
+    st = device_error_since(ws, ws->checked_epoch);
+    ws->checked_epoch = ws->epoch;
+    if (st) return st;
     *out_bytes = n_bytes;
   }
   return LCF_SUCCESS;

@@ -32,8 +32,7 @@ static_assert(sizeof(StreamHeader) == 32, "header layout");
 
 // ---- launch context shared by all chunk kernels ----------------------------
 struct LaunchCtx {
-  unsigned long long* ticket;  // monotonically increasing ticket counter
-  unsigned long long ticket_base;
+  unsigned long long* ticket;  // [0] tickets handed out, [1] retired CTAs (reset by the last)
   uint64_t* status;            // look-back status words, one per chunk
   uint32_t epoch;              // 1 .. 2^22-1, unique per launch between resets
   uint32_t* err;               // device error word

@@ -84,42 +84,27 @@ __device__ __forceinline__ bool read_header(const DecArgs& a, const LaunchCtx& c
   return true;
 }
 
-// Prologue of a speed/SPratio decode CTA (thread 0): ticket, header and size
-// entry validation, publication of the chunk's aggregate for the look-back.
-__device__ __forceinline__ DecChunk decode_chunk_begin(const DecArgs& a, const LaunchCtx& ctx,
-                                                       uint32_t wb, uint32_t CW) {
-  DecChunk d{};
-  d.c = atomicAdd(ctx.ticket, 1ull) - ctx.ticket_base;
-  uint64_t& n_chunks = d.n_chunks;
-  if (!read_header(a, ctx, d.n_words, n_chunks, d.base, d.payload_bytes)) {
-    if (d.c == 0) record_error(ctx, DERR_CORRUPT);
-    return d;
+// Grid of a persistent kernel: every SM filled to its occupancy, capped by the
+// amount of work.
+template <typename Kern> int persistent_grid(Kern kernel, int threads, size_t smem, uint64_t work) {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   }
-  if (d.n_words * wb > a.out_capacity) {
-    if (d.c == 0) record_error(ctx, DERR_SMALL);
-    return d;
-  }
-  if (d.c >= n_chunks) return d;
-  const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[d.c];
-  d.len = e & ~kRawFlag;
-  d.raw = e >> 31;
-  d.m = (uint32_t)umin64(CW, d.n_words - d.c * CW);
-  const uint32_t raw_len = d.m * wb;
-  if (d.raw ? d.len != raw_len : d.len >= raw_len) {
-    record_error(ctx, DERR_CORRUPT);
-    lookback_publish(ctx, d.c, 0);
-    return d;
-  }
-  lookback_publish(ctx, d.c, round16(d.len));
-  d.ok = 1;
-  return d;
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem);
+  if (per_sm < 1) per_sm = 1;
+  const uint64_t g = (uint64_t)sms * per_sm;
+  return (int)(work < g ? (work ? work : 1) : g);
 }
 
 template <typename U> void launch_speed_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
 template <typename U>
-void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, unsigned grid, cudaStream_t st);
+void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st);
 void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
-void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, unsigned grid, cudaStream_t st);
+void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st);
 void launch_write_header(const EncArgs& a, cudaStream_t st);
 
 }  // namespace lcf

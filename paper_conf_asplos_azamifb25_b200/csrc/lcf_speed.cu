@@ -1,26 +1,39 @@
 // lcf_speed.cu — SPspeed / DPspeed (§3.1) on sm_100a.
 //
-// One 256-thread CTA per 16 KiB chunk (L104), chunk index from a ticket so the
-// decoupled look-back (L122) only waits on CTAs that already run. Warp w owns
-// subchunks 4w..4w+3 (512 B each, L118): one coalesced 16-byte load per lane
-// per subchunk, so a lane holds K = 4 (f32) or 2 (f64) consecutive words.
+// Persistent, warp-specialised CTAs; chunks (16 KiB, L104) are handed out by a
+// global ticket so the decoupled look-back (L122) only ever waits on chunks
+// that running CTAs already own.
 //
-// Encode: DIFFMS in registers (neighbour word by shuffle) → per-subchunk width
-// by a warp max-reduction of bit lengths → TCMS retry if the maximum has no
-// leading zero (L114) → the chunk size is known before any packing, so the
-// aggregate is published at once → lanes emit their K·w-bit strings into the
-// shared-memory output buffer (lcf::emit_bits_warp) while warp 0 resolves the
-// look-back → coalesced 16-byte stores at the resolved offset.
-// Decode: the size-table entry gives the aggregate immediately → look-back →
-// 16-byte loads of the payload into shared memory → each lane funnel-shifts
-// its K fields out → unTCMS → DIFFMS⁻¹ as a block-wide prefix sum (L132).
+// Encode CTA (320 threads):
+//   warp 0  loader : ticket → 1-D TMA bulk load of the chunk into a 3-stage
+//                    shared-memory ring (mbarrier complete_tx)
+//   warp 1  storer : decoupled look-back for the chunk's output offset →
+//                    1-D TMA bulk store of the packed chunk → size-table entry
+//   warps 2-9      : DIFFMS in registers (L110–112) → per-subchunk width by a
+//                    warp OR-reduction (bitlen(max) = bitlen(OR)) with the TCMS
+//                    retry (L114) → aggregate published as soon as the size is
+//                    known → bit packing (L116) into a 2-slot output ring.
+// Decode CTA (288 threads):
+//   warp 0  loader : ticket → size entry → aggregate published at once →
+//                    look-back → TMA bulk load of the payload (4 stages)
+//   warps 1-8      : unpack (funnel shifts) → unTCMS → DIFFMS⁻¹ as a CTA-wide
+//                    prefix sum (L132) → 16-byte coalesced stores.
+// Each compute warp owns subchunks 4w..4w+3 (512 B, L118); a lane holds K = 4
+// (f32) or 2 (f64) consecutive words of each.
 #include "lcf_kernels.cuh"
+#include "lcf_pipe.cuh"
 
 namespace lcf {
 
 namespace {
 
-constexpr int kThreads = 256, kWarps = 8, kSubPerWarp = 4;
+constexpr int kCompWarps = 8, kSubPerWarp = 4;
+constexpr int kEncStages = 3, kEncOut = 2, kDecStages = 4;
+constexpr int kEncThreads = (2 + kCompWarps) * 32;
+constexpr int kDecThreads = (1 + kCompWarps) * 32;
+constexpr uint32_t kCompThreads = kCompWarps * 32;
+constexpr uint64_t kNoChunk = ~0ull;
+constexpr uint32_t kBarCompute = 1;  // named barrier of the compute warps
 
 template <typename U> struct Cfg {
   static constexpr int W = 8 * sizeof(U);
@@ -29,7 +42,24 @@ template <typename U> struct Cfg {
   static constexpr int K = SW / 32;             // words per lane per subchunk
 };
 
-// K consecutive words of one lane <-> one 16-byte vector
+struct EncSmem {
+  alignas(128) uint32_t in[kEncStages][kChunkBytes / 4];
+  alignas(128) uint32_t out[kEncOut][(kChunkBytes + 64) / 4];
+  uint64_t full_in[kEncStages], empty_in[kEncStages], full_out[kEncOut], empty_out[kEncOut];
+  uint64_t in_chunk[kEncStages], out_chunk[kEncOut];
+  uint32_t out_len[kEncOut], out_raw[kEncOut];
+  uint32_t hdr[kEncOut][32];
+};
+
+template <typename U> struct DecSmem {
+  alignas(128) uint32_t in[kDecStages][(kChunkBytes + 64) / 4];
+  uint64_t full_in[kDecStages], empty_in[kDecStages];
+  uint64_t chunk[kDecStages];
+  uint32_t len[kDecStages], flags[kDecStages];  // flags: bit0 raw, bit1 bad
+  U wtot[2][kCompWarps];
+};
+
+// ---- word <-> 16-byte vector --------------------------------------------------
 template <typename U> __device__ __forceinline__ void unpack16(const uint4& q, U* v);
 template <> __device__ __forceinline__ void unpack16<uint32_t>(const uint4& q, uint32_t* v) {
   v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w;
@@ -46,343 +76,538 @@ template <> __device__ __forceinline__ uint4 pack16<uint64_t>(const uint64_t* v)
   return make_uint4((uint32_t)v[0], (uint32_t)(v[0] >> 32), (uint32_t)v[1], (uint32_t)(v[1] >> 32));
 }
 
-// Lane string of K fields of width w (K·w ≤ 128 bits) as a 128-bit value.
-__device__ __forceinline__ void make_string(const uint32_t* v, unsigned w, uint64_t& lo, uint64_t& hi) {
-  const uint64_t a = (uint64_t)v[0] | ((uint64_t)v[1] << w);  // 2w bits
-  const uint64_t b = (uint64_t)v[2] | ((uint64_t)v[3] << w);
-  const unsigned s = 2 * w;
-  if (s == 64) { lo = a; hi = b; }
-  else if (s == 0) { lo = 0; hi = 0; }
-  else { lo = a | (b << s); hi = b >> (64 - s); }
+// ---- MPLG width: bitlen(max) == bitlen(OR) over the subchunk --------------------
+__device__ __forceinline__ uint32_t warp_width(const uint32_t* v) {
+  const uint32_t o = __reduce_or_sync(0xFFFFFFFFu, v[0] | v[1] | v[2] | v[3]);
+  return 32 - __clz(o);
 }
-__device__ __forceinline__ void make_string(const uint64_t* v, unsigned w, uint64_t& lo, uint64_t& hi) {
+__device__ __forceinline__ uint32_t warp_width(const uint64_t* v) {
+  const uint64_t x = v[0] | v[1];
+  const uint32_t hi = __reduce_or_sync(0xFFFFFFFFu, (uint32_t)(x >> 32));
+  const uint32_t lo = __reduce_or_sync(0xFFFFFFFFu, (uint32_t)x);
+  return hi ? 64 - __clz(hi) : 32 - __clz(lo);
+}
+
+// ---- a lane's K fields of width w as one bit string (4 words, ≤ 128 bits) -------
+__device__ __forceinline__ void make_string(const uint32_t* v, uint32_t w, uint32_t* S) {
+  const uint32_t a_lo = v[0] | shl_c(v[1], w), a_hi = __funnelshift_lc(v[1], 0u, w);
+  const uint32_t b_lo = v[2] | shl_c(v[3], w), b_hi = __funnelshift_lc(v[3], 0u, w);
+  if (w >= 16) {  // b goes to bit 2w ≥ 32
+    const uint32_t t = 2 * w - 32;
+    S[0] = a_lo;
+    S[1] = a_hi | shl_c(b_lo, t);
+    S[2] = __funnelshift_lc(b_lo, b_hi, t);
+    S[3] = __funnelshift_lc(b_hi, 0u, t);
+  } else {
+    const uint32_t t = 2 * w;
+    S[0] = a_lo | shl_c(b_lo, t);
+    S[1] = a_hi | __funnelshift_lc(b_lo, b_hi, t);
+    S[2] = __funnelshift_lc(b_hi, 0u, t);
+    S[3] = 0;
+  }
+}
+__device__ __forceinline__ void make_string(const uint64_t* v, uint32_t w, uint32_t* S) {
+  uint64_t lo, hi;
   if (w == 64) { lo = v[0]; hi = v[1]; }
   else if (w == 0) { lo = 0; hi = 0; }
   else { lo = v[0] | (v[1] << w); hi = v[1] >> (64 - w); }
+  S[0] = (uint32_t)lo; S[1] = (uint32_t)(lo >> 32); S[2] = (uint32_t)hi; S[3] = (uint32_t)(hi >> 32);
 }
-__device__ __forceinline__ void split_string(uint64_t lo, uint64_t hi, unsigned w, uint32_t* v) {
+
+// Lanes' strings of equal length L = K·w ≥ 32 bits, lane l at bit l·L of the
+// word-aligned subchunk stream `buf`: every word is shared by ≤ 2 lanes, so one
+// shuffle hands the partial last word to the next lane. Every word of the
+// stream is written exactly once.
+__device__ __forceinline__ void emit_equal(uint32_t* buf, uint32_t lane, uint32_t L, const uint32_t* S) {
+  const uint32_t P = lane * L, F = P >> 5, r = P & 31;
+  uint32_t T[5];
+  T[0] = S[0] << r;
+  T[1] = __funnelshift_l(S[0], S[1], r);
+  T[2] = __funnelshift_l(S[1], S[2], r);
+  T[3] = __funnelshift_l(S[2], S[3], r);
+  T[4] = __funnelshift_l(S[3], 0u, r);
+  const uint32_t e = (r + L - 1) >> 5;  // index of the last word touched (0..4)
+  const uint32_t last = e == 1 ? T[1] : e == 2 ? T[2] : e == 3 ? T[3] : e == 4 ? T[4] : T[0];
+  const uint32_t in = __shfl_up_sync(0xFFFFFFFFu, last, 1);
+  if (r) T[0] |= in;
+  const bool keep_last = ((r + L) & 31) == 0 || lane == 31;
+#pragma unroll
+  for (uint32_t j = 0; j < 5; ++j)
+    if (j < e || (j == e && keep_last)) buf[F + j] = T[j];
+}
+
+// ---- shared-memory field extraction (decode) ------------------------------------
+__device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uint32_t* v) {
   const uint32_t m = w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u);
-  v[0] = (uint32_t)lo & m;
-  v[1] = (uint32_t)(w >= 64 ? 0 : (lo >> w)) & m;
-  uint64_t l2 = lo, h2 = hi;
-  shr128(l2, h2, 2 * w);
-  v[2] = (uint32_t)l2 & m;
-  v[3] = (uint32_t)(w >= 64 ? 0 : (l2 >> w)) & m;
-  if (w == 0) v[0] = v[1] = v[2] = v[3] = 0;
+  v[0] = U4[0] & m;
+  v[1] = __funnelshift_rc(U4[0], U4[1], w) & m;
+  uint32_t lo, hi, s;
+  if (w >= 16) { lo = U4[1]; hi = U4[2]; s = 2 * w - 32; }
+  else { lo = U4[0]; hi = U4[1]; s = 2 * w; }
+  v[2] = __funnelshift_rc(lo, hi, s) & m;
+  const uint32_t p3 = 3 * w, i3 = p3 >> 5, s3 = p3 & 31;
+  const uint32_t x0 = i3 == 0 ? U4[0] : i3 == 1 ? U4[1] : i3 == 2 ? U4[2] : U4[3];
+  const uint32_t x1 = i3 == 0 ? U4[1] : i3 == 1 ? U4[2] : U4[3];
+  v[3] = __funnelshift_r(x0, x1, s3) & m;
 }
-__device__ __forceinline__ void split_string(uint64_t lo, uint64_t hi, unsigned w, uint64_t* v) {
+__device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uint64_t* v) {
+  const uint64_t lo = (uint64_t)U4[0] | ((uint64_t)U4[1] << 32), hi = (uint64_t)U4[2] | ((uint64_t)U4[3] << 32);
   const uint64_t m = mask64(w);
   v[0] = lo & m;
   uint64_t l2 = lo, h2 = hi;
   shr128(l2, h2, w);
   v[1] = l2 & m;
-  if (w == 0) v[0] = v[1] = 0;
 }
 
 template <typename U> __device__ __forceinline__ U shfl_up1(U v) { return __shfl_up_sync(0xFFFFFFFFu, v, 1); }
 template <typename U> __device__ __forceinline__ U shfl_idx(U v, int l) { return __shfl_sync(0xFFFFFFFFu, v, l); }
 
+__device__ __forceinline__ uint32_t chunk_words(uint64_t n_words_total, uint64_t gc, uint32_t CW) {
+  return (uint32_t)umin64((uint64_t)CW, n_words_total - gc * CW);
+}
+
+// Ticket dispenser shared by the persistent kernels: ticket[0] counts handed
+// out tickets, ticket[1] counts CTAs that drew their final (failing) ticket;
+// the last one resets both for the next launch on the stream.
+__device__ __forceinline__ void ticket_retire(const LaunchCtx& ctx) {
+  if (atomicAdd(ctx.ticket + 1, 1ull) == gridDim.x - 1) {
+    ctx.ticket[0] = 0;
+    ctx.ticket[1] = 0;
+  }
+}
+
+// =================================== encode ======================================
 template <typename U>
-__global__ void __launch_bounds__(kThreads) speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t cw,
+                                            uint32_t lane) {
   using C = Cfg<U>;
   constexpr int W = C::W, CW = C::CW, SW = C::SW, K = C::K;
-  __shared__ __align__(16) uint32_t s_out[(kChunkBytes + 64) / 4];
-  __shared__ uint32_t s_subbytes[32], s_suboff[32];
-  __shared__ uint64_t s_c, s_excl;
-  __shared__ uint32_t s_len, s_raw;
-
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_c = atomicAdd(ctx.ticket, 1ull) - ctx.ticket_base;
-  __syncthreads();
-  const uint64_t c = s_c;
-  const uint64_t gc = a.first_chunk + c;
-  const uint32_t m = (uint32_t)umin64((uint64_t)CW, a.n_words_total - gc * CW);
-  const U* src = reinterpret_cast<const U*>(a.in) + c * CW;
-
-  // ---- load (16 B per lane per subchunk) and DIFFMS (L110–112) ----
-  U v[kSubPerWarp][K];
-#pragma unroll
-  for (int q = 0; q < kSubPerWarp; ++q) {
-    const uint32_t i0 = (warp * kSubPerWarp + q) * SW + lane * K;
-    if (i0 + K <= m) {
-      unpack16<U>(__ldcs(reinterpret_cast<const uint4*>(src + i0)), v[q]);
-    } else {
-#pragma unroll
-      for (int j = 0; j < K; ++j) v[q][j] = (i0 + j < m) ? src[i0 + j] : (U)0;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kEncStages, ph = (it / kEncStages) & 1;
+    const uint32_t o = it % kEncOut, pho = (it / kEncOut) & 1;
+    mbar_wait(&S.full_in[s], ph);
+    const uint64_t t = S.in_chunk[s];
+    if (t == kNoChunk) {  // forward the end marker to the storer
+      mbar_wait(&S.empty_out[o], pho ^ 1);
+      if (cw == 0 && lane == 0) S.out_chunk[o] = kNoChunk;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.full_out[o]);
+      return;
     }
-  }
-  const uint32_t wfirst = warp * kSubPerWarp * SW;
-  U carry = (warp > 0 && wfirst - 1 < m) ? src[wfirst - 1] : (U)0;
-  uint32_t wq[kSubPerWarp];
+    const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, CW);
+    const bool full = m == (uint32_t)CW;
+    const U* in = reinterpret_cast<const U*>(S.in[s]);
+    U v[kSubPerWarp][K];
 #pragma unroll
-  for (int q = 0; q < kSubPerWarp; ++q) {
-    const U next_carry = shfl_idx(v[q][K - 1], 31);
-    U p = shfl_up1(v[q][K - 1]);
-    if (lane == 0) p = carry;
-    carry = next_carry;
-    const uint32_t i0 = (warp * kSubPerWarp + q) * SW + lane * K;
+    for (int q = 0; q < kSubPerWarp; ++q)
+      unpack16<U>(reinterpret_cast<const uint4*>(in)[(cw * kSubPerWarp + q) * 32 + lane], v[q]);
+    const uint32_t wfirst = cw * kSubPerWarp * SW;
+    U carry = (cw > 0 && wfirst - 1 < m) ? in[wfirst - 1] : (U)0;
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[s]);  // stage consumed (raw chunks re-read global)
+
+    // DIFFMS (L110–112) and MPLG widths with the TCMS retry (L114–118)
+    uint32_t wq[kSubPerWarp];
 #pragma unroll
-    for (int j = K - 1; j >= 0; --j) {
-      const U prev = j ? v[q][j - 1] : p;
-      v[q][j] = (i0 + j < m) ? tcms((U)(v[q][j] - prev)) : (U)0;
-    }
-    // ---- MPLG width per subchunk (L114–118) ----
-    int bl = 0;
+    for (int q = 0; q < kSubPerWarp; ++q) {
+      const U next_carry = shfl_idx(v[q][K - 1], 31);
+      U p = shfl_up1(v[q][K - 1]);
+      if (lane == 0) p = carry;
+      carry = next_carry;
+      const uint32_t i0 = (cw * kSubPerWarp + q) * SW + lane * K;
 #pragma unroll
-    for (int j = 0; j < K; ++j) bl = max(bl, bitlen(v[q][j]));
-    int wmax = (int)__reduce_max_sync(0xFFFFFFFFu, (unsigned)bl);
-    uint32_t flag = 0;
-    if (wmax == W) {  // maximum has no leading zero: TCMS once more
-      flag = 1;
-      bl = 0;
-#pragma unroll
-      for (int j = 0; j < K; ++j) {
-        v[q][j] = tcms(v[q][j]);
-        bl = max(bl, bitlen(v[q][j]));
+      for (int j = K - 1; j >= 0; --j) {
+        const U prev = j ? v[q][j - 1] : p;
+        const U u = tcms((U)(v[q][j] - prev));
+        v[q][j] = (full || i0 + j < m) ? u : (U)0;
       }
-      wmax = (int)__reduce_max_sync(0xFFFFFFFFu, (unsigned)bl);
+      uint32_t w = warp_width(v[q]);
+      uint32_t flag = 0;
+      if (w == (uint32_t)W) {
+        flag = 1;
+#pragma unroll
+        for (int j = 0; j < K; ++j) v[q][j] = tcms(v[q][j]);
+        w = warp_width(v[q]);
+      }
+      wq[q] = w | (flag << 7);
     }
-    wq[q] = (uint32_t)wmax | (flag << 7);
-    if (lane == 0) {
-      const int s = warp * kSubPerWarp + q;
-      const int64_t rem = (int64_t)m - (int64_t)s * SW;
-      const uint32_t ms = rem <= 0 ? 0u : (uint32_t)(rem < SW ? rem : SW);
-      s_subbytes[s] = (ms * (uint32_t)wmax + 7) / 8;
-      reinterpret_cast<uint8_t*>(s_out)[s] = ms ? (uint8_t)wq[q] : (uint8_t)0;
+    mbar_wait(&S.empty_out[o], pho ^ 1);  // output slot free
+    if (lane < kSubPerWarp) {
+      const uint32_t sub = cw * kSubPerWarp + lane;
+      const uint32_t h = lane == 0 ? wq[0] : lane == 1 ? wq[1] : lane == 2 ? wq[2] : wq[3];
+      S.hdr[o][sub] = (sub * SW < m) ? h : 0u;
     }
-  }
-  __syncthreads();
+    named_bar_sync(kBarCompute, kCompThreads);
 
-  // ---- chunk size, raw decision, aggregate published before packing ----
-  if (warp == 0) {
-    const uint32_t S = (m + SW - 1) / SW;
-    const uint32_t hdr = (S + 7) & ~7u;
-    const uint32_t b = s_subbytes[lane];
+    // chunk layout: header bytes, subchunk offsets, size, raw decision
+    const uint32_t S_sub = (m + SW - 1) / SW, hdr_bytes = (S_sub + 7) & ~7u;
+    const uint32_t h = S.hdr[o][lane];
+    const int32_t rem = (int32_t)m - (int32_t)(lane * SW);
+    const uint32_t ms = rem <= 0 ? 0u : (rem < SW ? (uint32_t)rem : (uint32_t)SW);
+    const uint32_t b = (ms * (h & 0x7F) + 7) >> 3;
     uint32_t incl = b;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, incl, d);
-      if (lane >= d) incl += o;
+      const uint32_t x = __shfl_up_sync(0xFFFFFFFFu, incl, d);
+      if ((int)lane >= d) incl += x;
     }
-    s_suboff[lane] = hdr + incl - b;
-    const uint32_t total = hdr + __shfl_sync(0xFFFFFFFFu, incl, 31);
+    const uint32_t total = hdr_bytes + __shfl_sync(0xFFFFFFFFu, incl, 31);
     const uint32_t raw_len = m * (uint32_t)sizeof(U);
     const bool raw = total >= raw_len;  // L104, ties → raw
     const uint32_t len = raw ? raw_len : total;
-    if (lane == 0) {
-      s_len = len;
-      s_raw = raw;
-      lookback_publish(ctx, c, round16(len));
-    }
-    if (!raw && lane < 16 && len + lane < round16(len))  // zero pad bytes
-      reinterpret_cast<uint8_t*>(s_out)[len + lane] = 0;
-  }
-  __syncthreads();
-  const uint32_t len = s_len;
-  const bool raw = s_raw;
-
-  if (warp == 0) {
-    const uint64_t excl = lookback_warp(ctx, c, round16(len));
-    if (lane == 0) s_excl = excl;
-  }
-  if (!raw) {
-#pragma unroll
-    for (int q = 0; q < kSubPerWarp; ++q) {
-      const uint32_t w = wq[q] & 0x7F;
-      if (w == 0) continue;
-      const int s = warp * kSubPerWarp + q;
-      const unsigned Lb = K * w;
-      uint64_t lo, hi;
-      make_string(v[q], w, lo, hi);
-      emit_bits_warp(s_out, (uint64_t)s_suboff[s] * 8 + (uint64_t)lane * Lb, Lb, lo, hi, false, Lb >= 32);
-    }
-  }
-  __syncthreads();
-
-  // ---- store at the resolved offset (16-byte granules) ----
-  uint8_t* dst = a.payload + s_excl;
-  const uint32_t n16 = (uint32_t)(round16(len) / 16);
-  if (!raw) {
-    for (uint32_t i = tid; i < n16; i += kThreads)
-      __stcs(reinterpret_cast<uint4*>(dst) + i, reinterpret_cast<const uint4*>(s_out)[i]);
-  } else {
-    const uint8_t* rsrc = reinterpret_cast<const uint8_t*>(src);
-    for (uint32_t i = tid; i < n16; i += kThreads) {
-      uint4 val;
-      if (16 * i + 16 <= len) {
-        val = __ldcs(reinterpret_cast<const uint4*>(rsrc) + i);
-      } else {
-        uint32_t wv[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j)
-          wv[j] = (16 * i + 4 * j < len) ? reinterpret_cast<const uint32_t*>(rsrc)[4 * i + j] : 0u;
-        val = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+    uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
+    if (cw == 0) {
+      if (lane == 0) {
+        lookback_publish(ctx, t, round16(len));
+        S.out_chunk[o] = t;
+        S.out_len[o] = len;
+        S.out_raw[o] = raw;
       }
-      __stcs(reinterpret_cast<uint4*>(dst) + i, val);
+      if (!raw && lane < hdr_bytes) ob[lane] = (uint8_t)h;
+    }
+    if (raw) {  // store the chunk's own bytes (re-read; L2-resident or HBM)
+      const uint4* src = reinterpret_cast<const uint4*>(reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes);
+      for (uint32_t g = cw * 32 + lane; g < round16(len) / 16; g += kCompThreads) {
+        uint4 val;
+        if (16 * g + 16 <= len) {
+          val = __ldcs(src + g);
+        } else {
+          const uint32_t* s32 = reinterpret_cast<const uint32_t*>(src + g);
+          val.x = s32[0];
+          val.y = 16 * g + 4 < len ? s32[1] : 0u;
+          val.z = 16 * g + 8 < len ? s32[2] : 0u;
+          val.w = 16 * g + 12 < len ? s32[3] : 0u;
+        }
+        reinterpret_cast<uint4*>(ob)[g] = val;
+      }
+    } else {
+      const uint32_t excl = hdr_bytes + incl - b;  // this lane's subchunk offset
+#pragma unroll
+      for (int q = 0; q < kSubPerWarp; ++q) {
+        const uint32_t sub = cw * kSubPerWarp + q;
+        const uint32_t w = wq[q] & 0x7F;
+        const uint32_t off = __shfl_sync(0xFFFFFFFFu, excl, sub);
+        if (w == 0 || sub >= S_sub) continue;
+        const uint32_t L = K * w;
+        uint32_t Sg[4];
+        make_string(v[q], w, Sg);
+        uint32_t* buf = S.out[o] + (off >> 2);
+        if (L >= 32) {
+          emit_equal(buf, lane, L, Sg);
+        } else {
+          emit_bits_warp(buf, (uint64_t)lane * L, L, (uint64_t)Sg[0] | ((uint64_t)Sg[1] << 32),
+                         (uint64_t)Sg[2] | ((uint64_t)Sg[3] << 32), false, false);
+        }
+      }
+      // zero pad [len, round16(len)): done by the warp owning the last subchunk
+      if ((S_sub - 1) / kSubPerWarp == cw) {
+        __syncwarp();
+        if (lane < 16 && len + lane < round16(len)) ob[len + lane] = 0;
+      }
+    }
+    fence_proxy_async_smem();  // packed bytes → visible to the TMA store
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.full_out[o]);
+  }
+}
+
+__device__ __forceinline__ void enc_storer(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane) {
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t o = it % kEncOut, ph = (it / kEncOut) & 1;
+    mbar_wait(&S.full_out[o], ph);
+    const uint64_t t = S.out_chunk[o];
+    if (t == kNoChunk) break;
+    const uint32_t len = S.out_len[o], raw = S.out_raw[o];
+    const uint64_t excl = lookback_warp(ctx, t, round16(len));
+    if (lane == 0) {
+      tma_store_1d(a.payload + excl, S.out[o], (uint32_t)round16(len));
+      tma_store_commit();
+      a.table[t] = len | (raw ? kRawFlag : 0u);
+      if (t == a.n_chunks - 1) finish_encode(a, excl + round16(len));
+      if (t == 0)
+        for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
+      tma_store_wait_read0();
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_out[o]);
+  }
+  if (lane == 0) tma_store_wait_all0();
+}
+
+__device__ __forceinline__ void enc_loader(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
+                                           uint32_t wb) {
+  const uint32_t CW = kChunkBytes / wb;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kEncStages, ph = (it / kEncStages) & 1;
+    mbar_wait(&S.empty_in[s], ph ^ 1);
+    uint64_t t = 0;
+    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
+    t = __shfl_sync(0xFFFFFFFFu, t, 0);
+    if (t >= a.n_chunks) {
+      if (lane == 0) {
+        S.in_chunk[s] = kNoChunk;
+        mbar_arrive(&S.full_in[s]);
+        ticket_retire(ctx);
+      }
+      return;
+    }
+    const uint32_t bytes = chunk_words(a.n_words_total, a.first_chunk + t, CW) * wb;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes;
+    if ((bytes & 15) == 0) {
+      if (lane == 0) {
+        S.in_chunk[s] = t;
+        mbar_arrive_expect_tx(&S.full_in[s], bytes);
+        tma_load_1d(S.in[s], src, bytes, &S.full_in[s]);
+      }
+    } else {  // ragged tail chunk: plain loads
+      for (uint32_t i = lane; i < bytes / 4; i += 32) S.in[s][i] = reinterpret_cast<const uint32_t*>(src)[i];
+      if (lane == 0) S.in_chunk[s] = t;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.full_in[s]);
     }
   }
-  if (tid == 0) {
-    a.table[c] = len | (raw ? kRawFlag : 0u);
-    if (c == a.n_chunks - 1) finish_encode(a, s_excl + round16(len));
-  }
-  if (c == 0 && tid < 16 && tid < a.pad_len) a.pad_start[tid] = 0;
 }
 
 template <typename U>
-__global__ void __launch_bounds__(kThreads) speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kEncThreads) speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  EncSmem& S = *reinterpret_cast<EncSmem*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kEncStages; ++i) {
+      mbar_init(&S.full_in[i], 1);
+      mbar_init(&S.empty_in[i], kCompWarps);
+    }
+    for (int i = 0; i < kEncOut; ++i) {
+      mbar_init(&S.full_out[i], kCompWarps);
+      mbar_init(&S.empty_out[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0) enc_loader(S, a, ctx, lane, sizeof(U));
+  else if (warp == 1) enc_storer(S, a, ctx, lane);
+  else enc_compute<U>(S, a, ctx, warp - 2, lane);
+}
+
+// =================================== decode ======================================
+template <typename U>
+__device__ __forceinline__ void dec_loader(DecSmem<U>& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t lane) {
+  using C = Cfg<U>;
+  uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
+  const bool hdr_ok = read_header(a, ctx, n_words, n_chunks, base, payload);
+  const bool small = hdr_ok && n_words * sizeof(U) > a.out_capacity;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
+    mbar_wait(&S.empty_in[s], ph ^ 1);
+    uint64_t t = 0;
+    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
+    t = __shfl_sync(0xFFFFFFFFu, t, 0);
+    if (!hdr_ok || small || t >= n_chunks) {
+      if (lane == 0) {
+        if (t == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
+        if (t == 0 && small) record_error(ctx, DERR_SMALL);
+        S.chunk[s] = kNoChunk;
+        mbar_arrive(&S.full_in[s]);
+        ticket_retire(ctx);
+      }
+      return;
+    }
+    const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[t];
+    const uint32_t len = e & ~kRawFlag, raw = e >> 31;
+    const uint32_t m = chunk_words(n_words, t, C::CW);
+    bool bad = raw ? len != m * sizeof(U) : len >= m * sizeof(U);
+    if (lane == 0) lookback_publish(ctx, t, bad ? 0 : round16(len));
+    const uint64_t excl = lookback_warp(ctx, t, bad ? 0 : round16(len));
+    const uint64_t end = excl + round16(len);
+    if (!bad && (end > payload || (t == n_chunks - 1 && end != payload))) bad = true;
+    if (lane == 0) {
+      if (bad) record_error(ctx, DERR_CORRUPT);
+      S.chunk[s] = t;
+      S.len[s] = len;
+      S.flags[s] = raw | (bad ? 2u : 0u);
+      if (!bad && len) {
+        mbar_arrive_expect_tx(&S.full_in[s], (uint32_t)round16(len));
+        tma_load_1d(S.in[s], a.stream + base + excl, (uint32_t)round16(len), &S.full_in[s]);
+      } else {
+        mbar_arrive(&S.full_in[s]);
+      }
+    }
+  }
+}
+
+template <typename U>
+__device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t cw,
+                                            uint32_t lane) {
   using C = Cfg<U>;
   constexpr int W = C::W, CW = C::CW, SW = C::SW, K = C::K;
-  __shared__ __align__(16) uint32_t s_in[(kChunkBytes + 64) / 4];
-  __shared__ uint32_t s_suboff[32], s_hdr[32];
-  __shared__ U s_wtot[kWarps];
-  __shared__ uint64_t s_excl;
-  __shared__ DecChunk s_ch;
-
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_ch = decode_chunk_begin(a, ctx, sizeof(U), CW);
-  __syncthreads();
-  const DecChunk ch = s_ch;
-  if (!ch.ok) return;
-  if (warp == 0) {
-    const uint64_t excl = lookback_warp(ctx, ch.c, round16(ch.len));
-    if (lane == 0) {
-      s_excl = excl;
-      const uint64_t end = excl + round16(ch.len);
-      if (end > ch.payload_bytes || (ch.c == ch.n_chunks - 1 && end != ch.payload_bytes)) {
-        record_error(ctx, DERR_CORRUPT);
-        s_ch.ok = 0;
-      }
+  const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
+  const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / sizeof(U);
+  uint32_t scan_it = 0;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
+    mbar_wait(&S.full_in[s], ph);
+    const uint64_t t = S.chunk[s];
+    if (t == kNoChunk) return;
+    const uint32_t len = S.len[s], fl = S.flags[s];
+    const uint32_t m = chunk_words(n_words, t, CW);
+    U* dst = reinterpret_cast<U*>(a.out) + t * CW;
+    const uint32_t* in = S.in[s];
+    if (fl & 2) {  // malformed entry: nothing to decode
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      continue;
     }
-  }
-  __syncthreads();
-  if (!s_ch.ok) return;
-  const uint8_t* psrc = a.stream + ch.base + s_excl;
-  const uint32_t n16 = (uint32_t)(round16(ch.len) / 16);
-  U* dst = reinterpret_cast<U*>(a.out) + ch.c * CW;
-  const uint32_t m = ch.m;
-
-  if (ch.raw) {  // raw chunk: copy (len = m·sizeof(U))
-    for (uint32_t i = tid; i < n16; i += kThreads) {
-      const uint4 val = __ldcs(reinterpret_cast<const uint4*>(psrc) + i);
-      if (16 * i + 16 <= ch.len) {
-        __stcs(reinterpret_cast<uint4*>(dst) + i, val);
-      } else {
-        const uint32_t wv[4] = {val.x, val.y, val.z, val.w};
-        for (int j = 0; j < 4; ++j)
-          if (16 * i + 4 * j < ch.len) reinterpret_cast<uint32_t*>(dst)[4 * i + j] = wv[j];
+    if (fl & 1) {  // raw chunk: copy
+      for (uint32_t g = cw * 32 + lane; g < round16(len) / 16; g += kCompThreads) {
+        const uint4 val = reinterpret_cast<const uint4*>(in)[g];
+        if (16 * g + 16 <= len) {
+          __stcs(reinterpret_cast<uint4*>(dst) + g, val);
+        } else {
+          const uint32_t wv[4] = {val.x, val.y, val.z, val.w};
+          for (int j = 0; j < 4; ++j)
+            if (16 * g + 4 * j < len) reinterpret_cast<uint32_t*>(dst)[4 * g + j] = wv[j];
+        }
       }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      continue;
     }
-    return;
-  }
-  for (uint32_t i = tid; i < n16; i += kThreads)
-    reinterpret_cast<uint4*>(s_in)[i] = __ldcs(reinterpret_cast<const uint4*>(psrc) + i);
-  __syncthreads();
-
-  // ---- MPLG header: widths, flags, subchunk offsets (L114–118) ----
-  if (warp == 0) {
-    const uint32_t S = (m + SW - 1) / SW;
-    const uint32_t hdr = (S + 7) & ~7u;
-    const int64_t rem = (int64_t)m - (int64_t)lane * SW;
-    const uint32_t ms = rem <= 0 ? 0u : (uint32_t)(rem < SW ? rem : SW);
-    uint32_t h = ms ? reinterpret_cast<const uint8_t*>(s_in)[lane] : 0u;
-    bool bad = (h & 0x7F) > (uint32_t)W;
-    if (bad) h = 0;
-    const uint32_t b = (ms * (h & 0x7F) + 7) / 8;
+    // ---- MPLG header: widths, flags, subchunk offsets (L114–118) ----
+    const uint32_t S_sub = (m + SW - 1) / SW, hdr_bytes = (S_sub + 7) & ~7u;
+    const int32_t rem = (int32_t)m - (int32_t)(lane * SW);
+    const uint32_t ms = rem <= 0 ? 0u : (rem < SW ? (uint32_t)rem : (uint32_t)SW);
+    uint32_t h = ms ? reinterpret_cast<const uint8_t*>(in)[lane] : 0u;
+    const bool badw = (h & 0x7F) > (uint32_t)W;
+    if (badw) h = 0;
+    const uint32_t b = (ms * (h & 0x7F) + 7) >> 3;
     uint32_t incl = b;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, incl, d);
-      if (lane >= d) incl += o;
+      const uint32_t x = __shfl_up_sync(0xFFFFFFFFu, incl, d);
+      if ((int)lane >= d) incl += x;
     }
-    s_suboff[lane] = hdr + incl - b;
-    s_hdr[lane] = h;
-    const uint32_t total = hdr + __shfl_sync(0xFFFFFFFFu, incl, 31);
-    if (__any_sync(0xFFFFFFFFu, bad) || total != ch.len || hdr > ch.len) {
-      if (lane == 0) {
-        record_error(ctx, DERR_CORRUPT);
-        s_ch.ok = 0;
+    const uint32_t total = hdr_bytes + __shfl_sync(0xFFFFFFFFu, incl, 31);
+    if (__any_sync(0xFFFFFFFFu, badw) || total != len) {  // every compute warp agrees
+      if (cw == 0 && lane == 0) record_error(ctx, DERR_CORRUPT);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      continue;
+    }
+    const uint32_t excl_b = hdr_bytes + incl - b;
+    const uint32_t nwords = (uint32_t)(round16(len) / 4);
+    // ---- unpack K fields per lane, unTCMS, differences ----
+    U d[kSubPerWarp][K];
+    U lane_tot[kSubPerWarp];
+#pragma unroll
+    for (int q = 0; q < kSubPerWarp; ++q) {
+      const uint32_t sub = cw * kSubPerWarp + q;
+      const uint32_t hq = __shfl_sync(0xFFFFFFFFu, h, sub);
+      const uint32_t off = __shfl_sync(0xFFFFFFFFu, excl_b, sub);
+      const uint32_t w = hq & 0x7F;
+      const uint32_t P = off * 8 + lane * K * w, F = P >> 5, r = P & 31;
+      uint32_t T[5], U4[4];
+#pragma unroll
+      for (int j = 0; j < 5; ++j) T[j] = (w && F + j < nwords) ? in[F + j] : 0u;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) U4[j] = __funnelshift_r(T[j], T[j + 1], r);
+      split_string(U4, w, d[q]);
+      U tot = 0;
+#pragma unroll
+      for (int j = 0; j < K; ++j) {
+        U u = d[q][j];
+        if (hq >> 7) u = tcms_inv(u);
+        d[q][j] = tcms_inv(u);
+        tot += d[q][j];
+      }
+      lane_tot[q] = tot;
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[s]);  // stage fully read
+    // ---- DIFFMS⁻¹: CTA-wide inclusive prefix sum mod 2^W (L132) ----
+    U wcarry = 0, excl_q[kSubPerWarp];
+#pragma unroll
+    for (int q = 0; q < kSubPerWarp; ++q) {
+      U inc = lane_tot[q];
+#pragma unroll
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const U x = __shfl_up_sync(0xFFFFFFFFu, inc, dd);
+        if ((int)lane >= dd) inc += x;
+      }
+      excl_q[q] = wcarry + inc - lane_tot[q];
+      wcarry += shfl_idx(inc, 31);
+    }
+    const uint32_t sb = scan_it++ & 1;
+    if (lane == 0) S.wtot[sb][cw] = wcarry;
+    named_bar_sync(kBarCompute, kCompThreads);
+    U wbase = 0;
+#pragma unroll
+    for (uint32_t i = 0; i < kCompWarps; ++i)
+      if (i < cw) wbase += S.wtot[sb][i];
+#pragma unroll
+    for (int q = 0; q < kSubPerWarp; ++q) {
+      U run = wbase + excl_q[q];
+      U x[K];
+#pragma unroll
+      for (int j = 0; j < K; ++j) {
+        run += d[q][j];
+        x[j] = run;
+      }
+      const uint32_t i0 = (cw * kSubPerWarp + q) * SW + lane * K;
+      if (i0 + K <= m) {
+        __stcs(reinterpret_cast<uint4*>(dst + i0), pack16<U>(x));
+      } else {
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+          if (i0 + j < m) dst[i0 + j] = x[j];
       }
     }
   }
-  __syncthreads();
-  if (!s_ch.ok) return;
+}
 
-  // ---- unpack K fields per lane, unTCMS, local sums ----
-  const uint32_t nwords = n16 * 4;
-  U d[kSubPerWarp][K];
-  U lane_tot[kSubPerWarp];
-#pragma unroll
-  for (int q = 0; q < kSubPerWarp; ++q) {
-    const int s = warp * kSubPerWarp + q;
-    const uint32_t h = s_hdr[s];
-    const uint32_t w = h & 0x7F;
-    const uint64_t off = (uint64_t)s_suboff[s] * 8 + (uint64_t)lane * K * w;
-    const uint32_t F = (uint32_t)(off >> 5), r = (uint32_t)(off & 31);
-    uint32_t t[5];
-#pragma unroll
-    for (int j = 0; j < 5; ++j) t[j] = (w && F + j < nwords) ? s_in[F + j] : 0u;
-    const uint64_t lo = (uint64_t)__funnelshift_r(t[0], t[1], r) | ((uint64_t)__funnelshift_r(t[1], t[2], r) << 32);
-    const uint64_t hi = (uint64_t)__funnelshift_r(t[2], t[3], r) | ((uint64_t)__funnelshift_r(t[3], t[4], r) << 32);
-    split_string(lo, hi, w, d[q]);
-    U tot = 0;
-#pragma unroll
-    for (int j = 0; j < K; ++j) {
-      U u = d[q][j];
-      if (h >> 7) u = tcms_inv(u);
-      d[q][j] = tcms_inv(u);  // DIFFMS difference
-      tot += d[q][j];
+template <typename U>
+__global__ void __launch_bounds__(kDecThreads) speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  DecSmem<U>& S = *reinterpret_cast<DecSmem<U>*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kDecStages; ++i) {
+      mbar_init(&S.full_in[i], 1);
+      mbar_init(&S.empty_in[i], kCompWarps);
     }
-    lane_tot[q] = tot;
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  // ---- DIFFMS⁻¹: block-wide inclusive prefix sum mod 2^W (L132) ----
-  U wcarry = 0;
-  U excl_q[kSubPerWarp];
-#pragma unroll
-  for (int q = 0; q < kSubPerWarp; ++q) {
-    U incl = lane_tot[q];
-#pragma unroll
-    for (int dd = 1; dd < 32; dd <<= 1) {
-      const U o = __shfl_up_sync(0xFFFFFFFFu, incl, dd);
-      if (lane >= dd) incl += o;
-    }
-    excl_q[q] = wcarry + incl - lane_tot[q];
-    wcarry += shfl_idx(incl, 31);
-  }
-  if (lane == 0) s_wtot[warp] = wcarry;
   __syncthreads();
-  U wbase = 0;
-  for (int i = 0; i < warp; ++i) wbase += s_wtot[i];
-#pragma unroll
-  for (int q = 0; q < kSubPerWarp; ++q) {
-    U run = wbase + excl_q[q];
-    U x[K];
-#pragma unroll
-    for (int j = 0; j < K; ++j) {
-      run += d[q][j];
-      x[j] = run;
-    }
-    const uint32_t i0 = (warp * kSubPerWarp + q) * SW + lane * K;
-    if (i0 + K <= m) {
-      __stcs(reinterpret_cast<uint4*>(dst + i0), pack16<U>(x));
-    } else {
-#pragma unroll
-      for (int j = 0; j < K; ++j)
-        if (i0 + j < m) dst[i0 + j] = x[j];
-    }
-  }
+  if (warp == 0) dec_loader<U>(S, a, ctx, lane);
+  else dec_compute<U>(S, a, ctx, warp - 1, lane);
 }
 
 }  // namespace
 
 template <typename U> void launch_speed_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st) {
-  speed_encode_kernel<U><<<(unsigned)a.n_chunks, kThreads, 0, st>>>(a, ctx);
+  const size_t smem = sizeof(EncSmem);
+  static const bool init = [&] {
+    cudaFuncSetAttribute(speed_encode_kernel<U>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return true;
+  }();
+  (void)init;
+  const int grid = persistent_grid(speed_encode_kernel<U>, kEncThreads, smem, a.n_chunks);
+  speed_encode_kernel<U><<<grid, kEncThreads, smem, st>>>(a, ctx);
 }
-template <typename U> void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, unsigned grid, cudaStream_t st) {
-  speed_decode_kernel<U><<<grid, kThreads, 0, st>>>(a, ctx);
+template <typename U>
+void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st) {
+  const size_t smem = sizeof(DecSmem<U>);
+  static const bool init = [&] {
+    cudaFuncSetAttribute(speed_decode_kernel<U>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return true;
+  }();
+  (void)init;
+  const int grid = persistent_grid(speed_decode_kernel<U>, kDecThreads, smem, max_chunks);
+  speed_decode_kernel<U><<<grid, kDecThreads, smem, st>>>(a, ctx);
 }
 template void launch_speed_encode<uint32_t>(const EncArgs&, const LaunchCtx&, cudaStream_t);
 template void launch_speed_encode<uint64_t>(const EncArgs&, const LaunchCtx&, cudaStream_t);
-template void launch_speed_decode<uint32_t>(const DecArgs&, const LaunchCtx&, unsigned, cudaStream_t);
-template void launch_speed_decode<uint64_t>(const DecArgs&, const LaunchCtx&, unsigned, cudaStream_t);
+template void launch_speed_decode<uint32_t>(const DecArgs&, const LaunchCtx&, uint64_t, cudaStream_t);
+template void launch_speed_decode<uint64_t>(const DecArgs&, const LaunchCtx&, uint64_t, cudaStream_t);
 
 }  // namespace lcf

@@ -43,6 +43,7 @@ def gpu_roundtrip(L, algo, x_dev):
 
 
 def check_parity(L, orc, algo, words: np.ndarray, name=""):
+    words = np.ascontiguousarray(words).reshape(-1)
     x = to_dev(words)
     s_gpu, y = gpu_roundtrip(L, algo, x)
     s_orc = orc.compress(algo, words)
@@ -52,7 +53,7 @@ def check_parity(L, orc, algo, words: np.ndarray, name=""):
         bad = [i for i in range(min(len(t1), len(t2))) if t1[i] != t2[i] or c1[i] != c2[i]]
         raise AssertionError(f"{algo}/{name}: stream differs (len {len(s_gpu)} vs {len(s_orc)}; "
                              f"headers {h1 == h2}; first bad chunk {bad[:5]})")
-    assert torch.equal(y, x), f"{algo}/{name}: decompressed bits differ"
+    assert torch.equal(y.reshape(-1), x.reshape(-1)), f"{algo}/{name}: decompressed bits differ"
     # cross-decode: oracle decodes the GPU stream (identical bytes) and GPU decodes oracle's
     assert np.array_equal(orc.decompress(algo, s_gpu), words)
     return len(s_gpu)
@@ -150,7 +151,7 @@ def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
         assert tab[0] == table[c], (c, tab[0], table[c])
         assert pay[:tab[0] & 0x7FFFFFFF] == chunks[c][1], c
     y = L.decompress(algo, s)
-    assert torch.equal(y, x_dev)
+    assert torch.equal(y, x_dev.reshape(-1))
     return len(stream)
 
 
@@ -161,7 +162,7 @@ def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
 def test_full_size_sampled_parity(L, orc, algo, config, field):
     if algo not in algos_available(L):
         pytest.skip(f"{algo} not built")
-    x = datagen.field(config, field, device="cuda")
+    x = datagen.field(config, field, device="cuda").reshape(-1)
     x = x.view(tdt(algo))
     sampled_chunk_parity(L, orc, algo, x)
     del x

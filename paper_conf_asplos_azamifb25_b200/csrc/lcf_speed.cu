@@ -28,8 +28,25 @@ namespace lcf {
 namespace {
 
 constexpr int kCompWarps = 8, kSubPerWarp = 4;
-constexpr int kEncStages = 3, kEncOut = 2, kDecStages = 4;
-constexpr int kEncThreads = (2 + kCompWarps) * 32;
+#ifndef LCF_ENC_STAGES
+#define LCF_ENC_STAGES 3
+#endif
+#ifndef LCF_ENC_OUT
+#define LCF_ENC_OUT 3
+#endif
+#ifndef LCF_ENC_STORERS
+#define LCF_ENC_STORERS 1
+#endif
+#ifndef LCF_DEC_STAGES
+#define LCF_DEC_STAGES 4
+#endif
+#ifndef LCF_DEC_BATCH
+#define LCF_DEC_BATCH 4
+#endif
+constexpr int kEncStages = LCF_ENC_STAGES, kEncOut = LCF_ENC_OUT, kStorers = LCF_ENC_STORERS;
+constexpr int kDecStages = LCF_DEC_STAGES, kDecBatch = LCF_DEC_BATCH;
+static_assert(kStorers == 1 || kEncOut % kStorers == 0, "each output slot belongs to one storer");
+constexpr int kEncThreads = (1 + kStorers + kCompWarps) * 32;
 constexpr int kDecThreads = (1 + kCompWarps) * 32;
 constexpr uint32_t kCompThreads = kCompWarps * 32;
 constexpr uint64_t kNoChunk = ~0ull;
@@ -48,7 +65,7 @@ struct EncSmem {
   uint64_t full_in[kEncStages], empty_in[kEncStages], full_out[kEncOut], empty_out[kEncOut];
   uint64_t in_chunk[kEncStages], out_chunk[kEncOut];
   uint32_t out_len[kEncOut], out_raw[kEncOut];
-  uint32_t hdr[kEncOut][32];
+  uint32_t hdr[2][32];
 };
 
 template <typename U> struct DecSmem {
@@ -187,11 +204,14 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
     const uint32_t o = it % kEncOut, pho = (it / kEncOut) & 1;
     mbar_wait(&S.full_in[s], ph);
     const uint64_t t = S.in_chunk[s];
-    if (t == kNoChunk) {  // forward the end marker to the storer
-      mbar_wait(&S.empty_out[o], pho ^ 1);
-      if (cw == 0 && lane == 0) S.out_chunk[o] = kNoChunk;
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&S.full_out[o]);
+    if (t == kNoChunk) {  // forward the end marker to every storer
+      for (uint32_t j = 0; j < kStorers; ++j) {
+        const uint32_t oj = (it + j) % kEncOut, phj = ((it + j) / kEncOut) & 1;
+        mbar_wait(&S.empty_out[oj], phj ^ 1);
+        if (cw == 0 && lane == 0) S.out_chunk[oj] = kNoChunk;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.full_out[oj]);
+      }
       return;
     }
     const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, CW);
@@ -231,17 +251,18 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
       }
       wq[q] = w | (flag << 7);
     }
-    mbar_wait(&S.empty_out[o], pho ^ 1);  // output slot free
+    // widths → shared ring (2 entries, reused every other chunk), then the
+    // chunk size and the aggregate BEFORE waiting for an output slot, so the
+    // look-back of later chunks never waits on this CTA's storer
+    const uint32_t hb = it & 1;
     if (lane < kSubPerWarp) {
       const uint32_t sub = cw * kSubPerWarp + lane;
-      const uint32_t h = lane == 0 ? wq[0] : lane == 1 ? wq[1] : lane == 2 ? wq[2] : wq[3];
-      S.hdr[o][sub] = (sub * SW < m) ? h : 0u;
+      const uint32_t hh = lane == 0 ? wq[0] : lane == 1 ? wq[1] : lane == 2 ? wq[2] : wq[3];
+      S.hdr[hb][sub] = (sub * SW < m) ? hh : 0u;
     }
     named_bar_sync(kBarCompute, kCompThreads);
-
-    // chunk layout: header bytes, subchunk offsets, size, raw decision
     const uint32_t S_sub = (m + SW - 1) / SW, hdr_bytes = (S_sub + 7) & ~7u;
-    const uint32_t h = S.hdr[o][lane];
+    const uint32_t h = S.hdr[hb][lane];
     const int32_t rem = (int32_t)m - (int32_t)(lane * SW);
     const uint32_t ms = rem <= 0 ? 0u : (rem < SW ? (uint32_t)rem : (uint32_t)SW);
     const uint32_t b = (ms * (h & 0x7F) + 7) >> 3;
@@ -255,10 +276,11 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
     const uint32_t raw_len = m * (uint32_t)sizeof(U);
     const bool raw = total >= raw_len;  // L104, ties → raw
     const uint32_t len = raw ? raw_len : total;
+    if (cw == 0 && lane == 0) lookback_publish(ctx, t, round16(len));
+    mbar_wait(&S.empty_out[o], pho ^ 1);  // output slot free
     uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
     if (cw == 0) {
       if (lane == 0) {
-        lookback_publish(ctx, t, round16(len));
         S.out_chunk[o] = t;
         S.out_len[o] = len;
         S.out_raw[o] = raw;
@@ -311,8 +333,9 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
   }
 }
 
-__device__ __forceinline__ void enc_storer(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane) {
-  for (uint32_t it = 0;; ++it) {
+__device__ __forceinline__ void enc_storer(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
+                                           uint32_t first) {
+  for (uint32_t it = first;; it += kStorers) {
     const uint32_t o = it % kEncOut, ph = (it / kEncOut) & 1;
     mbar_wait(&S.full_out[o], ph);
     const uint64_t t = S.out_chunk[o];
@@ -326,10 +349,10 @@ __device__ __forceinline__ void enc_storer(EncSmem& S, const EncArgs& a, const L
       if (t == a.n_chunks - 1) finish_encode(a, excl + round16(len));
       if (t == 0)
         for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
-      tma_store_wait_read0();
+      tma_store_wait_read0();  // the slot's bytes have been read by the TMA unit
+      mbar_arrive(&S.empty_out[o]);
     }
     __syncwarp();
-    if (lane == 0) mbar_arrive(&S.empty_out[o]);
   }
   if (lane == 0) tma_store_wait_all0();
 }
@@ -386,8 +409,8 @@ __global__ void __launch_bounds__(kEncThreads) speed_encode_kernel(EncArgs a, La
   }
   __syncthreads();
   if (warp == 0) enc_loader(S, a, ctx, lane, sizeof(U));
-  else if (warp == 1) enc_storer(S, a, ctx, lane);
-  else enc_compute<U>(S, a, ctx, warp - 2, lane);
+  else if (warp <= kStorers) enc_storer(S, a, ctx, lane, warp - 1);
+  else enc_compute<U>(S, a, ctx, warp - 1 - kStorers, lane);
 }
 
 // =================================== decode ======================================
@@ -397,40 +420,67 @@ __device__ __forceinline__ void dec_loader(DecSmem<U>& S, const DecArgs& a, cons
   uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
   const bool hdr_ok = read_header(a, ctx, n_words, n_chunks, base, payload);
   const bool small = hdr_ok && n_words * sizeof(U) > a.out_capacity;
-  for (uint32_t it = 0;; ++it) {
-    const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
-    mbar_wait(&S.empty_in[s], ph ^ 1);
-    uint64_t t = 0;
-    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
-    t = __shfl_sync(0xFFFFFFFFu, t, 0);
-    if (!hdr_ok || small || t >= n_chunks) {
+  uint32_t it = 0;
+  for (;;) {
+    // a ticket claims kDecBatch consecutive chunks: one look-back per batch,
+    // the batch's own offsets from its size-table entries
+    uint64_t tb = 0;
+    if (lane == 0) tb = atomicAdd(ctx.ticket, 1ull);
+    tb = __shfl_sync(0xFFFFFFFFu, tb, 0) * kDecBatch;
+    if (!hdr_ok || small || tb >= n_chunks) {
+      const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
+      mbar_wait(&S.empty_in[s], ph ^ 1);
       if (lane == 0) {
-        if (t == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
-        if (t == 0 && small) record_error(ctx, DERR_SMALL);
+        if (tb == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
+        if (tb == 0 && small) record_error(ctx, DERR_SMALL);
         S.chunk[s] = kNoChunk;
         mbar_arrive(&S.full_in[s]);
         ticket_retire(ctx);
       }
       return;
     }
-    const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[t];
-    const uint32_t len = e & ~kRawFlag, raw = e >> 31;
-    const uint32_t m = chunk_words(n_words, t, C::CW);
-    bool bad = raw ? len != m * sizeof(U) : len >= m * sizeof(U);
-    if (lane == 0) lookback_publish(ctx, t, bad ? 0 : round16(len));
-    const uint64_t excl = lookback_warp(ctx, t, bad ? 0 : round16(len));
+    const uint32_t nb = (uint32_t)umin64(kDecBatch, n_chunks - tb);
+    const uint64_t t = tb + lane;
+    uint32_t len = 0, raw = 0;
+    bool bad = false;
+    if (lane < nb) {
+      const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[t];
+      len = e & ~kRawFlag;
+      raw = e >> 31;
+      const uint32_t m = chunk_words(n_words, t, C::CW);
+      bad = raw ? len != m * sizeof(U) : len >= m * sizeof(U);
+      lookback_publish(ctx, t, bad ? 0 : round16(len));
+    }
+    const uint64_t agg = (lane < nb && !bad) ? round16(len) : 0;
+    uint64_t x = agg;  // exclusive prefix inside the batch
+#pragma unroll
+    for (int d = 1; d < kDecBatch; d <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+      if ((int)lane >= d) x += y;
+    }
+    x -= agg;
+    const uint64_t base_b = lookback_warp(ctx, tb, __shfl_sync(0xFFFFFFFFu, agg, 0));
+    const uint64_t excl = base_b + x;
+    if (lane > 0 && lane < nb) st_relaxed_u64(ctx.status + t, make_status(kFlagInc, ctx.epoch, excl + agg));
     const uint64_t end = excl + round16(len);
-    if (!bad && (end > payload || (t == n_chunks - 1 && end != payload))) bad = true;
-    if (lane == 0) {
-      if (bad) record_error(ctx, DERR_CORRUPT);
-      S.chunk[s] = t;
-      S.len[s] = len;
-      S.flags[s] = raw | (bad ? 2u : 0u);
-      if (!bad && len) {
-        mbar_arrive_expect_tx(&S.full_in[s], (uint32_t)round16(len));
-        tma_load_1d(S.in[s], a.stream + base + excl, (uint32_t)round16(len), &S.full_in[s]);
-      } else {
-        mbar_arrive(&S.full_in[s]);
+    if (lane < nb && !bad && (end > payload || (t == n_chunks - 1 && end != payload))) bad = true;
+    for (uint32_t j = 0; j < nb; ++j, ++it) {
+      const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
+      const uint32_t lj = __shfl_sync(0xFFFFFFFFu, len, j), rj = __shfl_sync(0xFFFFFFFFu, raw, j);
+      const bool bj = __shfl_sync(0xFFFFFFFFu, bad, j);
+      const uint64_t ej = __shfl_sync(0xFFFFFFFFu, excl, j);
+      mbar_wait(&S.empty_in[s], ph ^ 1);
+      if (lane == 0) {
+        if (bj) record_error(ctx, DERR_CORRUPT);
+        S.chunk[s] = tb + j;
+        S.len[s] = lj;
+        S.flags[s] = rj | (bj ? 2u : 0u);
+        if (!bj && lj) {
+          mbar_arrive_expect_tx(&S.full_in[s], (uint32_t)round16(lj));
+          tma_load_1d(S.in[s], a.stream + base + ej, (uint32_t)round16(lj), &S.full_in[s]);
+        } else {
+          mbar_arrive(&S.full_in[s]);
+        }
       }
     }
   }

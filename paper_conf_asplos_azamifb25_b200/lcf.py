@@ -12,7 +12,7 @@ import ctypes
 import os
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "liblcf.so")
+LIB_PATH = os.environ.get("LCF_LIB_PATH") or os.path.join(PKG, "liblcf.so")
 
 ALGOS = {"SPspeed": 0, "SPratio": 1, "DPspeed": 2, "DPratio": 3}
 DTYPES = {"float32": 0, "float64": 1}

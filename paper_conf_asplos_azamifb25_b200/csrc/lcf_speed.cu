@@ -29,16 +29,16 @@ namespace {
 
 constexpr int kCompWarps = 8, kSubPerWarp = 4;
 #ifndef LCF_ENC_STAGES
-#define LCF_ENC_STAGES 3
+#define LCF_ENC_STAGES 2
 #endif
 #ifndef LCF_ENC_OUT
-#define LCF_ENC_OUT 3
+#define LCF_ENC_OUT 2
 #endif
 #ifndef LCF_ENC_STORERS
 #define LCF_ENC_STORERS 1
 #endif
 #ifndef LCF_DEC_STAGES
-#define LCF_DEC_STAGES 4
+#define LCF_DEC_STAGES 3
 #endif
 #ifndef LCF_DEC_BATCH
 #define LCF_DEC_BATCH 4
@@ -235,11 +235,15 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
       if (lane == 0) p = carry;
       carry = next_carry;
       const uint32_t i0 = (cw * kSubPerWarp + q) * SW + lane * K;
+      if (full) {
 #pragma unroll
-      for (int j = K - 1; j >= 0; --j) {
-        const U prev = j ? v[q][j - 1] : p;
-        const U u = tcms((U)(v[q][j] - prev));
-        v[q][j] = (full || i0 + j < m) ? u : (U)0;
+        for (int j = K - 1; j >= 0; --j) v[q][j] = tcms((U)(v[q][j] - (j ? v[q][j - 1] : p)));
+      } else {
+#pragma unroll
+        for (int j = K - 1; j >= 0; --j) {
+          const U u = tcms((U)(v[q][j] - (j ? v[q][j - 1] : p)));
+          v[q][j] = (i0 + j < m) ? u : (U)0;
+        }
       }
       uint32_t w = warp_width(v[q]);
       uint32_t flag = 0;

@@ -125,9 +125,17 @@ __device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t
 __device__ __forceinline__ int bitlen(uint32_t v) { return 32 - __clz(v); }
 __device__ __forceinline__ int bitlen(uint64_t v) { return 64 - __clzll(v); }
 __device__ __forceinline__ uint32_t tcms(uint32_t d) { return (d << 1) ^ (uint32_t)((int32_t)d >> 31); }
-__device__ __forceinline__ uint64_t tcms(uint64_t d) { return (d << 1) ^ (uint64_t)((int64_t)d >> 63); }
+__device__ __forceinline__ uint64_t tcms(uint64_t d) {  // on 32-bit halves: one shared sign mask
+  const uint32_t lo = (uint32_t)d, hi = (uint32_t)(d >> 32);
+  const uint32_t m = (uint32_t)((int32_t)hi >> 31);
+  return ((uint64_t)(__funnelshift_l(lo, hi, 1) ^ m) << 32) | ((lo << 1) ^ m);
+}
 __device__ __forceinline__ uint32_t tcms_inv(uint32_t u) { return (u >> 1) ^ (0u - (u & 1u)); }
-__device__ __forceinline__ uint64_t tcms_inv(uint64_t u) { return (u >> 1) ^ (0ull - (u & 1ull)); }
+__device__ __forceinline__ uint64_t tcms_inv(uint64_t u) {  // on 32-bit halves: one shared sign mask
+  const uint32_t lo = (uint32_t)u, hi = (uint32_t)(u >> 32);
+  const uint32_t m = (uint32_t)((int32_t)(lo << 31) >> 31);
+  return ((uint64_t)((hi >> 1) ^ m) << 32) | (__funnelshift_r(lo, hi, 1) ^ m);
+}
 
 // 128-bit value (lo, hi) shifted left by s (0..127) / right by s.
 __device__ __forceinline__ void shl128(uint64_t& lo, uint64_t& hi, unsigned s) {

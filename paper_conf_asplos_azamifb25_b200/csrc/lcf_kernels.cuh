@@ -1,6 +1,10 @@
 // lcf_kernels.cuh — argument blocks and launchers of the codec kernels, plus
 // the per-chunk prologue/epilogue shared by all chunk kernels.
 #pragma once
+#include <map>
+#include <mutex>
+#include <utility>
+
 #include "lcf_internal.cuh"
 
 namespace lcf {
@@ -85,18 +89,26 @@ __device__ __forceinline__ bool read_header(const DecArgs& a, const LaunchCtx& c
 }
 
 // Grid of a persistent kernel: every SM filled to its occupancy, capped by the
-// amount of work.
-template <typename Kern> int persistent_grid(Kern kernel, int threads, size_t smem, uint64_t work) {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  }
-  int per_sm = 0;
+// amount of work. The resident capacity is computed once per (kernel, device):
+// the occupancy query costs microseconds of host time that would otherwise sit
+// between the caller's start event and the launch.
+inline int resident_capacity(const void* kernel, int threads, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> g(mu);
+  auto key = std::make_pair(kernel, dev);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  int sms = 0, per_sm = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem);
   if (per_sm < 1) per_sm = 1;
-  const uint64_t g = (uint64_t)sms * per_sm;
+  return cache[key] = sms * per_sm;
+}
+template <typename Kern> int persistent_grid(Kern kernel, int threads, size_t smem, uint64_t work) {
+  const uint64_t g = (uint64_t)resident_capacity(reinterpret_cast<const void*>(kernel), threads, smem);
   return (int)(work < g ? (work ? work : 1) : g);
 }
 

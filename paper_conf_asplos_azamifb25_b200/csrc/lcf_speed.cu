@@ -124,11 +124,19 @@ __device__ __forceinline__ void make_string(const uint32_t* v, uint32_t w, uint3
   }
 }
 __device__ __forceinline__ void make_string(const uint64_t* v, uint32_t w, uint32_t* S) {
-  uint64_t lo, hi;
-  if (w == 64) { lo = v[0]; hi = v[1]; }
-  else if (w == 0) { lo = 0; hi = 0; }
-  else { lo = v[0] | (v[1] << w); hi = v[1] >> (64 - w); }
-  S[0] = (uint32_t)lo; S[1] = (uint32_t)(lo >> 32); S[2] = (uint32_t)hi; S[3] = (uint32_t)(hi >> 32);
+  const uint32_t a0 = (uint32_t)v[0], a1 = (uint32_t)(v[0] >> 32), b0 = (uint32_t)v[1], b1 = (uint32_t)(v[1] >> 32);
+  if (w >= 32) {  // v1 goes to bit w = 32 + s
+    const uint32_t s = w - 32;
+    S[0] = a0;
+    S[1] = a1 | shl_c(b0, s);
+    S[2] = __funnelshift_lc(b0, b1, s);
+    S[3] = __funnelshift_lc(b1, 0u, s);
+  } else {
+    S[0] = a0 | shl_c(b0, w);
+    S[1] = a1 | __funnelshift_lc(b0, b1, w);
+    S[2] = __funnelshift_lc(b1, 0u, w);
+    S[3] = 0;
+  }
 }
 
 // Lanes' strings of equal length L = K·w ≥ 32 bits, lane l at bit l·L of the
@@ -168,12 +176,17 @@ __device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uin
   v[3] = __funnelshift_r(x0, x1, s3) & m;
 }
 __device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uint64_t* v) {
-  const uint64_t lo = (uint64_t)U4[0] | ((uint64_t)U4[1] << 32), hi = (uint64_t)U4[2] | ((uint64_t)U4[3] << 32);
-  const uint64_t m = mask64(w);
-  v[0] = lo & m;
-  uint64_t l2 = lo, h2 = hi;
-  shr128(l2, h2, w);
-  v[1] = l2 & m;
+  // 32-bit pieces: field 0 = bits [0, w), field 1 = bits [w, 2w) of the window
+  const uint32_t mlo = w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u);
+  const uint32_t mhi = w >= 64 ? 0xFFFFFFFFu : (w <= 32 ? 0u : ((1u << (w - 32)) - 1u));
+  v[0] = ((uint64_t)(U4[1] & mhi) << 32) | (U4[0] & mlo);
+  const uint32_t sh = w & 31;
+  uint32_t a0, a1, a2;
+  if (w >= 64) { a0 = U4[2]; a1 = U4[3]; a2 = 0; }
+  else if (w >= 32) { a0 = U4[1]; a1 = U4[2]; a2 = U4[3]; }
+  else { a0 = U4[0]; a1 = U4[1]; a2 = U4[2]; }
+  const uint32_t lo = __funnelshift_r(a0, a1, sh) & mlo, hi = __funnelshift_r(a1, a2, sh) & mhi;
+  v[1] = ((uint64_t)hi << 32) | lo;
 }
 
 template <typename U> __device__ __forceinline__ U shfl_up1(U v) { return __shfl_up_sync(0xFFFFFFFFu, v, 1); }
@@ -549,7 +562,6 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
       continue;
     }
     const uint32_t excl_b = hdr_bytes + incl - b;
-    const uint32_t nwords = (uint32_t)(round16(len) / 4);
     // ---- unpack K fields per lane, unTCMS, differences ----
     U d[kSubPerWarp][K];
     U lane_tot[kSubPerWarp];
@@ -562,7 +574,7 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
       const uint32_t P = off * 8 + lane * K * w, F = P >> 5, r = P & 31;
       uint32_t T[5], U4[4];
 #pragma unroll
-      for (int j = 0; j < 5; ++j) T[j] = (w && F + j < nwords) ? in[F + j] : 0u;
+      for (int j = 0; j < 5; ++j) T[j] = in[F + j];  // ≤ 16 B past len: inside the slack, masked off
 #pragma unroll
       for (int j = 0; j < 4; ++j) U4[j] = __funnelshift_r(T[j], T[j + 1], r);
       split_string(U4, w, d[q]);

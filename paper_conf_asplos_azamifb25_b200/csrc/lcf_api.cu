@@ -160,6 +160,7 @@ lcf_status_t enqueue_encode(Workspace* ws, EncArgs& a) {
   switch (a.algo) {
     case LCF_SPSPEED: launch_speed_encode<uint32_t>(a, ctx, ws->stream); break;
     case LCF_DPSPEED: launch_speed_encode<uint64_t>(a, ctx, ws->stream); break;
+    case LCF_SPRATIO: launch_spratio_encode(a, ctx, ws->stream); break;
     default: return LCF_ERROR_INVALID_ARGUMENT;
   }
   ++g_launches;
@@ -194,7 +195,7 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
   if (in_bytes % wb || !d_out || !aligned16(d_out) || (in_bytes && (!d_in || !aligned16(d_in))))
     return LCF_ERROR_INVALID_ARGUMENT;
   if (out_capacity < lcf_max_compressed_size(algo, dtype, in_bytes)) return LCF_ERROR_BUFFER_TOO_SMALL;
-  if (algo == LCF_DPRATIO || algo == LCF_SPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
+  if (algo == LCF_DPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
@@ -236,7 +237,7 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   if (!d_in || !aligned16(d_in) || (out_capacity && (!d_out || !aligned16(d_out))))
     return LCF_ERROR_INVALID_ARGUMENT;
   if (in_bytes < kHeaderBytes) return LCF_ERROR_CORRUPT_STREAM;
-  if (algo == LCF_DPRATIO || algo == LCF_SPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
+  if (algo == LCF_DPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
@@ -274,6 +275,7 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   switch (algo) {
     case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, grid, stream); break;
     case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, grid, stream); break;
+    case LCF_SPRATIO: launch_spratio_decode(a, ctx, grid, stream); break;
     default: return LCF_ERROR_INVALID_ARGUMENT;
   }
   ++g_launches;

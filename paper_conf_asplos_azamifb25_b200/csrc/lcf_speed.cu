@@ -20,8 +20,7 @@
 //                    prefix sum (L132) → 16-byte coalesced stores.
 // Each compute warp owns subchunks 4w..4w+3 (512 B, L118); a lane holds K = 4
 // (f32) or 2 (f64) consecutive words of each.
-#include "lcf_kernels.cuh"
-#include "lcf_pipe.cuh"
+#include "lcf_persist.cuh"
 
 namespace lcf {
 
@@ -49,7 +48,6 @@ static_assert(kStorers == 1 || kEncOut % kStorers == 0, "each output slot belong
 constexpr int kEncThreads = (1 + kStorers + kCompWarps) * 32;
 constexpr int kDecThreads = (1 + kCompWarps) * 32;
 constexpr uint32_t kCompThreads = kCompWarps * 32;
-constexpr uint64_t kNoChunk = ~0ull;
 constexpr uint32_t kBarCompute = 1;  // named barrier of the compute warps
 
 template <typename U> struct Cfg {
@@ -192,20 +190,6 @@ __device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uin
 template <typename U> __device__ __forceinline__ U shfl_up1(U v) { return __shfl_up_sync(0xFFFFFFFFu, v, 1); }
 template <typename U> __device__ __forceinline__ U shfl_idx(U v, int l) { return __shfl_sync(0xFFFFFFFFu, v, l); }
 
-__device__ __forceinline__ uint32_t chunk_words(uint64_t n_words_total, uint64_t gc, uint32_t CW) {
-  return (uint32_t)umin64((uint64_t)CW, n_words_total - gc * CW);
-}
-
-// Ticket dispenser shared by the persistent kernels: ticket[0] counts handed
-// out tickets, ticket[1] counts CTAs that drew their final (failing) ticket;
-// the last one resets both for the next launch on the stream.
-__device__ __forceinline__ void ticket_retire(const LaunchCtx& ctx) {
-  if (atomicAdd(ctx.ticket + 1, 1ull) == gridDim.x - 1) {
-    ctx.ticket[0] = 0;
-    ctx.ticket[1] = 0;
-  }
-}
-
 // =================================== encode ======================================
 template <typename U>
 __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t cw,
@@ -217,14 +201,8 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
     const uint32_t o = it % kEncOut, pho = (it / kEncOut) & 1;
     mbar_wait(&S.full_in[s], ph);
     const uint64_t t = S.in_chunk[s];
-    if (t == kNoChunk) {  // forward the end marker to every storer
-      for (uint32_t j = 0; j < kStorers; ++j) {
-        const uint32_t oj = (it + j) % kEncOut, phj = ((it + j) / kEncOut) & 1;
-        mbar_wait(&S.empty_out[oj], phj ^ 1);
-        if (cw == 0 && lane == 0) S.out_chunk[oj] = kNoChunk;
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&S.full_out[oj]);
-      }
+    if (t == kNoChunk) {
+      enc_forward_end<kEncOut, kStorers>(S, it, cw, lane);
       return;
     }
     const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, CW);
@@ -350,64 +328,6 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
   }
 }
 
-__device__ __forceinline__ void enc_storer(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
-                                           uint32_t first) {
-  for (uint32_t it = first;; it += kStorers) {
-    const uint32_t o = it % kEncOut, ph = (it / kEncOut) & 1;
-    mbar_wait(&S.full_out[o], ph);
-    const uint64_t t = S.out_chunk[o];
-    if (t == kNoChunk) break;
-    const uint32_t len = S.out_len[o], raw = S.out_raw[o];
-    const uint64_t excl = lookback_warp(ctx, t, round16(len));
-    if (lane == 0) {
-      tma_store_1d(a.payload + excl, S.out[o], (uint32_t)round16(len));
-      tma_store_commit();
-      a.table[t] = len | (raw ? kRawFlag : 0u);
-      if (t == a.n_chunks - 1) finish_encode(a, excl + round16(len));
-      if (t == 0)
-        for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
-      tma_store_wait_read0();  // the slot's bytes have been read by the TMA unit
-      mbar_arrive(&S.empty_out[o]);
-    }
-    __syncwarp();
-  }
-  if (lane == 0) tma_store_wait_all0();
-}
-
-__device__ __forceinline__ void enc_loader(EncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
-                                           uint32_t wb) {
-  const uint32_t CW = kChunkBytes / wb;
-  for (uint32_t it = 0;; ++it) {
-    const uint32_t s = it % kEncStages, ph = (it / kEncStages) & 1;
-    mbar_wait(&S.empty_in[s], ph ^ 1);
-    uint64_t t = 0;
-    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
-    t = __shfl_sync(0xFFFFFFFFu, t, 0);
-    if (t >= a.n_chunks) {
-      if (lane == 0) {
-        S.in_chunk[s] = kNoChunk;
-        mbar_arrive(&S.full_in[s]);
-        ticket_retire(ctx);
-      }
-      return;
-    }
-    const uint32_t bytes = chunk_words(a.n_words_total, a.first_chunk + t, CW) * wb;
-    const uint8_t* src = reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes;
-    if ((bytes & 15) == 0) {
-      if (lane == 0) {
-        S.in_chunk[s] = t;
-        mbar_arrive_expect_tx(&S.full_in[s], bytes);
-        tma_load_1d(S.in[s], src, bytes, &S.full_in[s]);
-      }
-    } else {  // ragged tail chunk: plain loads
-      for (uint32_t i = lane; i < bytes / 4; i += 32) S.in[s][i] = reinterpret_cast<const uint32_t*>(src)[i];
-      if (lane == 0) S.in_chunk[s] = t;
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&S.full_in[s]);
-    }
-  }
-}
-
 template <typename U>
 __global__ void __launch_bounds__(kEncThreads) speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
@@ -425,84 +345,12 @@ __global__ void __launch_bounds__(kEncThreads) speed_encode_kernel(EncArgs a, La
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (warp == 0) enc_loader(S, a, ctx, lane, sizeof(U));
-  else if (warp <= kStorers) enc_storer(S, a, ctx, lane, warp - 1);
+  if (warp == 0) enc_loader<kEncStages>(S, a, ctx, lane, sizeof(U));
+  else if (warp <= kStorers) enc_storer<kEncOut, kStorers>(S, a, ctx, lane, warp - 1);
   else enc_compute<U>(S, a, ctx, warp - 1 - kStorers, lane);
 }
 
 // =================================== decode ======================================
-template <typename U>
-__device__ __forceinline__ void dec_loader(DecSmem<U>& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t lane) {
-  using C = Cfg<U>;
-  uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
-  const bool hdr_ok = read_header(a, ctx, n_words, n_chunks, base, payload);
-  const bool small = hdr_ok && n_words * sizeof(U) > a.out_capacity;
-  uint32_t it = 0;
-  for (;;) {
-    // a ticket claims kDecBatch consecutive chunks: one look-back per batch,
-    // the batch's own offsets from its size-table entries
-    uint64_t tb = 0;
-    if (lane == 0) tb = atomicAdd(ctx.ticket, 1ull);
-    tb = __shfl_sync(0xFFFFFFFFu, tb, 0) * kDecBatch;
-    if (!hdr_ok || small || tb >= n_chunks) {
-      const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
-      mbar_wait(&S.empty_in[s], ph ^ 1);
-      if (lane == 0) {
-        if (tb == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
-        if (tb == 0 && small) record_error(ctx, DERR_SMALL);
-        S.chunk[s] = kNoChunk;
-        mbar_arrive(&S.full_in[s]);
-        ticket_retire(ctx);
-      }
-      return;
-    }
-    const uint32_t nb = (uint32_t)umin64(kDecBatch, n_chunks - tb);
-    const uint64_t t = tb + lane;
-    uint32_t len = 0, raw = 0;
-    bool bad = false;
-    if (lane < nb) {
-      const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[t];
-      len = e & ~kRawFlag;
-      raw = e >> 31;
-      const uint32_t m = chunk_words(n_words, t, C::CW);
-      bad = raw ? len != m * sizeof(U) : len >= m * sizeof(U);
-      lookback_publish(ctx, t, bad ? 0 : round16(len));
-    }
-    const uint64_t agg = (lane < nb && !bad) ? round16(len) : 0;
-    uint64_t x = agg;  // exclusive prefix inside the batch
-#pragma unroll
-    for (int d = 1; d < kDecBatch; d <<= 1) {
-      const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
-      if ((int)lane >= d) x += y;
-    }
-    x -= agg;
-    const uint64_t base_b = lookback_warp(ctx, tb, __shfl_sync(0xFFFFFFFFu, agg, 0));
-    const uint64_t excl = base_b + x;
-    if (lane > 0 && lane < nb) st_relaxed_u64(ctx.status + t, make_status(kFlagInc, ctx.epoch, excl + agg));
-    const uint64_t end = excl + round16(len);
-    if (lane < nb && !bad && (end > payload || (t == n_chunks - 1 && end != payload))) bad = true;
-    for (uint32_t j = 0; j < nb; ++j, ++it) {
-      const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
-      const uint32_t lj = __shfl_sync(0xFFFFFFFFu, len, j), rj = __shfl_sync(0xFFFFFFFFu, raw, j);
-      const bool bj = __shfl_sync(0xFFFFFFFFu, bad, j);
-      const uint64_t ej = __shfl_sync(0xFFFFFFFFu, excl, j);
-      mbar_wait(&S.empty_in[s], ph ^ 1);
-      if (lane == 0) {
-        if (bj) record_error(ctx, DERR_CORRUPT);
-        S.chunk[s] = tb + j;
-        S.len[s] = lj;
-        S.flags[s] = rj | (bj ? 2u : 0u);
-        if (!bj && lj) {
-          mbar_arrive_expect_tx(&S.full_in[s], (uint32_t)round16(lj));
-          tma_load_1d(S.in[s], a.stream + base + ej, (uint32_t)round16(lj), &S.full_in[s]);
-        } else {
-          mbar_arrive(&S.full_in[s]);
-        }
-      }
-    }
-  }
-}
-
 template <typename U>
 __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t cw,
                                             uint32_t lane) {
@@ -644,7 +492,7 @@ __global__ void __launch_bounds__(kDecThreads) speed_decode_kernel(DecArgs a, La
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (warp == 0) dec_loader<U>(S, a, ctx, lane);
+  if (warp == 0) dec_loader<kDecStages, kDecBatch>(S, a, ctx, lane, sizeof(U));
   else dec_compute<U>(S, a, ctx, warp - 1, lane);
 }
 
@@ -668,7 +516,7 @@ void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_ch
     return true;
   }();
   (void)init;
-  const int grid = persistent_grid(speed_decode_kernel<U>, kDecThreads, smem, max_chunks);
+  const int grid = persistent_grid(speed_decode_kernel<U>, kDecThreads, smem, (max_chunks + kDecBatch - 1) / kDecBatch);
   speed_decode_kernel<U><<<grid, kDecThreads, smem, st>>>(a, ctx);
 }
 template void launch_speed_encode<uint32_t>(const EncArgs&, const LaunchCtx&, cudaStream_t);

@@ -1,0 +1,578 @@
+// lcf_spratio.cu — SPratio = RZE ∘ BIT₃₂ ∘ DIFFMS₃₂ (§3.2)
+// on sm_100a, in the persistent warp-specialised pipeline of lcf_persist.cuh.
+//
+// Compute threads: 128 (4 warps); thread g owns the 32-word group g of a chunk.
+// Encode, per chunk:
+//   1. thread g reads its group from the TMA-loaded stage with a per-thread
+//      quad rotation (bank-conflict-free), DIFFMS in the rotated order
+//   2. BIT (L140–142, L162): 32×32 bit transpose in registers (5 butterfly
+//      stages); rows are fed reversed so plane p comes out MSB-first; the
+//      quad rotation becomes a bit rotation of each plane word, undone with one
+//      funnel shift → T[p·G + g] into shared memory (plane-major)
+//   3. RZE (L144–148, L164): byte bitmap B1 of 16-byte units with a packed
+//      8-way CTA scan of the unit counts; repetition elimination B1→B2 (CTA
+//      scan), B2→B3 and B3→B4 in warp 0 (warp scan, ballot); every section
+//      size is known before a byte is written, so the aggregate is published
+//      first; then the non-zero and non-repeating bytes are scattered.
+// Decode inverts the stages from the end of the payload (B4 → B3 → B2 → B1 →
+// D), transposes back, and runs DIFFMS⁻¹ as a serial per-group scan plus a CTA
+// scan of the group totals.
+#include "lcf_persist.cuh"
+
+namespace lcf {
+namespace {
+
+constexpr int kRW = 4;                  // compute warps
+constexpr uint32_t kRT = kRW * 32;      // compute threads: one 32-word group each
+constexpr int kRStages = 2, kROut = 2, kRDecStages = 2, kRDecBatch = 4;
+constexpr int kREncThreads = (2 + kRW) * 32, kRDecThreads = (1 + kRW) * 32;
+constexpr uint32_t kBarR = 1;           // named barrier of the compute warps
+
+__device__ __forceinline__ void bar_r() { named_bar_sync(kBarR, kRT); }
+
+// ---- 32×32 bit transpose (Hacker's Delight transpose32, fully unrolled) -------
+template <int J, uint32_t M> __device__ __forceinline__ void tp_stage(uint32_t (&A)[32]) {
+#pragma unroll
+  for (int k = 0; k < 32; ++k) {
+    if (k & J) continue;
+    const uint32_t t = (A[k] ^ (A[k + J] >> J)) & M;
+    A[k] ^= t;
+    A[k + J] ^= t << J;
+  }
+}
+// A[i] = row i with column c at bit 31−c  →  A'[c] bit (31−i) = A[i] bit (31−c)
+__device__ __forceinline__ void transpose32(uint32_t (&A)[32]) {
+  tp_stage<16, 0x0000FFFFu>(A);
+  tp_stage<8, 0x00FF00FFu>(A);
+  tp_stage<4, 0x0F0F0F0Fu>(A);
+  tp_stage<2, 0x33333333u>(A);
+  tp_stage<1, 0x55555555u>(A);
+}
+
+// 4-bit mask of the non-zero bytes of w (bit b ↔ byte b)
+__device__ __forceinline__ uint32_t nz_nibble(uint32_t w) {
+  const uint32_t t = (((w & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | w) & 0x80808080u;
+  return (t * 0x00204081u) >> 28;
+}
+__device__ __forceinline__ uint32_t nz_mask16(const uint4& q) {
+  return nz_nibble(q.x) | (nz_nibble(q.y) << 4) | (nz_nibble(q.z) << 8) | (nz_nibble(q.w) << 12);
+}
+
+// Exclusive scan over the 128 compute threads; `sh` is a 4-entry slot used
+// once per chunk (reuse is separated by later barriers).
+template <typename T>
+__device__ __forceinline__ T cta_excl_scan(T v, T* sh, uint32_t cw, uint32_t lane, T& total) {
+  T x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const T y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+    if ((int)lane >= d) x += y;
+  }
+  if (lane == 31) sh[cw] = x;
+  bar_r();
+  T base = 0;
+  total = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < kRW; ++i) {
+    const T s = sh[i];
+    if (i < cw) base += s;
+    total += s;
+  }
+  return base + x - v;
+}
+
+struct RZESizes {
+  uint32_t L, L1, L2, L3, L4;
+};
+__device__ __forceinline__ RZESizes rze_sizes(uint32_t L) {
+  RZESizes z;
+  z.L = L;
+  z.L1 = (L + 7) / 8;
+  z.L2 = (z.L1 + 7) / 8;
+  z.L3 = (z.L2 + 7) / 8;
+  z.L4 = (z.L3 + 7) / 8;
+  return z;
+}
+
+struct REncSmem {
+  alignas(128) uint32_t in[kRStages][4096];
+  alignas(128) uint32_t out[kROut][(kChunkBytes + 64) / 4];
+  alignas(128) uint32_t T[4096];  // BIT output = RZE input D
+  alignas(16) uint8_t B1[2048 + 16];
+  alignas(16) uint8_t B2[256 + 16];
+  uint64_t full_in[kRStages], empty_in[kRStages], full_out[kROut], empty_out[kROut];
+  uint64_t in_chunk[kRStages], out_chunk[kROut];
+  uint32_t out_len[kROut], out_raw[kROut];
+  uint64_t sc64[2][kRW];
+  uint32_t sc32[2][kRW];
+  uint32_t b3;  // B3 bytes (≤ 32), kept by warp 0 in registers; B4 here
+};
+
+struct RDecSmem {
+  alignas(128) uint32_t in[kRDecStages][(kChunkBytes + 64) / 4];
+  alignas(128) uint32_t T[4096];
+  alignas(128) uint32_t X[kRT * 33];  // decoded words, 33-word row stride (conflict-free)
+  alignas(16) uint8_t B1[2048 + 16];
+  alignas(16) uint8_t B2[256 + 16];
+  uint64_t full_in[kRDecStages], empty_in[kRDecStages];
+  uint64_t chunk[kRDecStages];
+  uint32_t len[kRDecStages], flags[kRDecStages];
+  uint64_t sc64[2][kRW];
+  uint32_t sc32[3][kRW];
+  int32_t s2, bad;
+};
+
+// =================================== encode ======================================
+__device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t cw,
+                                              uint32_t lane) {
+  const uint32_t g = cw * 32 + lane;  // this thread's group
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kRStages, ph = (it / kRStages) & 1;
+    const uint32_t o = it % kROut, pho = (it / kROut) & 1;
+    mbar_wait(&S.full_in[s], ph);
+    const uint64_t t = S.in_chunk[s];
+    if (t == kNoChunk) {
+      enc_forward_end<kROut, 1>(S, it, cw, lane);
+      return;
+    }
+    const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, 4096);
+    const uint32_t G = m / 32;  // full groups; m mod 32 leftover words are copied (A-9)
+    const uint32_t* in = S.in[s];
+
+    // ---- 1. DIFFMS (L110–112) in the rotated order, 2. BIT (L140–142) ----
+    if (g < G) {
+      const uint32_t gr = g & 7, rot = 4 * gr;
+      uint32_t A[32];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {  // a'[4q..4q+3] = words 32g + 4((q+gr)&7) .. : conflict-free
+        const uint4 v = reinterpret_cast<const uint4*>(in)[8 * g + ((q + gr) & 7)];
+        A[4 * q] = v.x; A[4 * q + 1] = v.y; A[4 * q + 2] = v.z; A[4 * q + 3] = v.w;
+      }
+      const uint32_t xprev = g ? in[32 * g - 1] : 0u;
+      uint32_t U[32];
+#pragma unroll
+      for (int j = 0; j < 32; ++j) U[j] = tcms(A[j] - A[(j + 31) & 31]);
+#pragma unroll
+      for (int k = 0; k < 8; ++k)  // word 32g sits at rotated index (32 − 4gr) mod 32
+        if (((8 - gr) & 7) == (uint32_t)k) U[4 * k] = tcms(A[4 * k] - xprev);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) A[i] = U[31 - i];  // rows reversed → planes MSB-first
+      transpose32(A);
+#pragma unroll
+      for (int p = 0; p < 32; ++p) S.T[p * G + g] = __funnelshift_l(A[p], A[p], rot);  // undo rotation
+    } else if (g == G && (m & 31)) {  // leftover words: DIFFMS, copied unchanged by BIT
+      for (uint32_t i = 32 * G; i < m; ++i) S.T[i] = tcms(in[i] - (i ? in[i - 1] : 0u));
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[s]);
+    const RZESizes z = rze_sizes(4 * m);
+    const uint32_t NU = (z.L + 15) / 16;  // 16-byte units of D
+    if (m < 4096) {  // ragged chunk: zero D beyond L and the bitmap tails
+      for (uint32_t i = m + g; i < 4096; i += kRT) S.T[i] = 0;
+      for (uint32_t i = g; i < (2048 + 16) / 4; i += kRT) reinterpret_cast<uint32_t*>(S.B1)[i] = 0;
+    }
+    bar_r();
+
+    // ---- 3. RZE (L144–148): B1 and counts of the units u = g + 128k ----
+    uint64_t pk[2] = {0, 0};
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint32_t u = g + kRT * k;
+      if (u < NU) {
+        const uint32_t mk = nz_mask16(reinterpret_cast<const uint4*>(S.T)[u]);
+        reinterpret_cast<uint16_t*>(S.B1)[u] = (uint16_t)mk;
+        pk[k >> 2] |= (uint64_t)__popc(mk) << (16 * (k & 3));
+      }
+    }
+    uint64_t tot0, tot1;
+    const uint64_t ex0 = cta_excl_scan<uint64_t>(pk[0], S.sc64[0], cw, lane, tot0);
+    const uint64_t ex1 = cta_excl_scan<uint64_t>(pk[1], S.sc64[1], cw, lane, tot1);
+    uint32_t nnzD = 0, koff[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint64_t tk = (k < 4 ? tot0 : tot1) >> (16 * (k & 3)) & 0xFFFF;
+      koff[k] = nnzD + (uint32_t)(((k < 4 ? ex0 : ex1) >> (16 * (k & 3))) & 0xFFFF);
+      nnzD += (uint32_t)tk;
+    }
+    // B1 → B2 (bytes [16g, 16g+16) of B1), repetition elimination (L146)
+    uint32_t c1 = 0;
+    uint4 b1v = make_uint4(0, 0, 0, 0);
+    if (16 * g < z.L1) {
+      b1v = reinterpret_cast<const uint4*>(S.B1)[g];
+      const uint32_t prev = g ? S.B1[16 * g - 1] : 0u;
+      const uint32_t w[4] = {b1v.x, b1v.y, b1v.z, b1v.w};
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const uint32_t cur = (w[j >> 2] >> (8 * (j & 3))) & 0xFF;
+        const uint32_t pre = j ? (w[(j - 1) >> 2] >> (8 * ((j - 1) & 3))) & 0xFF : prev;
+        if (cur != pre && 16 * g + j < z.L1) c1 |= 1u << j;
+      }
+      reinterpret_cast<uint16_t*>(S.B2)[g] = (uint16_t)c1;
+    } else if (2 * g < 256 + 16) {
+      reinterpret_cast<uint16_t*>(S.B2)[g] = 0;
+    }
+    uint32_t nr1;
+    const uint32_t off1 = cta_excl_scan<uint32_t>(__popc(c1), S.sc32[0], cw, lane, nr1);
+    // B2 → B3 → B4 in warp 0 (L2 ≤ 256 bytes, L3 ≤ 32 bytes)
+    uint32_t nr2 = 0, nr3 = 0, b3 = 0, c2 = 0, off2 = 0, b2w0 = 0, b2w1 = 0, b4 = 0;
+    if (cw == 0) {
+      // lane handles B2 bytes [8·lane, 8·lane+8)
+      b2w0 = reinterpret_cast<const uint32_t*>(S.B2)[2 * lane];
+      b2w1 = reinterpret_cast<const uint32_t*>(S.B2)[2 * lane + 1];
+      const uint32_t prevb = __shfl_up_sync(0xFFFFFFFFu, b2w1 >> 24, 1);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const uint32_t cur = ((j < 4 ? b2w0 : b2w1) >> (8 * (j & 3))) & 0xFF;
+        const uint32_t pre = j ? (((j - 1) < 4 ? b2w0 : b2w1) >> (8 * ((j - 1) & 3))) & 0xFF : (lane ? prevb : 0u);
+        if (cur != pre && 8 * lane + j < z.L2) c2 |= 1u << j;
+      }
+      b3 = c2;  // B3 byte `lane`
+      uint32_t x = __popc(c2);
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+        if ((int)lane >= d) x += y;
+      }
+      off2 = x - __popc(c2);
+      nr2 = __shfl_sync(0xFFFFFFFFu, x, 31);
+      const uint32_t pb3 = __shfl_up_sync(0xFFFFFFFFu, b3, 1);
+      const bool ch3 = lane < z.L3 && b3 != (lane ? pb3 : 0u);
+      b4 = __ballot_sync(0xFFFFFFFFu, ch3);
+      nr3 = __popc(b4);
+    }
+    // totals: every thread needs the final length; warp 0 broadcasts through smem
+    if (cw == 0 && lane == 0) S.sc32[1][0] = nr2 | (nr3 << 16);
+    bar_r();
+    {
+      const uint32_t v = S.sc32[1][0];
+      nr2 = v & 0xFFFF;
+      nr3 = v >> 16;
+    }
+    const uint32_t total = nnzD + nr1 + nr2 + nr3 + z.L4;
+    const uint32_t raw_len = 4 * m;
+    const bool raw = total >= raw_len;  // L104, ties → raw
+    const uint32_t len = raw ? raw_len : total;
+    if (cw == 0 && lane == 0) lookback_publish(ctx, t, round16(len));
+    mbar_wait(&S.empty_out[o], pho ^ 1);
+    uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
+    if (cw == 0 && lane == 0) {
+      S.out_chunk[o] = t;
+      S.out_len[o] = len;
+      S.out_raw[o] = raw;
+    }
+    if (raw) {
+      const uint4* src = reinterpret_cast<const uint4*>(reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes);
+      for (uint32_t q = g; q < round16(len) / 16; q += kRT) {
+        uint4 val;
+        if (16 * q + 16 <= len) {
+          val = __ldcs(src + q);
+        } else {
+          const uint32_t* s32 = reinterpret_cast<const uint32_t*>(src + q);
+          val.x = s32[0];
+          val.y = 16 * q + 4 < len ? s32[1] : 0u;
+          val.z = 16 * q + 8 < len ? s32[2] : 0u;
+          val.w = 16 * q + 12 < len ? s32[3] : 0u;
+        }
+        reinterpret_cast<uint4*>(ob)[q] = val;
+      }
+    } else {
+      // nz(D): non-zero bytes of every unit at its scanned offset
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t u = g + kRT * k;
+        if (u >= NU) continue;
+        const uint4 v = reinterpret_cast<const uint4*>(S.T)[u];
+        const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+        uint32_t p = koff[k];
+#pragma unroll
+        for (int b = 0; b < 16; ++b) {
+          const uint32_t by = (w[b >> 2] >> (8 * (b & 3))) & 0xFF;
+          if (by) ob[p++] = (uint8_t)by;
+        }
+      }
+      // nr(B1)
+      {
+        uint32_t p = nnzD + off1;
+        const uint32_t w[4] = {b1v.x, b1v.y, b1v.z, b1v.w};
+#pragma unroll
+        for (int j = 0; j < 16; ++j)
+          if ((c1 >> j) & 1) ob[p++] = (uint8_t)(w[j >> 2] >> (8 * (j & 3)));
+      }
+      if (cw == 0) {
+        // nr(B2), nr(B3), B4
+        uint32_t p = nnzD + nr1 + off2;
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          if ((c2 >> j) & 1) ob[p++] = (uint8_t)((j < 4 ? b2w0 : b2w1) >> (8 * (j & 3)));
+        if ((b4 >> lane) & 1) ob[nnzD + nr1 + nr2 + __popc(b4 & ((1u << lane) - 1))] = (uint8_t)b3;
+        if (lane < z.L4) ob[total - z.L4 + lane] = (uint8_t)(b4 >> (8 * lane));
+        if (lane < 16 && total + lane < round16(total)) ob[total + lane] = 0;
+      }
+    }
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.full_out[o]);
+    bar_r();  // T, B1, B2 and the scan slots are rewritten by the next chunk
+  }
+}
+
+__global__ void __launch_bounds__(kREncThreads) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kRStages; ++i) {
+      mbar_init(&S.full_in[i], 1);
+      mbar_init(&S.empty_in[i], kRW);
+    }
+    for (int i = 0; i < kROut; ++i) {
+      mbar_init(&S.full_out[i], kRW);
+      mbar_init(&S.empty_out[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0) enc_loader<kRStages>(S, a, ctx, lane, 4);
+  else if (warp == 1) enc_storer<kROut, 1>(S, a, ctx, lane, 0);
+  else r_enc_compute(S, a, ctx, warp - 2, lane);
+}
+
+// =================================== decode ======================================
+__device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t cw,
+                                              uint32_t lane) {
+  const uint32_t g = cw * 32 + lane;
+  const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
+  const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / 4;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kRDecStages, ph = (it / kRDecStages) & 1;
+    mbar_wait(&S.full_in[s], ph);
+    const uint64_t t = S.chunk[s];
+    if (t == kNoChunk) return;
+    const uint32_t len = S.len[s], fl = S.flags[s];
+    const uint32_t m = chunk_words(n_words, t, 4096);
+    uint32_t* dst = reinterpret_cast<uint32_t*>(a.out) + t * 4096;
+    const uint8_t* in = reinterpret_cast<const uint8_t*>(S.in[s]);
+    if (fl & 2) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      continue;
+    }
+    if (fl & 1) {  // raw chunk: copy
+      for (uint32_t q = g; q < round16(len) / 16; q += kRT) {
+        const uint4 val = reinterpret_cast<const uint4*>(in)[q];
+        if (16 * q + 16 <= len) {
+          __stcs(reinterpret_cast<uint4*>(dst) + q, val);
+        } else {
+          const uint32_t wv[4] = {val.x, val.y, val.z, val.w};
+          for (int j = 0; j < 4; ++j)
+            if (16 * q + 4 * j < len) dst[4 * q + j] = wv[j];
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      continue;
+    }
+    const RZESizes z = rze_sizes(4 * m);
+    const uint32_t G = m / 32, NU = (z.L + 15) / 16;
+    // ---- RZE⁻¹ from the end: B4 → B3 → B2 (warp 0) ----
+    if (cw == 0) {
+      int32_t bad = len < z.L4;
+      uint32_t b4 = 0;
+      if (!bad)
+        for (uint32_t i = 0; i < z.L4; ++i) b4 |= (uint32_t)in[len - z.L4 + i] << (8 * i);
+      const uint32_t v3 = z.L3 >= 32 ? 0xFFFFFFFFu : ((1u << z.L3) - 1u);
+      const int32_t s3 = (int32_t)len - (int32_t)z.L4 - __popc(b4 & v3);
+      if (s3 < 0) bad = 1;
+      const uint32_t r3 = __popc(b4 & v3 & (0xFFFFFFFFu >> (31 - lane)));
+      const uint32_t b3 = (!bad && lane < z.L3 && r3) ? in[s3 + r3 - 1] : 0u;  // B3 byte `lane`
+      // B2 bytes [8·lane, 8·lane+8): bits of B3 byte `lane`
+      const uint32_t vb = (8 * lane >= z.L2) ? 0u : (z.L2 - 8 * lane >= 8 ? 0xFFu : ((1u << (z.L2 - 8 * lane)) - 1u));
+      const uint32_t bits2 = b3 & vb;
+      uint32_t x = __popc(bits2);
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+        if ((int)lane >= d) x += y;
+      }
+      const uint32_t cnt2 = __shfl_sync(0xFFFFFFFFu, x, 31);
+      const int32_t s2 = s3 - (int32_t)cnt2;
+      if (s2 < 0) bad = 1;
+      bad = __any_sync(0xFFFFFFFFu, bad);
+      uint32_t r = x - __popc(bits2);
+      uint32_t wv[2] = {0, 0};
+      // rank r counts set bits before byte j; value = nr2[r−1] of the last set bit
+      const uint32_t prev_r = r;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        r += (bits2 >> j) & 1;
+        const uint32_t val = (!bad && r) ? in[s2 + r - 1] : 0u;
+        wv[j >> 2] |= val << (8 * (j & 3));
+      }
+      (void)prev_r;
+      reinterpret_cast<uint32_t*>(S.B2)[2 * lane] = wv[0];
+      reinterpret_cast<uint32_t*>(S.B2)[2 * lane + 1] = wv[1];
+      if (lane == 0) {
+        S.s2 = s2;
+        S.bad = bad;
+      }
+    }
+    bar_r();
+    int32_t bad = S.bad;
+    const int32_t s2 = S.s2;
+    // ---- B1: bytes [16g, 16g+16), bits = B2 bytes 2g, 2g+1 ----
+    uint32_t bits1 = 0;
+    if (16 * g < z.L1) {
+      bits1 = reinterpret_cast<const uint16_t*>(S.B2)[g];
+      const uint32_t nvalid = z.L1 - 16 * g;
+      if (nvalid < 16) bits1 &= (1u << nvalid) - 1u;
+    }
+    uint32_t cnt1;
+    uint32_t r1 = cta_excl_scan<uint32_t>(__popc(bits1), S.sc32[0], cw, lane, cnt1);
+    const int32_t s1 = s2 - (int32_t)cnt1;
+    if (s1 < 0) bad = 1;
+    if (16 * g < 2048 + 16) {
+      uint32_t wv[4] = {0, 0, 0, 0};
+      if (!bad) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          r1 += (bits1 >> j) & 1;
+          const uint32_t val = r1 ? in[s1 + r1 - 1] : 0u;
+          wv[j >> 2] |= val << (8 * (j & 3));
+        }
+      }
+      if (16 * g < z.L1) reinterpret_cast<uint4*>(S.B1)[g] = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+    }
+    bar_r();
+    // ---- D: units u = g + 128k, bits = B1 bytes 2u, 2u+1 ----
+    uint32_t ub[8];
+    uint64_t pk[2] = {0, 0};
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint32_t u = g + kRT * k;
+      ub[k] = 0;
+      if (u < NU) {
+        ub[k] = reinterpret_cast<const uint16_t*>(S.B1)[u];
+        const uint32_t nvalid = z.L - 16 * u;
+        if (nvalid < 16) ub[k] &= (1u << nvalid) - 1u;
+        pk[k >> 2] |= (uint64_t)__popc(ub[k]) << (16 * (k & 3));
+      }
+    }
+    uint64_t tot0, tot1;
+    const uint64_t ex0 = cta_excl_scan<uint64_t>(pk[0], S.sc64[0], cw, lane, tot0);
+    const uint64_t ex1 = cta_excl_scan<uint64_t>(pk[1], S.sc64[1], cw, lane, tot1);
+    uint32_t nnz = 0, koff[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      koff[k] = nnz + (uint32_t)(((k < 4 ? ex0 : ex1) >> (16 * (k & 3))) & 0xFFFF);
+      nnz += (uint32_t)(((k < 4 ? tot0 : tot1) >> (16 * (k & 3))) & 0xFFFF);
+    }
+    if ((int32_t)nnz != s1) bad = 1;  // nz(D) must end where nr(B1) starts
+    if (bad) {  // every compute thread reached the same verdict from the same smem data
+      if (g == 0) record_error(ctx, DERR_CORRUPT);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_in[s]);
+      bar_r();  // keep the barrier count of every compute warp in step
+      continue;
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint32_t u = g + kRT * k;
+      if (u >= NU) continue;
+      uint32_t wv[4] = {0, 0, 0, 0}, p = koff[k];
+#pragma unroll
+      for (int b = 0; b < 16; ++b)
+        if ((ub[k] >> b) & 1) wv[b >> 2] |= (uint32_t)in[p++] << (8 * (b & 3));
+      reinterpret_cast<uint4*>(S.T)[u] = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[s]);  // payload fully consumed
+    bar_r();
+    // ---- BIT⁻¹ (rows out reversed) and DIFFMS⁻¹ (serial + CTA scan) ----
+    uint32_t X[32];
+    uint32_t tot = 0;
+    if (g < G) {
+#pragma unroll
+      for (int p = 0; p < 32; ++p) X[p] = S.T[p * G + g];
+      transpose32(X);
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {  // U[i] = A'[31−i]
+        const uint32_t tmp = X[i];
+        X[i] = X[31 - i];
+        X[31 - i] = tmp;
+      }
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        tot += tcms_inv(X[i]);
+        X[i] = tot;
+      }
+    } else if (g == G && (m & 31)) {
+      for (uint32_t i = 32 * G; i < m; ++i) tot += tcms_inv(S.T[i]);
+    }
+    uint32_t all;
+    const uint32_t base = cta_excl_scan<uint32_t>(tot, S.sc32[1], cw, lane, all);
+    if (g < G) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) S.X[g * 33 + i] = X[i] + base;
+    } else if (g == G && (m & 31)) {
+      uint32_t run = base;
+      for (uint32_t i = 32 * G; i < m; ++i) {
+        run += tcms_inv(S.T[i]);
+        S.X[G * 33 + (i - 32 * G)] = run;
+      }
+    }
+    bar_r();
+    // coalesced 16-byte stores of words n = 4q .. 4q+3
+    for (uint32_t q = g; q < 1024; q += kRT) {
+      const uint32_t n = 4 * q;
+      if (n >= m) break;
+      const uint32_t* row = S.X + (n >> 5) * 33 + (n & 31);
+      if (n + 4 <= m) {
+        __stcs(reinterpret_cast<uint4*>(dst) + q, make_uint4(row[0], row[1], row[2], row[3]));
+      } else {
+        for (uint32_t j = 0; n + j < m; ++j) dst[n + j] = row[j];
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kRDecThreads) spratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  RDecSmem& S = *reinterpret_cast<RDecSmem*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kRDecStages; ++i) {
+      mbar_init(&S.full_in[i], 1);
+      mbar_init(&S.empty_in[i], kRW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0) dec_loader<kRDecStages, kRDecBatch>(S, a, ctx, lane, 4);
+  else r_dec_compute(S, a, ctx, warp - 1, lane);
+}
+
+}  // namespace
+
+void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st) {
+  const size_t smem = sizeof(REncSmem);
+  static const bool init = [&] {
+    cudaFuncSetAttribute(spratio_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return true;
+  }();
+  (void)init;
+  const int grid = persistent_grid(spratio_encode_kernel, kREncThreads, smem, a.n_chunks);
+  spratio_encode_kernel<<<grid, kREncThreads, smem, st>>>(a, ctx);
+}
+
+void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st) {
+  const size_t smem = sizeof(RDecSmem);
+  static const bool init = [&] {
+    cudaFuncSetAttribute(spratio_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return true;
+  }();
+  (void)init;
+  const int grid = persistent_grid(spratio_decode_kernel, kRDecThreads, smem, (max_chunks + kRDecBatch - 1) / kRDecBatch);
+  spratio_decode_kernel<<<grid, kRDecThreads, smem, st>>>(a, ctx);
+}
+
+}  // namespace lcf

@@ -156,6 +156,14 @@ EncArgs enc_args(int algo, const void* in, uint64_t in_bytes) {
 
 lcf_status_t enqueue_encode(Workspace* ws, EncArgs& a) {
   if (lcf_status_t s = grow(ws->status, ws->status_cap, a.n_chunks, ws->stream, true)) return s;
+  if (a.algo == LCF_DPRATIO) {
+    const size_t need = dpratio_fcm_workspace(a.n_words_total);
+    if (lcf_status_t s = grow(reinterpret_cast<uint8_t*&>(ws->scratch[2]), ws->scratch_cap[2], need, ws->stream, false))
+      return s;
+    LaunchCtx ctx = make_ctx(ws);
+    g_launches += launch_dpratio_encode(a, ctx, ws->scratch[2], ws->scratch_cap[2], ws->stream);
+    return last_launch_status();
+  }
   LaunchCtx ctx = make_ctx(ws);
   switch (a.algo) {
     case LCF_SPSPEED: launch_speed_encode<uint32_t>(a, ctx, ws->stream); break;
@@ -195,7 +203,7 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
   if (in_bytes % wb || !d_out || !aligned16(d_out) || (in_bytes && (!d_in || !aligned16(d_in))))
     return LCF_ERROR_INVALID_ARGUMENT;
   if (out_capacity < lcf_max_compressed_size(algo, dtype, in_bytes)) return LCF_ERROR_BUFFER_TOO_SMALL;
-  if (algo == LCF_DPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
+  if (algo == LCF_DPRATIO && in_bytes / 8 >= (1ull << 31)) return LCF_ERROR_INVALID_ARGUMENT;  // CUB sort index
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
@@ -237,7 +245,6 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   if (!d_in || !aligned16(d_in) || (out_capacity && (!d_out || !aligned16(d_out))))
     return LCF_ERROR_INVALID_ARGUMENT;
   if (in_bytes < kHeaderBytes) return LCF_ERROR_CORRUPT_STREAM;
-  if (algo == LCF_DPRATIO) return LCF_ERROR_INVALID_ARGUMENT;  // TODO
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
@@ -259,11 +266,13 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
     }
   } else {
     const uint64_t by_table = (in_bytes - kHeaderBytes) / 4;
-    const uint64_t by_out = (out_capacity + kChunkBytes - 1) / kChunkBytes;
+    const uint64_t by_out = (algo == LCF_DPRATIO ? 2 : 1) * ((out_capacity + kChunkBytes - 1) / kChunkBytes);
     grid = by_table < by_out ? by_table : by_out;
     if (grid == 0) grid = 1;  // still validate the header on the device
   }
   if (lcf_status_t s = grow(ws->status, ws->status_cap, grid, stream, true)) return s;
+  if (algo == LCF_DPRATIO)
+    if (lcf_status_t s = grow(ws->tile_flag, ws->tile_cap, grid / 2 + 1, stream, true)) return s;
   DecArgs a{};
   a.stream = static_cast<const uint8_t*>(d_in);
   a.stream_bytes = in_bytes;
@@ -271,11 +280,13 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   a.out_capacity = out_capacity;
   a.algo = (uint32_t)algo;
   a.word_bytes = word_bytes_of(algo);
+  a.tile_flag = ws->tile_flag;
   LaunchCtx ctx = make_ctx(ws);
   switch (algo) {
     case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, grid, stream); break;
     case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, grid, stream); break;
     case LCF_SPRATIO: launch_spratio_decode(a, ctx, grid, stream); break;
+    case LCF_DPRATIO: launch_dpratio_decode(a, ctx, grid / 2 + 1, stream); break;
     default: return LCF_ERROR_INVALID_ARGUMENT;
   }
   ++g_launches;

@@ -1,0 +1,784 @@
+// lcf_dpratio.cu — DPratio = per chunk (RARE ∘ RAZE ∘ DIFFMS₆₄) over FCM(x)
+// (§3.2) on sm_100a.
+//
+// Compress (4 launches):
+//   fcm_hash_kernel   h(i) from x[i−1..i−3] (A-13) and the index, coalesced
+//   CUB radix sort    (h, i) pairs on the 20 key bits — stable, so equal hashes
+//                     stay in index order (L197: "we use the CUB library")
+//   fcm_match_kernel  per sorted position: the nearest of the 4 preceding pairs
+//                     with the same hash and the same 64-bit word (A-14); the
+//                     block stages its sorted window and the gathered words in
+//                     shared memory, then scatters the 32-bit distance
+//   dpratio_encode    persistent pipeline; item = 2048-word tile t → chunk 2t
+//                     (V) and 2t+1 (Dist) (A-16); per chunk DIFFMS₆₄ → RAZE →
+//                     RARE in shared memory (L201: histogram of leading-zero
+//                     counts by warp-aggregated shared atomics; k from the prefix
+//                     sums; bit fields emitted with warp segmented scans)
+// Decompress (1 launch): dpratio_decode — per tile: RARE⁻¹ → RAZE⁻¹ → DIFFMS⁻¹
+//   for V and Dist, then the FCM decode of the tile (L197) fused in: references
+//   inside the tile are resolved by pointer jumping in shared memory, references
+//   to earlier tiles read the already written output after an acquire on that
+//   tile's completion flag (tiles complete in ticket order, so no cycles).
+#include <cub/cub.cuh>
+
+#include "lcf_persist.cuh"
+
+namespace lcf {
+namespace {
+
+constexpr int kDW = 8;                 // compute warps
+constexpr uint32_t kDT = kDW * 32;     // compute threads
+constexpr int kDOut = 2, kDBatch = 4;  // output slots (encode), tiles per ticket (decode)
+constexpr int kDEncThreads = (2 + kDW) * 32, kDDecThreads = (1 + kDW) * 32;
+constexpr uint32_t kBarD = 1;
+constexpr uint32_t kTileWords = 2048;
+constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
+
+__device__ __forceinline__ void bar_d() { named_bar_sync(kBarD, kDT); }
+__device__ __forceinline__ bool bar_d_or(bool p) {
+  uint32_t r;
+  asm volatile("{\n .reg .pred pi, po;\n setp.ne.u32 pi, %1, 0;\n bar.red.or.pred po, %2, %3, pi;\n selp.u32 %0, 1, 0, po;\n}"
+               : "=r"(r)
+               : "r"((uint32_t)p), "r"(kBarD), "r"(kDT)
+               : "memory");
+  return r != 0;
+}
+
+// =============================== FCM encode kernels ===============================
+__global__ void fcm_hash_kernel(const uint64_t* __restrict__ x, uint64_t n, uint32_t* __restrict__ key,
+                                uint32_t* __restrict__ idx) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t a = i >= 1 ? x[i - 1] : 0, b = i >= 2 ? x[i - 2] : 0, c = i >= 3 ? x[i - 3] : 0;
+    key[i] = (uint32_t)(((a * FCM_K1) ^ (b * FCM_K2) ^ (c * FCM_K3)) >> 44);
+    idx[i] = (uint32_t)i;
+  }
+}
+
+constexpr int kMatchBlock = 256;
+__global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
+                                                                const uint32_t* __restrict__ key,
+                                                                const uint32_t* __restrict__ idx,
+                                                                uint32_t* __restrict__ dist) {
+  __shared__ uint32_t sk[kMatchBlock + 4], si[kMatchBlock + 4];
+  __shared__ uint64_t sx[kMatchBlock + 4];
+  for (uint64_t b0 = blockIdx.x * (uint64_t)kMatchBlock; b0 < n; b0 += (uint64_t)gridDim.x * kMatchBlock) {
+    // window: sorted positions [b0 − 4, b0 + kMatchBlock)
+    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {
+      const int64_t k = (int64_t)b0 - 4 + j;
+      if (k >= 0 && (uint64_t)k < n) {
+        sk[j] = key[k];
+        si[j] = idx[k];
+        sx[j] = x[si[j]];  // gathered once per sorted position
+      } else {
+        sk[j] = 0xFFFFFFFFu;  // never equals a 20-bit hash
+      }
+    }
+    __syncthreads();
+    const uint64_t k = b0 + threadIdx.x;
+    if (k < n) {
+      const int j = threadIdx.x + 4;
+      const uint32_t h = sk[j], i = si[j];
+      const uint64_t xi = sx[j];
+      uint32_t d = 0;
+#pragma unroll
+      for (int back = 1; back <= 4; ++back) {  // nearest first (A-14, pinned by Fig. 6)
+        if (sk[j - back] == h && sx[j - back] == xi) {
+          d = i - si[j - back];
+          break;
+        }
+      }
+      dist[i] = d;
+    }
+    __syncthreads();
+  }
+}
+
+// ============================ RAZE / RARE in shared memory ============================
+struct AdaptScratch {
+  uint32_t hist[65];
+  uint32_t cnt[64];     // per (round, warp) set counts → exclusive prefix
+  uint32_t b1[64];      // B1 bitmap words (n ≤ 2048 bits)
+  uint32_t k, flag, s1, s2;
+};
+
+__device__ __forceinline__ uint64_t ld_u64(const uint8_t* p) { return *reinterpret_cast<const uint64_t*>(p); }
+__device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
+
+// 64-bit field of width w (≤ 64) at bit position P of the little-endian word
+// stream at `base` (4-byte aligned; reads up to 12 bytes).
+__device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, uint32_t w) {
+  if (w == 0) return 0;
+  const uint32_t* p = base + (P >> 5);
+  const uint32_t r = P & 31;
+  const uint32_t lo = __funnelshift_r(p[0], p[1], r), hi = __funnelshift_r(p[1], p[2], r);
+  const uint64_t v = ((uint64_t)hi << 32) | lo;
+  return w >= 64 ? v : v & ((1ull << w) - 1);
+}
+
+// Encode L bytes at src (8-byte aligned) with RAZE (rare = false, L189) or RARE
+// (rare = true, L195) into dst (16-byte aligned, ≥ L + 3 + 32 bytes). All kDT
+// compute threads call it; returns the output length (FORMAT.md §6.2–6.3).
+__device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare, AdaptScratch& sc,
+                                    uint32_t tid) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  const uint32_t n = L / 8, tl = L % 8;
+  if (tid < 65) sc.hist[tid] = 0;
+  if (tid < 64) sc.b1[tid] = 0;
+  bar_d();
+  // ---- histogram of clz(v_i ⊕ ref_i), warp-aggregated shared atomics ----
+  uint64_t v[8], ref[8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const uint32_t i = tid + kDT * r;
+    v[r] = i < n ? ld_u64(src + 8 * i) : 0;
+    ref[r] = (rare && i < n && i > 0) ? ld_u64(src + 8 * (i - 1)) : 0;
+    const uint32_t z = i < n ? clz64(v[r] ^ ref[r]) : 65u;
+    const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
+    if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
+  }
+  bar_d();
+  // ---- k* = smallest argmin of est(k) = k·nz(k) + (64−k)·n, k ∈ 1..64 (A-17, A-18) ----
+  if (warp == 0) {
+    const uint32_t c0 = sc.hist[2 * lane], c1 = sc.hist[2 * lane + 1];
+    uint32_t s = c0 + c1;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, d);
+      if ((int)lane >= d) s += y;
+    }
+    const uint32_t before = s - c0 - c1;
+    const uint32_t kA = 2 * lane + 1, kB = 2 * lane + 2;  // nz(kA) = before + c0, nz(kB) = s
+    const uint32_t eA = kA * (before + c0) + (64 - kA) * n, eB = kB * s + (64 - kB) * n;
+    const uint32_t keyA = (eA << 7) | kA, keyB = (eB << 7) | kB;
+    const uint32_t best = __reduce_min_sync(0xFFFFFFFFu, keyA < keyB ? keyA : keyB);
+    if (lane == 0) sc.k = best & 127;
+  }
+  bar_d();
+  const uint32_t k = sc.k;
+  // ---- B1 bits and ranks (word i = tid + 256 r: warp ballots are B1 words) ----
+  uint64_t top[8];
+  uint32_t bal[8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const uint32_t i = tid + kDT * r;
+    top[r] = k == 64 ? v[r] : (v[r] >> (64 - k));
+    const uint64_t tref = k == 64 ? ref[r] : (ref[r] >> (64 - k));
+    const bool set = i < n && top[r] != tref;
+    bal[r] = __ballot_sync(0xFFFFFFFFu, set);
+    if (lane == 0) {
+      sc.b1[r * kDW + warp] = bal[r];
+      sc.cnt[r * kDW + warp] = __popc(bal[r]);
+    }
+  }
+  bar_d();
+  uint32_t nr1 = 0, nr2 = 0, b2 = 0, b3 = 0, c1m = 0, off1 = 0, b1w0 = 0, b1w1 = 0;
+  const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
+  if (warp == 0) {
+    // prefix of the 64 per-(round, warp) counts
+    const uint32_t a0 = sc.cnt[2 * lane], a1 = sc.cnt[2 * lane + 1];
+    uint32_t s = a0 + a1;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, d);
+      if ((int)lane >= d) s += y;
+    }
+    sc.cnt[2 * lane] = s - a0 - a1;
+    sc.cnt[2 * lane + 1] = s - a1;
+    const uint32_t nset = __shfl_sync(0xFFFFFFFFu, s, 31);
+    // B1 → B2 (lane: B1 bytes [8·lane, 8·lane+8) = words 2·lane, 2·lane+1)
+    b1w0 = sc.b1[2 * lane];
+    b1w1 = sc.b1[2 * lane + 1];
+    const uint32_t prevb = __shfl_up_sync(0xFFFFFFFFu, b1w1 >> 24, 1);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const uint32_t cur = ((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3))) & 0xFF;
+      const uint32_t pre = j ? (((j - 1) < 4 ? b1w0 : b1w1) >> (8 * ((j - 1) & 3))) & 0xFF : (lane ? prevb : 0u);
+      if (cur != pre && 8 * lane + j < L1) c1m |= 1u << j;
+    }
+    b2 = c1m;  // B2 byte `lane`
+    uint32_t x = __popc(c1m);
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+      if ((int)lane >= d) x += y;
+    }
+    off1 = x - __popc(c1m);
+    nr1 = __shfl_sync(0xFFFFFFFFu, x, 31);
+    const uint32_t pb2 = __shfl_up_sync(0xFFFFFFFFu, b2, 1);
+    b3 = __ballot_sync(0xFFFFFFFFu, lane < L2 && b2 != (lane ? pb2 : 0u));
+    nr2 = __popc(b3);
+    const uint32_t hib = (nset * k + 7) / 8, lob = (n * (64 - k) + 7) / 8;
+    const uint32_t total = 3 + hib + lob + tl + nr1 + nr2 + L3;
+    if (lane == 0) {
+      sc.flag = total >= 3 + L;  // bypass (A-23)
+      sc.s1 = total;
+      sc.s2 = hib;
+    }
+  }
+  bar_d();
+  const bool bypass = sc.flag;
+  const uint32_t total = sc.s1, hib = sc.s2;
+  if (bypass) {
+    for (uint32_t j = tid; j < L; j += kDT) dst[3 + j] = src[j];
+    if (tid == 0) {
+      dst[0] = (uint8_t)L;
+      dst[1] = (uint8_t)(L >> 8);
+      dst[2] = 0;
+    }
+    bar_d();
+    return 3 + L;
+  }
+  uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
+  for (uint32_t j = tid; j < (total + 7) / 4 + 1; j += kDT) dw[j] = 0;
+  bar_d();
+  // ---- HI: top fields of the set words (rank order), LO: low fields of all words ----
+  const uint64_t hi_base = 24, lo_base = 8ull * (3 + hib);
+  const uint32_t wl = 64 - k;
+  const uint64_t lmask = wl >= 64 ? ~0ull : ((1ull << wl) - 1);
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const uint32_t i = tid + kDT * r;
+    const bool set = (bal[r] >> lane) & 1;
+    const uint32_t rank = sc.cnt[r * kDW + warp] + __popc(bal[r] & ((1u << lane) - 1));
+    emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? top[r] : 0, 0, true);
+    if (wl) emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, i < n ? (v[r] & lmask) : 0, 0, true);
+  }
+  bar_d();
+  // ---- header, tail bytes, nr(B1), nr(B2), B3 ----
+  const uint32_t after = 3 + hib + (n * wl + 7) / 8;
+  if (tid == 0) {
+    dst[0] = (uint8_t)L;
+    dst[1] = (uint8_t)(L >> 8);
+    dst[2] = (uint8_t)k;
+  }
+  if (tid < tl) dst[after + tid] = src[8 * n + tid];
+  if (warp == 0) {
+    uint32_t p = after + tl + off1;
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if ((c1m >> j) & 1) dst[p++] = (uint8_t)((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
+    if ((b3 >> lane) & 1) dst[after + tl + nr1 + __popc(b3 & ((1u << lane) - 1))] = (uint8_t)b2;
+    if (lane < L3) dst[total - L3 + lane] = (uint8_t)(b3 >> (8 * lane));
+  }
+  bar_d();
+  return total;
+}
+
+// Decode a RAZE/RARE stream of `len` bytes at src (16-byte aligned, ≥ 16 bytes
+// of readable slack) into dst (8-byte aligned, capacity cap). Returns the
+// decoded length or −1 if malformed. All kDT compute threads call it.
+__device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, uint32_t cap, bool rare,
+                               AdaptScratch& sc, uint32_t tid) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  if (len < 3) return -1;
+  const uint32_t L = src[0] | ((uint32_t)src[1] << 8), k = src[2];
+  if (L > cap) return -1;
+  if (k == 0) {
+    if (len != 3 + L) return -1;
+    for (uint32_t j = tid; j < L; j += kDT) dst[j] = src[3 + j];
+    bar_d();
+    return (int)L;
+  }
+  if (k > 64) return -1;
+  const uint32_t n = L / 8, tl = L % 8, L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
+  const uint32_t wl = 64 - k;
+  if (warp == 0) {
+    int bad = len < 3 + L3;
+    uint32_t b3 = 0;
+    if (!bad)
+      for (uint32_t j = 0; j < L3; ++j) b3 |= (uint32_t)src[len - L3 + j] << (8 * j);
+    const uint32_t v2 = L2 >= 32 ? 0xFFFFFFFFu : ((1u << L2) - 1u);
+    const int32_t s2 = (int32_t)len - (int32_t)L3 - __popc(b3 & v2);
+    if (s2 < 3) bad = 1;
+    const uint32_t r2 = __popc(b3 & v2 & (0xFFFFFFFFu >> (31 - lane)));
+    const uint32_t b2 = (!bad && lane < L2 && r2) ? src[s2 + r2 - 1] : 0u;  // B2 byte `lane`
+    // B1 bytes [8·lane, 8·lane+8) from the bits of B2 byte `lane`
+    const uint32_t vb = (8 * lane >= L1) ? 0u : (L1 - 8 * lane >= 8 ? 0xFFu : ((1u << (L1 - 8 * lane)) - 1u));
+    const uint32_t bits = b2 & vb;
+    uint32_t x = __popc(bits);
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+      if ((int)lane >= d) x += y;
+    }
+    const int32_t s1 = s2 - (int32_t)__shfl_sync(0xFFFFFFFFu, x, 31);
+    if (s1 < 3) bad = 1;
+    bad = __any_sync(0xFFFFFFFFu, bad);
+    uint32_t r = x - __popc(bits), w0 = 0, w1 = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      r += (bits >> j) & 1;
+      const uint32_t val = (!bad && r) ? src[s1 + r - 1] : 0u;
+      if (j < 4) w0 |= val << (8 * j);
+      else w1 |= val << (8 * (j - 4));
+    }
+    // B1 words cover bits 64·lane .. : mask bits ≥ n
+    const uint32_t nb0 = n > 64 * lane ? n - 64 * lane : 0;
+    if (nb0 < 32) w0 &= nb0 ? ((1u << nb0) - 1u) : 0u;
+    if (nb0 < 64) w1 &= nb0 > 32 ? ((1u << (nb0 - 32)) - 1u) : 0u;
+    sc.b1[2 * lane] = w0;
+    sc.b1[2 * lane + 1] = w1;
+    const uint32_t cw0 = __popc(w0), cw1 = __popc(w1);
+    uint32_t c = cw0 + cw1;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, c, d);
+      if ((int)lane >= d) c += y;
+    }
+    sc.cnt[2 * lane] = c - cw0 - cw1;
+    sc.cnt[2 * lane + 1] = c - cw1;
+    const uint32_t nset = __shfl_sync(0xFFFFFFFFu, c, 31);
+    const uint32_t hib = (nset * k + 7) / 8, lob = (n * wl + 7) / 8;
+    if (!bad && (int32_t)(3 + hib + lob + tl) != s1) bad = 1;
+    if (lane == 0) {
+      sc.flag = bad;
+      sc.s2 = hib;
+    }
+  }
+  bar_d();
+  if (sc.flag) return -1;
+  const uint32_t hib = sc.s2;
+  const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
+  const uint64_t lo_base = 8ull * (3 + hib);
+  // word i = 32·(b1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const uint32_t i = tid + kDT * r;
+    const uint32_t q = r * kDW + warp;
+    const uint32_t bw = sc.b1[q];
+    const uint32_t re = sc.cnt[q] + __popc(bw & ((1u << lane) - 1));  // set words before i
+    const bool set = (bw >> lane) & 1;
+    if (i < n) {
+      uint64_t tp;
+      if (rare) {
+        const uint32_t ri = re + set;  // set words up to and including i
+        tp = ri ? get_field(sw, 24 + (uint64_t)(ri - 1) * k, k) : 0;
+      } else {
+        tp = set ? get_field(sw, 24 + (uint64_t)re * k, k) : 0;
+      }
+      const uint64_t lw = get_field(sw, lo_base + (uint64_t)i * wl, wl);
+      *reinterpret_cast<uint64_t*>(dst + 8 * i) = k == 64 ? tp : ((tp << wl) | lw);
+    }
+  }
+  if (tid < tl) dst[8 * n + tid] = src[lo_base / 8 + (n * wl + 7) / 8 + tid];
+  bar_d();
+  return (int)L;
+}
+
+// CTA-wide exclusive scan of u64 over the kDT compute threads (slot `sh`).
+__device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t* sh, uint32_t tid, uint64_t& total) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  uint64_t x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+    if ((int)lane >= d) x += y;
+  }
+  if (lane == 31) sh[warp] = x;
+  bar_d();
+  uint64_t base = 0;
+  total = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < kDW; ++i) {
+    const uint64_t s = sh[i];
+    if (i < warp) base += s;
+    total += s;
+  }
+  bar_d();  // the slot may be reused right away
+  return base + x - v;
+}
+
+// =================================== encode ======================================
+struct DEncSmem {
+  alignas(128) uint64_t xin[kTileWords];        // stage: x tile
+  alignas(128) uint32_t din[kTileWords];        // stage: FCM distances of the tile
+  alignas(128) uint64_t w[kTileWords + 8];      // DIFFMS words of V or Dist
+  alignas(128) uint8_t rz[kChunkBytes + 128];   // RAZE output
+  alignas(128) uint32_t out[kDOut][(kChunkBytes + 128) / 4];
+  uint64_t full_in[1], empty_in[1], full_out[kDOut], empty_out[kDOut];
+  uint64_t in_chunk[1], out_chunk[kDOut];
+  uint32_t out_len[kDOut], out_raw[kDOut];
+  AdaptScratch sc;
+};
+
+__device__ __forceinline__ void d_enc_loader(DEncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane) {
+  const uint64_t T = a.n_chunks / 2;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t ph = it & 1;
+    mbar_wait(&S.empty_in[0], ph ^ 1);
+    uint64_t t = 0;
+    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
+    t = __shfl_sync(0xFFFFFFFFu, t, 0);
+    if (t >= T) {
+      if (lane == 0) {
+        S.in_chunk[0] = kNoChunk;
+        mbar_arrive(&S.full_in[0]);
+        ticket_retire(ctx);
+      }
+      return;
+    }
+    const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
+    const uint64_t* xs = reinterpret_cast<const uint64_t*>(a.in) + t * kTileWords;
+    const uint32_t* ds = a.fcm_dist + t * kTileWords;
+    if ((m & 3) == 0) {
+      if (lane == 0) {
+        S.in_chunk[0] = t;
+        mbar_arrive_expect_tx(&S.full_in[0], 12 * m);
+        tma_load_1d(S.xin, xs, 8 * m, &S.full_in[0]);
+        tma_load_1d(S.din, ds, 4 * m, &S.full_in[0]);
+      }
+    } else {
+      for (uint32_t i = lane; i < m; i += 32) {
+        S.xin[i] = xs[i];
+        S.din[i] = ds[i];
+      }
+      if (lane == 0) S.in_chunk[0] = t;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.full_in[0]);
+    }
+  }
+}
+
+__device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t tid) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  uint32_t oit = 0;  // output-slot iteration (two chunks per tile)
+  for (uint32_t it = 0;; ++it) {
+    mbar_wait(&S.full_in[0], it & 1);
+    const uint64_t t = S.in_chunk[0];
+    if (t == kNoChunk) {
+      enc_forward_end<kDOut, 1>(S, oit, warp, lane);
+      return;
+    }
+    const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
+    for (uint32_t part = 0; part < 2; ++part, ++oit) {  // chunk 2t: V, chunk 2t+1: Dist (A-16)
+      const uint64_t c = 2 * t + part;
+      // FCM outputs (L170–185) and DIFFMS₆₄ (L187) into w[]
+      for (uint32_t i = tid; i < m; i += kDT) {
+        const uint32_t d = S.din[i], dp = i ? S.din[i - 1] : 0u;
+        uint64_t cur, prev;
+        if (part == 0) {
+          cur = d ? 0ull : S.xin[i];
+          prev = i ? (dp ? 0ull : S.xin[i - 1]) : 0ull;
+        } else {
+          cur = d;
+          prev = i ? (uint64_t)dp : 0ull;
+        }
+        S.w[i] = tcms((uint64_t)(cur - prev));
+      }
+      bar_d();
+      // RAZE then RARE (L189–201)
+      const uint32_t l1 = adaptive_encode(reinterpret_cast<const uint8_t*>(S.w), 8 * m, S.rz, false, S.sc, tid);
+      const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
+      mbar_wait(&S.empty_out[o], pho ^ 1);
+      uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
+      const uint32_t l2 = adaptive_encode(S.rz, l1, ob, true, S.sc, tid);
+      const uint32_t raw_len = 8 * m;
+      const bool raw = l2 >= raw_len;  // L104, ties → raw
+      const uint32_t len = raw ? raw_len : l2;
+      if (raw) {  // the V / Dist words themselves
+        for (uint32_t i = tid; i < m; i += kDT)
+          reinterpret_cast<uint64_t*>(ob)[i] = part == 0 ? (S.din[i] ? 0ull : S.xin[i]) : (uint64_t)S.din[i];
+        if (tid < 2 && (m & 1)) reinterpret_cast<uint64_t*>(ob)[m + tid] = 0;  // round16 pad
+      } else if (tid < 16 && len + tid < round16(len)) {
+        ob[len + tid] = 0;
+      }
+      if (tid == 0) {
+        lookback_publish(ctx, c, round16(len));
+        S.out_chunk[o] = c;
+        S.out_len[o] = len;
+        S.out_raw[o] = raw;
+      }
+      fence_proxy_async_smem();
+      bar_d();
+      if (lane == 0) mbar_arrive(&S.full_out[o]);
+    }
+    if (lane == 0) mbar_arrive(&S.empty_in[0]);
+  }
+}
+
+__global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    mbar_init(&S.full_in[0], 1);
+    mbar_init(&S.empty_in[0], kDW);
+    for (int i = 0; i < kDOut; ++i) {
+      mbar_init(&S.full_out[i], kDW);
+      mbar_init(&S.empty_out[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0) d_enc_loader(S, a, ctx, lane);
+  else if (warp == 1) enc_storer<kDOut, 1>(S, a, ctx, lane, 0);
+  else d_enc_compute(S, a, ctx, threadIdx.x - 64);
+}
+
+// =================================== decode ======================================
+struct DDecSmem {
+  alignas(128) uint8_t in[2][kChunkBytes + 128];  // stage: V and Dist payloads of a tile
+  alignas(128) uint8_t rz[kChunkBytes + 128];     // RARE⁻¹ output (RAZE stream)
+  alignas(128) uint64_t V[kTileWords + 8];        // V, then the decoded tile in place
+  alignas(128) uint64_t D[kTileWords + 8];
+  int32_t pj[2][kDT];                             // pointer jumping: target (−1 done)
+  uint64_t vj[2][kDT];
+  uint64_t full_in[1], empty_in[1];
+  uint64_t tile[1];
+  uint32_t len[1][2], flags[1];
+  uint64_t scan[kDW];
+  AdaptScratch sc;
+  int32_t bad;
+};
+
+__device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t lane) {
+  uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
+  const bool hdr_ok = read_header(a, ctx, n_words, n_chunks, base, payload);
+  const bool small = hdr_ok && n_words * 8 > a.out_capacity;
+  const uint64_t T = n_chunks / 2;
+  uint32_t it = 0;
+  for (;;) {
+    uint64_t tb = 0;
+    if (lane == 0) tb = atomicAdd(ctx.ticket, 1ull);
+    tb = __shfl_sync(0xFFFFFFFFu, tb, 0) * kDBatch;
+    if (!hdr_ok || small || tb >= T) {
+      mbar_wait(&S.empty_in[0], (it & 1) ^ 1);
+      if (lane == 0) {
+        if (tb == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
+        if (tb == 0 && small) record_error(ctx, DERR_SMALL);
+        S.tile[0] = kNoChunk;
+        mbar_arrive(&S.full_in[0]);
+        ticket_retire(ctx);
+      }
+      return;
+    }
+    const uint32_t nb = (uint32_t)umin64(kDBatch, T - tb);  // tiles; chunks 2tb .. 2tb + 2nb − 1
+    const uint64_t c = 2 * tb + lane;
+    uint32_t len = 0, raw = 0;
+    bool bad = false;
+    if (lane < 2 * nb) {
+      const uint32_t e = reinterpret_cast<const uint32_t*>(a.stream + kHeaderBytes)[c];
+      len = e & ~kRawFlag;
+      raw = e >> 31;
+      const uint32_t m = (uint32_t)umin64(kTileWords, n_words - (c / 2) * kTileWords);
+      bad = raw ? len != 8 * m : len >= 8 * m;
+      lookback_publish(ctx, c, bad ? 0 : round16(len));
+    }
+    const uint64_t agg = (lane < 2 * nb && !bad) ? round16(len) : 0;
+    uint64_t x = agg;
+#pragma unroll
+    for (int d = 1; d < 2 * kDBatch; d <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+      if ((int)lane >= d) x += y;
+    }
+    x -= agg;
+    const uint64_t base_b = lookback_warp(ctx, 2 * tb, __shfl_sync(0xFFFFFFFFu, agg, 0));
+    const uint64_t excl = base_b + x;
+    if (lane > 0 && lane < 2 * nb) st_relaxed_u64(ctx.status + c, make_status(kFlagInc, ctx.epoch, excl + agg));
+    const uint64_t end = excl + round16(len);
+    if (lane < 2 * nb && !bad && (end > payload || (c == n_chunks - 1 && end != payload))) bad = true;
+    for (uint32_t j = 0; j < nb; ++j, ++it) {
+      const uint32_t l0 = __shfl_sync(0xFFFFFFFFu, len, 2 * j), l1 = __shfl_sync(0xFFFFFFFFu, len, 2 * j + 1);
+      const uint32_t r0 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j), r1 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j + 1);
+      const bool b0 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j), b1 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j + 1);
+      const uint64_t e0 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j), e1 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j + 1);
+      mbar_wait(&S.empty_in[0], (it & 1) ^ 1);
+      if (lane == 0) {
+        const bool bb = b0 || b1;
+        if (bb) record_error(ctx, DERR_CORRUPT);
+        S.tile[0] = tb + j;
+        S.len[0][0] = l0;
+        S.len[0][1] = l1;
+        S.flags[0] = r0 | (r1 << 1) | (bb ? 4u : 0u);
+        const uint32_t tx = bb ? 0 : (uint32_t)(round16(l0) + round16(l1));
+        if (tx) {
+          mbar_arrive_expect_tx(&S.full_in[0], tx);
+          if (l0) tma_load_1d(S.in[0], a.stream + base + e0, (uint32_t)round16(l0), &S.full_in[0]);
+          if (l1) tma_load_1d(S.in[1], a.stream + base + e1, (uint32_t)round16(l1), &S.full_in[0]);
+        } else {
+          mbar_arrive(&S.full_in[0]);
+        }
+      }
+    }
+  }
+}
+
+// One chunk of a tile: RARE⁻¹ → RAZE⁻¹ → DIFFMS⁻¹ into arr[0..m). Returns false
+// if malformed.
+__device__ __forceinline__ bool d_decode_chunk(DDecSmem& S, const uint8_t* pay, uint32_t len, bool raw, uint32_t m,
+                                               uint64_t* arr, uint32_t tid) {
+  if (raw) {
+    for (uint32_t i = tid; i < m; i += kDT) arr[i] = reinterpret_cast<const uint64_t*>(pay)[i];
+    bar_d();
+    return true;
+  }
+  const int l1 = adaptive_decode(pay, len, S.rz, kChunkBytes + 3, true, S.sc, tid);
+  if (l1 < 0) return false;
+  const int l0 = adaptive_decode(S.rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, S.sc, tid);
+  if (l0 != (int)(8 * m)) return false;
+  // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8)
+  uint64_t v[8], run = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint32_t i = 8 * tid + j;
+    v[j] = i < m ? tcms_inv(arr[i]) : 0;
+    run += v[j];
+  }
+  uint64_t tot;
+  uint64_t acc = cta_scan_u64(run, S.scan, tid, tot);
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint32_t i = 8 * tid + j;
+    acc += v[j];
+    if (i < m) arr[i] = acc;
+  }
+  bar_d();
+  return true;
+}
+
+__device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t tid) {
+  const uint32_t lane = tid & 31;
+  const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
+  const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / 8;
+  uint64_t* out = reinterpret_cast<uint64_t*>(a.out);
+  for (uint32_t it = 0;; ++it) {
+    mbar_wait(&S.full_in[0], it & 1);
+    const uint64_t t = S.tile[0];
+    if (t == kNoChunk) return;
+    const uint32_t fl = S.flags[0];
+    const uint32_t m = (uint32_t)umin64(kTileWords, n_words - t * kTileWords);
+    bool ok = !(fl & 4);
+    if (ok) ok = d_decode_chunk(S, S.in[0], S.len[0][0], fl & 1, m, S.V, tid);
+    if (ok) ok = d_decode_chunk(S, S.in[1], S.len[0][1], (fl >> 1) & 1, m, S.D, tid);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[0]);
+    // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
+    const uint64_t t0 = t * kTileWords;
+    bool bad = !ok;
+    if (ok) {
+      for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
+        const uint32_t li = b + tid;
+        int32_t p = -1;
+        uint64_t val = 0;
+        if (li < m) {
+          const uint64_t d = S.D[li], gi = t0 + li;
+          if (d == 0) {
+            val = S.V[li];
+          } else if (d > gi || S.V[li] != 0) {
+            bad = true;
+          } else if (gi - d >= t0 + b) {
+            p = (int32_t)(gi - d - t0 - b);  // inside this block: resolve below
+          } else if (gi - d >= t0) {
+            val = S.V[gi - d - t0];  // earlier block of this tile: already final
+          } else {  // earlier tile: wait for its completion flag, then read the output
+            const uint64_t j = gi - d, tj = j / kTileWords;
+            while (ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
+            val = ld_cg_u64(out + j);
+          }
+        }
+        // pointer jumping inside the block (≤ 8 rounds; chains point backwards)
+        uint32_t par = 0;
+        S.pj[0][tid] = p;
+        S.vj[0][tid] = val;
+        while (bar_d_or(p >= 0)) {
+          if (p >= 0) {
+            const int32_t q = S.pj[par][p];
+            if (q < 0) {
+              val = S.vj[par][p];
+              p = -1;
+            } else {
+              p = q;
+            }
+          }
+          S.pj[par ^ 1][tid] = p;
+          S.vj[par ^ 1][tid] = val;
+          par ^= 1;
+        }
+        if (li < m) S.V[li] = val;  // x, in place
+        bar_d();
+      }
+    }
+    if (bar_d_or(bad)) {
+      if (tid == 0) record_error(ctx, DERR_CORRUPT);
+    } else {
+      for (uint32_t i = tid; i < m; i += kDT) __stcs(out + t0 + i, S.V[i]);
+    }
+    __threadfence();
+    bar_d();
+    if (tid == 0) st_release_u32(a.tile_flag + t, ctx.epoch);  // tile complete (also when malformed)
+  }
+}
+
+__global__ void __launch_bounds__(kDDecThreads) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  DDecSmem& S = *reinterpret_cast<DDecSmem*>(smem_raw);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    mbar_init(&S.full_in[0], 1);
+    mbar_init(&S.empty_in[0], kDW);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0) d_dec_loader(S, a, ctx, lane);
+  else d_dec_compute(S, a, ctx, threadIdx.x - 32);
+}
+
+}  // namespace
+
+// ---- host side -------------------------------------------------------------------
+size_t dpratio_fcm_workspace(uint64_t n) {
+  size_t temp = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                  (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 20);
+  return 4 * round16(n * 4) + round16(temp) + 256;
+}
+
+int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st) {
+  const uint64_t n = a0.n_words_total;
+  const uint64_t seg = round16(n * 4);
+  uint8_t* p = static_cast<uint8_t*>(ws);
+  uint32_t* key_in = reinterpret_cast<uint32_t*>(p);
+  uint32_t* key_out = reinterpret_cast<uint32_t*>(p + seg);
+  uint32_t* idx_in = reinterpret_cast<uint32_t*>(p + 2 * seg);
+  uint32_t* idx_out = reinterpret_cast<uint32_t*>(p + 3 * seg);
+  void* temp = p + 4 * seg;
+  size_t temp_bytes = ws_bytes - 4 * seg;
+  int launches = 0;
+  if (n) {
+    const int blocks = (int)umin64((n + 255) / 256, 148 * 16);
+    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_in, idx_in);
+    ++launches;
+    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, key_in, key_out, idx_in, idx_out, (int)n, 0, 20, st);
+    launches += 3;
+    uint32_t* dist = key_in;  // the unsorted keys are dead after the sort
+    const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
+    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_out,
+                                                      idx_out, dist);
+    ++launches;
+    EncArgs a = a0;
+    a.fcm_dist = dist;
+    const size_t smem = sizeof(DEncSmem);
+    static const bool init = [&] {
+      cudaFuncSetAttribute(dpratio_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      return true;
+    }();
+    (void)init;
+    const int grid = persistent_grid(dpratio_encode_kernel, kDEncThreads, smem, a.n_chunks / 2);
+    dpratio_encode_kernel<<<grid, kDEncThreads, smem, st>>>(a, ctx);
+    ++launches;
+  }
+  return launches;
+}
+
+void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st) {
+  const size_t smem = sizeof(DDecSmem);
+  static const bool init = [&] {
+    cudaFuncSetAttribute(dpratio_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return true;
+  }();
+  (void)init;
+  const int grid = persistent_grid(dpratio_decode_kernel, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
+  dpratio_decode_kernel<<<grid, kDDecThreads, smem, st>>>(a, ctx);
+}
+
+}  // namespace lcf

@@ -118,5 +118,8 @@ void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_ch
 void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
 void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st);
 void launch_write_header(const EncArgs& a, cudaStream_t st);
+size_t dpratio_fcm_workspace(uint64_t n_words);
+int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st);
+void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);
 
 }  // namespace lcf

@@ -46,48 +46,57 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
 
 // =============================== FCM encode kernels ===============================
 __global__ void fcm_hash_kernel(const uint64_t* __restrict__ x, uint64_t n, uint32_t* __restrict__ key,
-                                uint32_t* __restrict__ idx) {
+                                uint64_t* __restrict__ val) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t a = i >= 1 ? x[i - 1] : 0, b = i >= 2 ? x[i - 2] : 0, c = i >= 3 ? x[i - 3] : 0;
     key[i] = (uint32_t)(((a * FCM_K1) ^ (b * FCM_K2) ^ (c * FCM_K3)) >> 44);
-    idx[i] = (uint32_t)i;
+    // sort payload: the index and a 32-bit fold of x[i]; unequal folds prove
+    // unequal words, so the match kernel gathers x only for likely matches
+    const uint64_t xi = x[i];
+    val[i] = ((uint64_t)(uint32_t)(xi ^ (xi >> 32)) << 32) | (uint32_t)i;
   }
 }
 
 constexpr int kMatchBlock = 256;
+// One thread per sorted position k: the nearest of the pairs k−1 … k−4 with the
+// same hash and a bitwise-equal word is the match (L174, A-14, A-15). The
+// distance array is pre-zeroed; only matches are scattered.
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint32_t* __restrict__ key,
-                                                                const uint32_t* __restrict__ idx,
+                                                                const uint64_t* __restrict__ val,
                                                                 uint32_t* __restrict__ dist) {
-  __shared__ uint32_t sk[kMatchBlock + 4], si[kMatchBlock + 4];
-  __shared__ uint64_t sx[kMatchBlock + 4];
+  __shared__ uint32_t sk[kMatchBlock + 4];
+  __shared__ uint64_t sv[kMatchBlock + 4];
   for (uint64_t b0 = blockIdx.x * (uint64_t)kMatchBlock; b0 < n; b0 += (uint64_t)gridDim.x * kMatchBlock) {
-    // window: sorted positions [b0 − 4, b0 + kMatchBlock)
-    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {
+    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {  // sorted window [b0 − 4, b0 + 256)
       const int64_t k = (int64_t)b0 - 4 + j;
-      if (k >= 0 && (uint64_t)k < n) {
-        sk[j] = key[k];
-        si[j] = idx[k];
-        sx[j] = x[si[j]];  // gathered once per sorted position
-      } else {
-        sk[j] = 0xFFFFFFFFu;  // never equals a 20-bit hash
-      }
+      const bool in = k >= 0 && (uint64_t)k < n;
+      sk[j] = in ? key[k] : 0xFFFFFFFFu;  // never equals a 20-bit hash
+      sv[j] = in ? val[k] : 0;
     }
     __syncthreads();
     const uint64_t k = b0 + threadIdx.x;
     if (k < n) {
       const int j = threadIdx.x + 4;
-      const uint32_t h = sk[j], i = si[j];
-      const uint64_t xi = sx[j];
+      const uint32_t h = sk[j], i = (uint32_t)sv[j], fp = (uint32_t)(sv[j] >> 32);
       uint32_t d = 0;
+      uint64_t xi = 0;
+      bool have = false;
 #pragma unroll
-      for (int back = 1; back <= 4; ++back) {  // nearest first (A-14, pinned by Fig. 6)
-        if (sk[j - back] == h && sx[j - back] == xi) {
-          d = i - si[j - back];
-          break;
+      for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
+        if (sk[j - back] == h && (uint32_t)(sv[j - back] >> 32) == fp) {
+          const uint32_t jj = (uint32_t)sv[j - back];
+          if (!have) {
+            xi = x[i];
+            have = true;
+          }
+          if (x[jj] == xi) {
+            d = i - jj;
+            break;
+          }
         }
       }
-      dist[i] = d;
+      if (d) dist[i] = d;
     }
     __syncthreads();
   }
@@ -218,12 +227,17 @@ __device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst
   bar_d();
   const bool bypass = sc.flag;
   const uint32_t total = sc.s1, hib = sc.s2;
-  if (bypass) {
-    for (uint32_t j = tid; j < L; j += kDT) dst[3 + j] = src[j];
-    if (tid == 0) {
-      dst[0] = (uint8_t)L;
-      dst[1] = (uint8_t)(L >> 8);
-      dst[2] = 0;
+  if (bypass) {  // dst[3 + j] = src[j], one funnel shift per output word
+    const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
+    uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
+    const uint32_t nw = (L + 3 + 3) / 4;
+    for (uint32_t w = tid; w < nw; w += kDT) {
+      const uint32_t lo = w ? sw[w - 1] : 0u;
+      const uint32_t hi = 4 * w < L ? sw[w] : 0u;
+      uint32_t val = w ? __funnelshift_r(lo, hi, 8) : ((L & 0xFFFFu) | (hi << 24));
+      const uint32_t keep = 3 + L - 4 * w;  // bytes of this word inside the output
+      if (keep < 4) val &= (1u << (8 * keep)) - 1u;
+      dw[w] = val;
     }
     bar_d();
     return 3 + L;
@@ -240,8 +254,10 @@ __device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst
     const uint32_t i = tid + kDT * r;
     const bool set = (bal[r] >> lane) & 1;
     const uint32_t rank = sc.cnt[r * kDW + warp] + __popc(bal[r] & ((1u << lane) - 1));
-    emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? top[r] : 0, 0, true);
-    if (wl) emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, i < n ? (v[r] & lmask) : 0, 0, true);
+    if (bal[r])  // a warp without set words has nothing to emit
+      emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? top[r] : 0, 0, true);
+    if (wl) emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, i < n ? (v[r] & lmask) : 0, 0, true,
+                           wl >= 32 && kDT * r + 32 * warp + 31 < n);
   }
   bar_d();
   // ---- header, tail bytes, nr(B1), nr(B2), B3 ----
@@ -729,31 +745,31 @@ __global__ void __launch_bounds__(kDDecThreads) dpratio_decode_kernel(DecArgs a,
 size_t dpratio_fcm_workspace(uint64_t n) {
   size_t temp = 0;
   cub::DeviceRadixSort::SortPairs(nullptr, temp, (const uint32_t*)nullptr, (uint32_t*)nullptr,
-                                  (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 20);
-  return 4 * round16(n * 4) + round16(temp) + 256;
+                                  (const uint64_t*)nullptr, (uint64_t*)nullptr, (int)n, 0, 20);
+  return 2 * round16(n * 4) + 2 * round16(n * 8) + round16(temp) + 256;
 }
 
 int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st) {
   const uint64_t n = a0.n_words_total;
-  const uint64_t seg = round16(n * 4);
   uint8_t* p = static_cast<uint8_t*>(ws);
   uint32_t* key_in = reinterpret_cast<uint32_t*>(p);
-  uint32_t* key_out = reinterpret_cast<uint32_t*>(p + seg);
-  uint32_t* idx_in = reinterpret_cast<uint32_t*>(p + 2 * seg);
-  uint32_t* idx_out = reinterpret_cast<uint32_t*>(p + 3 * seg);
-  void* temp = p + 4 * seg;
-  size_t temp_bytes = ws_bytes - 4 * seg;
+  uint32_t* key_out = reinterpret_cast<uint32_t*>(p + round16(4 * n));
+  uint64_t* val_in = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n));
+  uint64_t* val_out = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n) + round16(8 * n));
+  void* temp = p + 2 * round16(4 * n) + 2 * round16(8 * n);
+  size_t temp_bytes = ws_bytes - (2 * round16(4 * n) + 2 * round16(8 * n));
   int launches = 0;
   if (n) {
     const int blocks = (int)umin64((n + 255) / 256, 148 * 16);
-    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_in, idx_in);
+    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_in, val_in);
     ++launches;
-    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, key_in, key_out, idx_in, idx_out, (int)n, 0, 20, st);
-    launches += 3;
+    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, key_in, key_out, val_in, val_out, (int)n, 0, 20, st);
+    launches += 5;  // histogram, exclusive sum, 3 onesweep passes
     uint32_t* dist = key_in;  // the unsorted keys are dead after the sort
+    cudaMemsetAsync(dist, 0, 4 * n, st);
     const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
     fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_out,
-                                                      idx_out, dist);
+                                                      val_out, dist);
     ++launches;
     EncArgs a = a0;
     a.fcm_dist = dist;

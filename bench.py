@@ -107,20 +107,37 @@ def dist_env():
 
 
 def make_fields(world, rank, device):
-    """Per-rank sub-blocks of N× larger global fields (weak scaling)."""
-    from paper_conf_asplos_azamifb25_b200 import datagen
+    """Per-field inputs. N = 1: the config's field. N > 1 (weak scaling): the
+    global input is the concatenation of N independent fields of the config
+    (replicas); chunk-local codecs get this rank's chunk-range shard of it,
+    DPratio (whole-array FCM) gets replica `rank` whole."""
+    from paper_conf_asplos_azamifb25_b200 import datagen, sharded
     fields = []
     for cfg, names, codecs in ((SP_CONFIG, SP_FIELDS, ("SPspeed", "SPratio")),
                                (DP_CONFIG, DP_FIELDS, ("DPspeed", "DPratio"))):
-        _, shape, _, _ = datagen.CONFIGS[cfg]
         for nm in names:
-            # rank r's block of a global field of shape (N·d0, d1, ...)
-            x = datagen.field(cfg, nm, device=device)
-            if world > 1:
-                x = x.contiguous()
-            x = x.reshape(-1)
-            fields.append((cfg, nm, codecs, x.view(torch.int32 if x.dtype == torch.float32 else torch.int64)))
+            reps = [datagen.field(cfg, nm, device=device, replica=r).reshape(-1) for r in range(world)]
+            wdt = torch.int32 if reps[0].dtype == torch.float32 else torch.int64
+            whole = torch.cat(reps).view(wdt) if world > 1 else reps[0].view(wdt)
+            total = whole.numel() * whole.element_size()
+            off, ln = sharded.shard_bytes(total, world, rank)
+            shard = whole.view(torch.uint8)[off:off + ln].view(wdt).clone()
+            own = reps[rank].view(wdt).clone()
+            del reps, whole
+            for codec in codecs:
+                x = own if (codec == "DPratio" or world == 1) else shard
+                fields.append((cfg, nm, codec, x, total))
+    torch.cuda.empty_cache()
     return fields
+
+
+def compress_op(lcf, j):
+    """Compress this rank's input; in sharded mode also all-gather the local
+    payload byte count (a device u64 at header byte 24) — the single
+    exchange of SURVEY §8(e), stream-ordered, no host sync."""
+    lcf.lcf_compress(j["codec"], None, j["x"], j["nbytes"], j["s"], j["cap"], sync=False)
+    if j["counts"] is not None:
+        torch.distributed.all_gather_into_tensor(j["counts"], j["s"][24:32].view(torch.int64))
 
 
 class Timer:
@@ -151,32 +168,32 @@ def run_lcf(args):
 
     # one job per (codec, field): buffers allocated once, outside the timed region
     jobs = []
-    for cfg, nm, fcodecs, x in fields:
+    for cfg, nm, codec, x, total in fields:
+        if codec not in codecs:
+            continue
         nbytes = x.numel() * x.element_size()
-        for codec in fcodecs:
-            if codec not in codecs:
+        cap = lcf.lcf_max_compressed_size(codec, None, nbytes)
+        s = torch.empty(cap, dtype=torch.uint8, device=dev)
+        y = torch.empty_like(x)
+        try:
+            n = lcf.lcf_compress(codec, None, x, nbytes, s, cap)
+        except lcf.LcfError as e:
+            if e.status == 1:
+                print(f"[bench] {codec} unavailable: {e}", file=sys.stderr)
                 continue
-            cap = lcf.lcf_max_compressed_size(codec, None, nbytes)
-            s = torch.empty(cap, dtype=torch.uint8, device=dev)
-            y = torch.empty_like(x)
-            try:
-                n = lcf.lcf_compress(codec, None, x, nbytes, s, cap)
-            except lcf.LcfError as e:
-                if e.status == 1:
-                    print(f"[bench] {codec} unavailable: {e}", file=sys.stderr)
-                    continue
-                raise
-            lcf.lcf_decompress(codec, None, s, n, y, nbytes)
-            assert torch.equal(x, y), f"{codec}/{nm}: round trip failed"
-            jobs.append({"codec": codec, "field": f"{cfg}/{nm}", "x": x, "s": s, "y": y, "cap": cap,
-                         "nbytes": nbytes, "sbytes": n, "ct": [], "dt": []})
+            raise
+        lcf.lcf_decompress(codec, None, s, n, y, nbytes)
+        assert torch.equal(x, y), f"{codec}/{nm}: round trip failed"
+        sharded_job = world > 1 and codec != "DPratio"
+        counts = torch.empty(world, dtype=torch.int64, device=dev) if sharded_job else None
+        jobs.append({"codec": codec, "field": f"{cfg}/{nm}", "x": x, "s": s, "y": y, "cap": cap,
+                     "nbytes": nbytes, "sbytes": n, "ct": [], "dt": [], "counts": counts})
     timer = Timer()
 
     def step(record):
         evs = []
         for j in jobs:
-            c = timer.time(lambda j=j: lcf.lcf_compress(j["codec"], None, j["x"], j["nbytes"], j["s"], j["cap"],
-                                                        sync=False))
+            c = timer.time(lambda j=j: compress_op(lcf, j))
             d = timer.time(lambda j=j: lcf.lcf_decompress(j["codec"], None, j["s"], j["sbytes"], j["y"],
                                                           j["nbytes"], sync=False))
             evs.append((j, c, d))

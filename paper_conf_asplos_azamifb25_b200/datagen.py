@@ -73,11 +73,13 @@ def multiscale(shape, gen: torch.Generator, device, octaves: int = 6, waves: int
     return out
 
 
-def field(config: str, name: str, device="cpu", origin=None, shape=None) -> torch.Tensor:
-    """One synthetic field of a named config (optionally a sub-block)."""
+def field(config: str, name: str, device="cpu", origin=None, shape=None, replica: int = 0) -> torch.Tensor:
+    """One synthetic field of a named config (optionally a sub-block);
+    `replica` > 0 draws an independent field of the same kind (multi-GPU
+    weak scaling concatenates replicas into one global stream)."""
     cid, full_shape, dtype, fields = CONFIGS[config]
     fid = fields[name]
-    g = _gen(seed_of(cid, fid), device)
+    g = _gen(seed_of(cid, fid) ^ (replica << 20), device)
     shp = tuple(shape or full_shape)
     if config == "hacc_280953867_f32":
         return _hacc(name, g, device, shp, origin)

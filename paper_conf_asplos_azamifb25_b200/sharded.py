@@ -1,0 +1,136 @@
+"""Multi-GPU mode: one process per GPU, chunk-range shards of ONE stream
+(BASELINE north_star "8-GPU mode").
+
+Rank g owns chunks [⌊gC/G⌋, ⌊(g+1)C/G⌋) of the global input. It compresses its
+shard into a *local* LCF1 stream. Chunks are context-free and shard boundaries
+are chunk boundaries, so the local size table and payload ARE the global
+stream's table slice and payload piece. The local payload byte count sits in
+the local header at byte 24; it is all-gathered as a device u64 (NCCL over
+NVLink/NVSwitch; gloo in the CPU tests) — the only exchange. An exclusive scan
+over ranks gives each piece's offset, and rank 0 writes the global header. The
+concatenation header ‖ table slices ‖ pad ‖ payload pieces is byte-identical to
+the 1-GPU stream. Decompression needs no exchange: every rank decodes its local
+stream.
+
+DPratio is not sharded by chunk range: FCM is a whole-array pass (L104). It
+runs whole fields per rank instead.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+HEADER = 32
+CHUNK = 16384
+
+
+def num_chunks(n_bytes: int) -> int:
+    return -(-n_bytes // CHUNK)
+
+
+def shard_chunks(n_bytes: int, world: int, rank: int):
+    """(first_chunk, n_chunks) of `rank`'s contiguous chunk range."""
+    C = num_chunks(n_bytes)
+    first = C * rank // world
+    last = C * (rank + 1) // world
+    return first, last - first
+
+
+def shard_bytes(n_bytes: int, world: int, rank: int):
+    """(byte offset, byte length) of `rank`'s shard of the input."""
+    first, k = shard_chunks(n_bytes, world, rank)
+    start = first * CHUNK
+    return start, max(0, min(n_bytes, (first + k) * CHUNK) - start)
+
+
+def round16(v: int) -> int:
+    return (v + 15) // 16 * 16
+
+
+@dataclass
+class Piece:
+    """One rank's part of the global stream."""
+    rank: int
+    first_chunk: int
+    n_chunks: int
+    local_stream: object  # uint8 tensor: local header ‖ table slice ‖ pad ‖ payload
+    payload_bytes: int
+    payload_offset: int   # offset of this piece inside the global payload
+    total_payload: int
+
+    def table_slice(self):
+        return self.local_stream[HEADER:HEADER + 4 * self.n_chunks]
+
+    def payload(self):
+        b = round16(HEADER + 4 * self.n_chunks)
+        return self.local_stream[b:b + self.payload_bytes]
+
+
+def exchange_counts(count_u64, group=None):
+    """All-gather one u64 per rank (a 1-element int64 tensor on the process
+    group's device) and return the list of counts — the single collective."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    out = torch.empty(world, dtype=torch.int64, device=count_u64.device)
+    dist.all_gather_into_tensor(out, count_u64.reshape(1).to(torch.int64), group=group)
+    return out
+
+
+def compress_sharded(algo: str, shard, total_bytes: int, local_compress, group=None) -> Piece:
+    """`shard` is this rank's slice of the global input (chunk-aligned);
+    `local_compress(algo, shard) -> uint8 tensor` is the codec (lcf on GPU,
+    the oracle in the CPU tests)."""
+    import torch
+    import torch.distributed as dist
+    if algo == "DPratio":
+        raise ValueError("DPratio runs whole fields per rank (FCM is a whole-array pass, L104)")
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    first, k = shard_chunks(total_bytes, world, rank)
+    local = local_compress(algo, shard)
+    count = local[24:32].view(torch.int64)  # local payload_bytes, left on its device
+    counts = exchange_counts(count, group).cpu().tolist()
+    offset = sum(counts[:rank])
+    return Piece(rank, first, k, local, counts[rank], offset, sum(counts))
+
+
+def global_header(algo: str, total_bytes: int, total_payload: int) -> bytes:
+    """The 32-byte LCF1 header (FORMAT.md §1) for the assembled stream."""
+    algo_id = {"SPspeed": 0, "SPratio": 1, "DPspeed": 2, "DPratio": 3}[algo]
+    wb = 4 if algo.startswith("SP") else 8
+    return (0x3146434C).to_bytes(4, "little") + bytes([1, algo_id, wb, 0]) + \
+        total_bytes.to_bytes(8, "little") + num_chunks(total_bytes).to_bytes(8, "little") + \
+        total_payload.to_bytes(8, "little")
+
+
+def assemble(algo: str, total_bytes: int, pieces) -> bytes:
+    """Concatenate gathered pieces (rank order) into the global stream bytes
+    (identity tests only; outside any timed region)."""
+    C = num_chunks(total_bytes)
+    tables = b"".join(bytes(p.table_slice().cpu().numpy().tobytes()) for p in pieces)
+    assert len(tables) == 4 * C
+    base = round16(HEADER + 4 * C)
+    pad = bytes(base - HEADER - 4 * C)
+    payload = b"".join(bytes(p.payload().cpu().numpy().tobytes()) for p in pieces)
+    total_payload = sum(p.payload_bytes for p in pieces)
+    return global_header(algo, total_bytes, total_payload) + tables + pad + payload
+
+
+def gather_pieces(piece: Piece, group=None):
+    """Rank 0 receives every rank's Piece (object collective; tests only)."""
+    import torch.distributed as dist
+    payload = (piece.rank, piece.first_chunk, piece.n_chunks, piece.local_stream.cpu(), piece.payload_bytes,
+               piece.payload_offset, piece.total_payload)
+    out = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, payload, group=group)
+    return [Piece(*o) for o in out]
+
+
+def lcf_local_compress(algo: str, shard):
+    """GPU shard codec: lcf_compress into a local stream (device tensor)."""
+    from . import lcf
+    return lcf.compress(algo, shard)
+
+
+def lcf_local_decompress(algo: str, local_stream, out=None):
+    from . import lcf
+    return lcf.decompress(algo, local_stream, out=out)

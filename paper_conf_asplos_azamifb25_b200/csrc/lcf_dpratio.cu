@@ -289,9 +289,11 @@ __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, u
   if (len < 3) return -1;
   const uint32_t L = src[0] | ((uint32_t)src[1] << 8), k = src[2];
   if (L > cap) return -1;
-  if (k == 0) {
+  if (k == 0) {  // bypass: dst[j] = src[3 + j], one funnel shift per word
     if (len != 3 + L) return -1;
-    for (uint32_t j = tid; j < L; j += kDT) dst[j] = src[3 + j];
+    const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
+    uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
+    for (uint32_t w = tid; w < (L + 3) / 4; w += kDT) dw[w] = __funnelshift_r(sw[w], sw[w + 1], 24);
     bar_d();
     return (int)L;
   }
@@ -632,21 +634,22 @@ __device__ __forceinline__ bool d_decode_chunk(DDecSmem& S, const uint8_t* pay, 
   if (l1 < 0) return false;
   const int l0 = adaptive_decode(S.rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, S.sc, tid);
   if (l0 != (int)(8 * m)) return false;
-  // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8)
+  // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8), moved as 16-byte pairs
   uint64_t v[8], run = 0;
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const uint32_t i = 8 * tid + j;
-    v[j] = i < m ? tcms_inv(arr[i]) : 0;
-    run += v[j];
+  for (int j = 0; j < 8; j += 2) {
+    const ulonglong2 q = reinterpret_cast<const ulonglong2*>(arr)[4 * tid + j / 2];
+    v[j] = 8 * tid + j < m ? tcms_inv((uint64_t)q.x) : 0;
+    v[j + 1] = 8 * tid + j + 1 < m ? tcms_inv((uint64_t)q.y) : 0;
+    run += v[j] + v[j + 1];
   }
   uint64_t tot;
   uint64_t acc = cta_scan_u64(run, S.scan, tid, tot);
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const uint32_t i = 8 * tid + j;
-    acc += v[j];
-    if (i < m) arr[i] = acc;
+  for (int j = 0; j < 8; j += 2) {
+    const uint64_t a0 = acc + v[j], a1 = a0 + v[j + 1];
+    acc = a1;
+    reinterpret_cast<ulonglong2*>(arr)[4 * tid + j / 2] = make_ulonglong2(a0, a1);  // words ≥ m: scratch
   }
   bar_d();
   return true;
@@ -744,27 +747,34 @@ __global__ void __launch_bounds__(kDDecThreads) dpratio_decode_kernel(DecArgs a,
 // ---- host side -------------------------------------------------------------------
 size_t dpratio_fcm_workspace(uint64_t n) {
   size_t temp = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const uint32_t*)nullptr, (uint32_t*)nullptr,
-                                  (const uint64_t*)nullptr, (uint64_t*)nullptr, (int)n, 0, 20);
+  cub::DoubleBuffer<uint32_t> dk(nullptr, nullptr);
+  cub::DoubleBuffer<uint64_t> dv(nullptr, nullptr);
+  cub::DeviceRadixSort::SortPairs(nullptr, temp, dk, dv, (int)n, 0, 20);
   return 2 * round16(n * 4) + 2 * round16(n * 8) + round16(temp) + 256;
 }
 
 int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st) {
   const uint64_t n = a0.n_words_total;
   uint8_t* p = static_cast<uint8_t*>(ws);
-  uint32_t* key_in = reinterpret_cast<uint32_t*>(p);
-  uint32_t* key_out = reinterpret_cast<uint32_t*>(p + round16(4 * n));
-  uint64_t* val_in = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n));
-  uint64_t* val_out = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n) + round16(8 * n));
+  uint32_t* key_a = reinterpret_cast<uint32_t*>(p);
+  uint32_t* key_b = reinterpret_cast<uint32_t*>(p + round16(4 * n));
+  uint64_t* val_a = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n));
+  uint64_t* val_b = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n) + round16(8 * n));
   void* temp = p + 2 * round16(4 * n) + 2 * round16(8 * n);
   size_t temp_bytes = ws_bytes - (2 * round16(4 * n) + 2 * round16(8 * n));
   int launches = 0;
   if (n) {
     const int blocks = (int)umin64((n + 255) / 256, 148 * 16);
-    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_in, val_in);
+    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_a, val_a);
     ++launches;
-    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, key_in, key_out, val_in, val_out, (int)n, 0, 20, st);
+    // (h, i) pairs by the 20 key bits; stable, so equal hashes keep index order
+    cub::DoubleBuffer<uint32_t> dk(key_a, key_b);
+    cub::DoubleBuffer<uint64_t> dv(val_a, val_b);
+    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, dk, dv, (int)n, 0, 20, st);
     launches += 5;  // histogram, exclusive sum, 3 onesweep passes
+    const uint32_t* key_out = dk.Current();
+    const uint64_t* val_out = dv.Current();
+    uint32_t* key_in = dk.Alternate();
     uint32_t* dist = key_in;  // the unsorted keys are dead after the sort
     cudaMemsetAsync(dist, 0, 4 * n, st);
     const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);

@@ -127,21 +127,22 @@ __device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, 
 // Encode L bytes at src (8-byte aligned) with RAZE (rare = false, L189) or RARE
 // (rare = true, L195) into dst (16-byte aligned, ≥ L + 3 + 32 bytes). All kDT
 // compute threads call it; returns the output length (FORMAT.md §6.2–6.3).
-__device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare, AdaptScratch& sc,
-                                    uint32_t tid) {
+// Word i = tid + 256·r (r = 0..7); the rounds are not unrolled and re-read the
+// words from shared memory, which keeps the code small (I-cache) and the
+// register count low (occupancy).
+__device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
+                                                 AdaptScratch& sc, uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint32_t n = L / 8, tl = L % 8;
+  const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
   if (tid < 65) sc.hist[tid] = 0;
-  if (tid < 64) sc.b1[tid] = 0;
   bar_d();
   // ---- histogram of clz(v_i ⊕ ref_i), warp-aggregated shared atomics ----
-  uint64_t v[8], ref[8];
-#pragma unroll
-  for (int r = 0; r < 8; ++r) {
+#pragma unroll 1
+  for (uint32_t r = 0; r < 8; ++r) {
     const uint32_t i = tid + kDT * r;
-    v[r] = i < n ? ld_u64(src + 8 * i) : 0;
-    ref[r] = (rare && i < n && i > 0) ? ld_u64(src + 8 * (i - 1)) : 0;
-    const uint32_t z = i < n ? clz64(v[r] ^ ref[r]) : 65u;
+    uint32_t z = 65u;
+    if (i < n) z = clz64(sv[i] ^ ((rare && i) ? sv[i - 1] : 0ull));
     const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
     if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
   }
@@ -164,23 +165,24 @@ __device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst
   }
   bar_d();
   const uint32_t k = sc.k;
-  // ---- B1 bits and ranks (word i = tid + 256 r: warp ballots are B1 words) ----
-  uint64_t top[8];
-  uint32_t bal[8];
-#pragma unroll
-  for (int r = 0; r < 8; ++r) {
+  const uint32_t sh = 64 - k;  // top(v) = v >> sh (k = 64: sh = 0)
+  // ---- B1 (warp ballots are the B1 words) and per-(round, warp) counts ----
+#pragma unroll 1
+  for (uint32_t r = 0; r < 8; ++r) {
     const uint32_t i = tid + kDT * r;
-    top[r] = k == 64 ? v[r] : (v[r] >> (64 - k));
-    const uint64_t tref = k == 64 ? ref[r] : (ref[r] >> (64 - k));
-    const bool set = i < n && top[r] != tref;
-    bal[r] = __ballot_sync(0xFFFFFFFFu, set);
+    bool set = false;
+    if (i < n) {
+      const uint64_t ref = (rare && i) ? sv[i - 1] : 0ull;
+      set = (sv[i] >> sh) != (ref >> sh);
+    }
+    const uint32_t bal = __ballot_sync(0xFFFFFFFFu, set);
     if (lane == 0) {
-      sc.b1[r * kDW + warp] = bal[r];
-      sc.cnt[r * kDW + warp] = __popc(bal[r]);
+      sc.b1[r * kDW + warp] = bal;
+      sc.cnt[r * kDW + warp] = __popc(bal);
     }
   }
   bar_d();
-  uint32_t nr1 = 0, nr2 = 0, b2 = 0, b3 = 0, c1m = 0, off1 = 0, b1w0 = 0, b1w1 = 0;
+  uint32_t nr1 = 0, b2 = 0, b3 = 0, c1m = 0, off1 = 0, b1w0 = 0, b1w1 = 0;
   const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
   if (warp == 0) {
     // prefix of the 64 per-(round, warp) counts
@@ -215,7 +217,7 @@ __device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst
     nr1 = __shfl_sync(0xFFFFFFFFu, x, 31);
     const uint32_t pb2 = __shfl_up_sync(0xFFFFFFFFu, b2, 1);
     b3 = __ballot_sync(0xFFFFFFFFu, lane < L2 && b2 != (lane ? pb2 : 0u));
-    nr2 = __popc(b3);
+    const uint32_t nr2 = __popc(b3);
     const uint32_t hib = (nset * k + 7) / 8, lob = (n * (64 - k) + 7) / 8;
     const uint32_t total = 3 + hib + lob + tl + nr1 + nr2 + L3;
     if (lane == 0) {
@@ -249,15 +251,20 @@ __device__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst
   const uint64_t hi_base = 24, lo_base = 8ull * (3 + hib);
   const uint32_t wl = 64 - k;
   const uint64_t lmask = wl >= 64 ? ~0ull : ((1ull << wl) - 1);
-#pragma unroll
-  for (int r = 0; r < 8; ++r) {
+#pragma unroll 1
+  for (uint32_t r = 0; r < 8; ++r) {
     const uint32_t i = tid + kDT * r;
-    const bool set = (bal[r] >> lane) & 1;
-    const uint32_t rank = sc.cnt[r * kDW + warp] + __popc(bal[r] & ((1u << lane) - 1));
-    if (bal[r])  // a warp without set words has nothing to emit
-      emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? top[r] : 0, 0, true);
-    if (wl) emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, i < n ? (v[r] & lmask) : 0, 0, true,
-                           wl >= 32 && kDT * r + 32 * warp + 31 < n);
+    const uint32_t q = r * kDW + warp;
+    const uint32_t bal = sc.b1[q];
+    const uint64_t v = i < n ? sv[i] : 0ull;
+    if (bal) {  // a warp without set words has nothing to emit
+      const bool set = (bal >> lane) & 1;
+      const uint32_t rank = sc.cnt[q] + __popc(bal & ((1u << lane) - 1));
+      emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? (v >> sh) : 0, 0, true);
+    }
+    if (wl)
+      emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, v & lmask, 0, true,
+                     wl >= 32 && kDT * r + 32 * warp + 31 < n);
   }
   bar_d();
   // ---- header, tail bytes, nr(B1), nr(B2), B3 ----

@@ -131,6 +131,25 @@ def make_fields(world, rank, device):
     return fields
 
 
+def kernel_bytes(j):
+    """Algorithmic bytes per launch of every kernel a job's compress and
+    decompress launch: the I/O the method itself must move."""
+    n, sb, codec = j["nbytes"], j["sbytes"], j["codec"]
+    words = n // (4 if codec.startswith("SP") else 8)
+    io = n + sb
+    if codec == "SPspeed":
+        return {"speed_encode_u32": io, "speed_decode_u32": io}
+    if codec == "DPspeed":
+        return {"speed_encode_u64": io, "speed_decode_u64": io}
+    if codec == "SPratio":
+        return {"spratio_encode": io, "spratio_decode": io}
+    return {"fcm_hash": 20 * words,                   # x in, 20-bit key + (fold, index) payload out
+            "cub_radix_sort_pairs": 76 * words,       # 3 passes × 12 B in/out + histogram read
+            "fcm_match": 12 * words,                  # sorted keys + payloads in (matches scattered)
+            "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
+            "dpratio_decode": sb + n}                 # stream in, x out
+
+
 def compress_op(lcf, j):
     """Compress this rank's input; in sharded mode also all-gather the local
     payload byte count (a device u64 at header byte 24) — the single
@@ -210,6 +229,8 @@ def run_lcf(args):
     if world > 1:
         torch.distributed.barrier()
     launches0 = lcf.lcf_launch_count()
+    lcf.lcf_profile_report()  # clear
+    lcf.lcf_profile_enable(True)
     with ClockSampler(local) as clk:
         t0 = time.perf_counter()
         for _ in range(args.steps):
@@ -217,12 +238,15 @@ def run_lcf(args):
         torch.cuda.synchronize()
         wall = time.perf_counter() - t0
     launches = lcf.lcf_launch_count() - launches0
+    lcf.lcf_profile_enable(False)
+    ktimes = lcf.lcf_profile_report()
     lcf.lcf_check_stream()
     for j in jobs:  # the timed outputs are still exact
         assert torch.equal(j["x"], j["y"]), j["codec"]
 
     hbm, peak_kind = peaks()
-    per_codec, tot_bytes, tot_ms, dominant = {}, 0, 0.0, None
+    per_codec, tot_bytes, tot_ms = {}, 0, 0.0
+    kbytes = {}
     for j in jobs:
         ct, dt = statistics.median(j["ct"]), statistics.median(j["dt"])
         moved = j["nbytes"] + j["sbytes"]
@@ -234,15 +258,27 @@ def run_lcf(args):
         }
         tot_bytes += 2 * j["nbytes"]
         tot_ms += ct + dt
-        for kind, t in (("compress", ct), ("decompress", dt)):
-            if dominant is None or t > dominant[2]:
-                dominant = (j, kind, t)
-    j, kind, t = dominant
-    moved = j["nbytes"] + j["sbytes"]
-    roofline = {"bound": "hbm", "achieved": moved / t / 1e6, "peak": hbm, "unit": "GB/s",
-                "frac": moved / t / 1e6 / hbm, "traffic": None,
-                "kernel": f"{j['codec']} {kind} ({j['field']})", "peak_kind": peak_kind,
-                "algorithmic_bytes_per_launch": moved}
+        for name, b in kernel_bytes(j).items():
+            kbytes[name] = kbytes.get(name, 0) + b * args.steps
+    # per-kernel live timing (CUDA events around every library launch, timed region only)
+    kernels = {}
+    for name, (cnt, ms) in ktimes.items():
+        if name not in kbytes or ms <= 0:
+            continue
+        kernels[name] = {"launches": cnt, "avg_ms": ms / cnt, "share": 0.0,
+                         "achieved_gbs": kbytes[name] / ms / 1e6, "frac": kbytes[name] / ms / 1e6 / hbm}
+    ksum = sum(ms for _, ms in ktimes.values()) or 1.0
+    for name in kernels:
+        kernels[name]["share"] = ktimes[name][1] / ksum
+    own = {k: v for k, v in kernels.items() if not k.startswith("cub_")}
+    dom = max(own, key=lambda k: ktimes[k][1]) if own else None
+    roofline = None
+    if dom:
+        d = kernels[dom]
+        roofline = {"bound": "hbm", "achieved": d["achieved_gbs"], "peak": hbm, "unit": "GB/s", "frac": d["frac"],
+                    "traffic": None, "kernel": dom, "peak_kind": peak_kind,
+                    "algorithmic_bytes_per_launch": kbytes[dom] / max(1, d["launches"]),
+                    "avg_launch_ms": d["avg_ms"], "share_of_step": d["share"]}
     value = tot_bytes / tot_ms / 1e6
     # aggregate over ranks: weak scaling, max step time
     ms_step = tot_ms
@@ -262,7 +298,7 @@ def run_lcf(args):
             "vs_baseline": None, "dtype": "u32/u64 (f32/f64 bits)", "data": "synthetic",
             "config": {"workload": WORKLOAD, "l2": "flushed (256 MiB write) before every timed call",
                        "parallelism": f"chunk-range shards x{world}" if world > 1 else "single GPU"},
-            "per_codec": per_codec, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "per_codec": per_codec, "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": clk.summary(),
         }
         print(json.dumps(line))

@@ -129,6 +129,14 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  * (bench/test accounting). */
 uint64_t lcf_launch_count(void);
 
+/* Kernel-time tracing. While enabled, the library brackets every kernel it
+ * launches with a pair of CUDA events on the launching stream (CUB's sort
+ * counts as one "kernel"). lcf_profile_report synchronises on the recorded
+ * events, writes "name launches total_ms\n" per kernel into buf (NUL-terminated,
+ * truncated to cap) and clears the record; it returns the untruncated length. */
+void lcf_profile_enable(int enable);
+size_t lcf_profile_report(char* buf, size_t cap);
+
 #ifdef __cplusplus
 }
 #endif

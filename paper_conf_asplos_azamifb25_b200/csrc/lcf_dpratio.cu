@@ -28,7 +28,10 @@ namespace {
 
 constexpr int kDW = 8;                 // compute warps
 constexpr uint32_t kDT = kDW * 32;     // compute threads
-constexpr int kDOut = 2, kDBatch = 4;  // output slots (encode), tiles per ticket (decode)
+#ifndef LCF_DP_OUT
+#define LCF_DP_OUT 2
+#endif
+constexpr int kDOut = LCF_DP_OUT, kDBatch = 4;  // output slots (encode), tiles per ticket (decode)
 constexpr int kDEncThreads = (2 + kDW) * 32, kDDecThreads = (1 + kDW) * 32;
 constexpr uint32_t kBarD = 1;
 constexpr uint32_t kTileWords = 2048;
@@ -110,7 +113,6 @@ struct AdaptScratch {
   uint32_t k, flag, s1, s2;
 };
 
-__device__ __forceinline__ uint64_t ld_u64(const uint8_t* p) { return *reinterpret_cast<const uint64_t*>(p); }
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
 
 // 64-bit field of width w (≤ 64) at bit position P of the little-endian word
@@ -772,21 +774,29 @@ int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, siz
   int launches = 0;
   if (n) {
     const int blocks = (int)umin64((n + 255) / 256, 148 * 16);
-    fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_a, val_a);
+    {
+      KTrace kt("fcm_hash", st);
+      fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_a, val_a);
+    }
     ++launches;
     // (h, i) pairs by the 20 key bits; stable, so equal hashes keep index order
     cub::DoubleBuffer<uint32_t> dk(key_a, key_b);
     cub::DoubleBuffer<uint64_t> dv(val_a, val_b);
-    cub::DeviceRadixSort::SortPairs(temp, temp_bytes, dk, dv, (int)n, 0, 20, st);
-    launches += 5;  // histogram, exclusive sum, 3 onesweep passes
+    {
+      KTrace kt("cub_radix_sort_pairs", st);
+      cub::DeviceRadixSort::SortPairs(temp, temp_bytes, dk, dv, (int)n, 0, 20, st);
+    }
     const uint32_t* key_out = dk.Current();
     const uint64_t* val_out = dv.Current();
     uint32_t* key_in = dk.Alternate();
     uint32_t* dist = key_in;  // the unsorted keys are dead after the sort
     cudaMemsetAsync(dist, 0, 4 * n, st);
     const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
-    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_out,
-                                                      val_out, dist);
+    {
+      KTrace kt("fcm_match", st);
+      fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_out,
+                                                        val_out, dist);
+    }
     ++launches;
     EncArgs a = a0;
     a.fcm_dist = dist;
@@ -797,6 +807,7 @@ int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, siz
     }();
     (void)init;
     const int grid = persistent_grid(dpratio_encode_kernel, kDEncThreads, smem, a.n_chunks / 2);
+    KTrace kt("dpratio_encode", st);
     dpratio_encode_kernel<<<grid, kDEncThreads, smem, st>>>(a, ctx);
     ++launches;
   }
@@ -811,6 +822,7 @@ void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
   }();
   (void)init;
   const int grid = persistent_grid(dpratio_decode_kernel, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
+  KTrace kt("dpratio_decode", st);
   dpratio_decode_kernel<<<grid, kDDecThreads, smem, st>>>(a, ctx);
 }
 

@@ -11,6 +11,16 @@ namespace lcf {
 
 __host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
+// Kernel-time tracing (lcf_profile_enable): when enabled, a pair of CUDA
+// events brackets every kernel the library launches, on the launching stream.
+struct KTrace {
+  KTrace(const char* name, cudaStream_t st);
+  ~KTrace();
+  const char* name;
+  cudaStream_t st;
+  void* rec;
+};
+
 // One compress launch covers chunks [first_chunk, first_chunk + n_chunks) of a
 // stream whose input has n_words_total words (FORMAT.md §2).
 struct EncArgs {

@@ -506,6 +506,7 @@ template <typename U> void launch_speed_encode(const EncArgs& a, const LaunchCtx
   }();
   (void)init;
   const int grid = persistent_grid(speed_encode_kernel<U>, kEncThreads, smem, a.n_chunks);
+  KTrace kt(sizeof(U) == 4 ? "speed_encode_u32" : "speed_encode_u64", st);
   speed_encode_kernel<U><<<grid, kEncThreads, smem, st>>>(a, ctx);
 }
 template <typename U>
@@ -517,6 +518,7 @@ void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_ch
   }();
   (void)init;
   const int grid = persistent_grid(speed_decode_kernel<U>, kDecThreads, smem, (max_chunks + kDecBatch - 1) / kDecBatch);
+  KTrace kt(sizeof(U) == 4 ? "speed_decode_u32" : "speed_decode_u64", st);
   speed_decode_kernel<U><<<grid, kDecThreads, smem, st>>>(a, ctx);
 }
 template void launch_speed_encode<uint32_t>(const EncArgs&, const LaunchCtx&, cudaStream_t);

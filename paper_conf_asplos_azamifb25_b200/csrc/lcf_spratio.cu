@@ -561,6 +561,7 @@ void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t 
   }();
   (void)init;
   const int grid = persistent_grid(spratio_encode_kernel, kREncThreads, smem, a.n_chunks);
+  KTrace kt("spratio_encode", st);
   spratio_encode_kernel<<<grid, kREncThreads, smem, st>>>(a, ctx);
 }
 
@@ -572,6 +573,7 @@ void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
   }();
   (void)init;
   const int grid = persistent_grid(spratio_decode_kernel, kRDecThreads, smem, (max_chunks + kRDecBatch - 1) / kRDecBatch);
+  KTrace kt("spratio_decode", st);
   spratio_decode_kernel<<<grid, kRDecThreads, smem, st>>>(a, ctx);
 }
 

@@ -56,6 +56,10 @@ def lib() -> ctypes.CDLL:
         L.lcf_write_header.restype = i32
         L.lcf_launch_count.argtypes = []
         L.lcf_launch_count.restype = u64
+        L.lcf_profile_enable.argtypes = [i32]
+        L.lcf_profile_enable.restype = None
+        L.lcf_profile_report.argtypes = [ctypes.c_char_p, sz]
+        L.lcf_profile_report.restype = sz
         _lib = L
     return _lib
 
@@ -180,6 +184,21 @@ def lcf_write_header(algo, dtype, total_in_bytes, total_payload_bytes, d_stream,
 
 def lcf_launch_count() -> int:
     return int(lib().lcf_launch_count())
+
+
+def lcf_profile_enable(enable: bool) -> None:
+    lib().lcf_profile_enable(1 if enable else 0)
+
+
+def lcf_profile_report() -> dict:
+    """{kernel name: (launches, total ms)} since enabling; clears the record."""
+    buf = ctypes.create_string_buffer(1 << 16)
+    lib().lcf_profile_report(buf, len(buf))
+    out = {}
+    for line in buf.value.decode().splitlines():
+        name, cnt, ms = line.split()
+        out[name] = (int(cnt), float(ms))
+    return out
 
 
 # ---- tensor conveniences (allocation + the calls above) ------------------------

@@ -110,7 +110,8 @@ struct AdaptScratch {
   uint32_t hist[65];
   uint32_t cnt[64];     // per (round, warp) set counts → exclusive prefix
   uint32_t b1[64];      // B1 bitmap words (n ≤ 2048 bits)
-  uint32_t k, flag, s1, s2;
+  uint32_t c1m[32], off1[32], b2[32];  // encoder plan → emit: warp 0's B2 bits, nr(B1) offsets
+  uint32_t k, flag, s1, s2, nr1, b3;
 };
 
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
@@ -132,8 +133,8 @@ __device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, 
 // Word i = tid + 256·r (r = 0..7); the rounds are not unrolled and re-read the
 // words from shared memory, which keeps the code small (I-cache) and the
 // register count low (occupancy).
-__device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
-                                                 AdaptScratch& sc, uint32_t tid) {
+__device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, bool rare, AdaptScratch& sc,
+                                               uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint32_t n = L / 8, tl = L % 8;
   const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
@@ -226,11 +227,30 @@ __device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L,
       sc.flag = total >= 3 + L;  // bypass (A-23)
       sc.s1 = total;
       sc.s2 = hib;
+      sc.nr1 = nr1;
+      sc.b3 = b3;
     }
+    sc.c1m[lane] = c1m;
+    sc.off1[lane] = off1;
+    sc.b2[lane] = b2;
   }
   bar_d();
+  return sc.flag ? 3 + L : sc.s1;
+}
+
+// Second half of RAZE/RARE: writes the planned output (adaptive_plan must have
+// run on the same input just before).
+__device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
+                                           AdaptScratch& sc, uint32_t tid) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  const uint32_t n = L / 8, tl = L % 8;
+  const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
+  const uint32_t k = sc.k, sh = 64 - k;
+  const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
+  (void)L1;
+  (void)L2;
   const bool bypass = sc.flag;
-  const uint32_t total = sc.s1, hib = sc.s2;
+  const uint32_t total = sc.s1, hib = sc.s2, nr1 = sc.nr1, b3 = sc.b3;
   if (bypass) {  // dst[3 + j] = src[j], one funnel shift per output word
     const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
     uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
@@ -244,7 +264,7 @@ __device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L,
       dw[w] = val;
     }
     bar_d();
-    return 3 + L;
+    return;
   }
   uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
   for (uint32_t j = tid; j < (total + 7) / 4 + 1; j += kDT) dw[j] = 0;
@@ -278,7 +298,9 @@ __device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L,
   }
   if (tid < tl) dst[after + tid] = src[8 * n + tid];
   if (warp == 0) {
-    uint32_t p = after + tl + off1;
+    const uint32_t c1m = sc.c1m[lane], b2 = sc.b2[lane];
+    const uint32_t b1w0 = sc.b1[2 * lane], b1w1 = sc.b1[2 * lane + 1];
+    uint32_t p = after + tl + sc.off1[lane];
 #pragma unroll
     for (int j = 0; j < 8; ++j)
       if ((c1m >> j) & 1) dst[p++] = (uint8_t)((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
@@ -286,7 +308,13 @@ __device__ __noinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L,
     if (lane < L3) dst[total - L3 + lane] = (uint8_t)(b3 >> (8 * lane));
   }
   bar_d();
-  return total;
+}
+
+__device__ __forceinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
+                                                    AdaptScratch& sc, uint32_t tid) {
+  const uint32_t len = adaptive_plan(src, L, rare, sc, tid);
+  adaptive_emit(src, L, dst, rare, sc, tid);
+  return len;
 }
 
 // Decode a RAZE/RARE stream of `len` bytes at src (16-byte aligned, ≥ 16 bytes
@@ -495,22 +523,25 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       bar_d();
       // RAZE then RARE (L189–201)
       const uint32_t l1 = adaptive_encode(reinterpret_cast<const uint8_t*>(S.w), 8 * m, S.rz, false, S.sc, tid);
-      const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
-      mbar_wait(&S.empty_out[o], pho ^ 1);
-      uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
-      const uint32_t l2 = adaptive_encode(S.rz, l1, ob, true, S.sc, tid);
+      // RARE is planned first: the chunk's size — and its aggregate for the
+      // look-back of later chunks — is known before an output slot is needed
+      const uint32_t l2 = adaptive_plan(S.rz, l1, true, S.sc, tid);
       const uint32_t raw_len = 8 * m;
       const bool raw = l2 >= raw_len;  // L104, ties → raw
       const uint32_t len = raw ? raw_len : l2;
+      if (tid == 0) lookback_publish(ctx, c, round16(len));
+      const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
+      mbar_wait(&S.empty_out[o], pho ^ 1);
+      uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       if (raw) {  // the V / Dist words themselves
         for (uint32_t i = tid; i < m; i += kDT)
           reinterpret_cast<uint64_t*>(ob)[i] = part == 0 ? (S.din[i] ? 0ull : S.xin[i]) : (uint64_t)S.din[i];
         if (tid < 2 && (m & 1)) reinterpret_cast<uint64_t*>(ob)[m + tid] = 0;  // round16 pad
-      } else if (tid < 16 && len + tid < round16(len)) {
-        ob[len + tid] = 0;
+      } else {
+        adaptive_emit(S.rz, l1, ob, true, S.sc, tid);
+        if (tid < 16 && len + tid < round16(len)) ob[len + tid] = 0;
       }
       if (tid == 0) {
-        lookback_publish(ctx, c, round16(len));
         S.out_chunk[o] = c;
         S.out_len[o] = len;
         S.out_raw[o] = raw;

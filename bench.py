@@ -131,6 +131,19 @@ def make_fields(world, rank, device):
     return fields
 
 
+def kernel_traffic():
+    """dram__bytes_read + dram__bytes_write per launch of each kernel on this
+    workload, from the newest committed `ncu --set full` summary
+    (profiles/<round>_kernel_traffic.json, scripts/profile_round.sh)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_kernel_traffic.json")))
+    if not files:
+        return {}
+    with open(files[-1]) as f:
+        d = json.load(f)
+    return {k.split(":", 1)[1]: v["dram_bytes_per_launch"] for k, v in d.items()}
+
+
 def kernel_bytes(j):
     """Algorithmic bytes per launch of every kernel a job's compress and
     decompress launch: the I/O the method itself must move."""
@@ -273,10 +286,11 @@ def run_lcf(args):
     own = {k: v for k, v in kernels.items() if not k.startswith("cub_")}
     dom = max(own, key=lambda k: ktimes[k][1]) if own else None
     roofline = None
+    traffic = kernel_traffic()
     if dom:
         d = kernels[dom]
         roofline = {"bound": "hbm", "achieved": d["achieved_gbs"], "peak": hbm, "unit": "GB/s", "frac": d["frac"],
-                    "traffic": None, "kernel": dom, "peak_kind": peak_kind,
+                    "traffic": traffic.get(dom), "kernel": dom, "peak_kind": peak_kind,
                     "algorithmic_bytes_per_launch": kbytes[dom] / max(1, d["launches"]),
                     "avg_launch_ms": d["avg_ms"], "share_of_step": d["share"]}
     value = tot_bytes / tot_ms / 1e6

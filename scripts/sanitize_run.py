@@ -1,0 +1,28 @@
+"""Small end-to-end run of all four codecs (and a corrupt stream) for
+compute-sanitizer (memcheck / racecheck / synccheck / initcheck)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_asplos_azamifb25_b200 import datagen, lcf  # noqa: E402
+
+for algo in ("SPspeed", "SPratio", "DPspeed", "DPratio"):
+    W = 32 if algo.startswith("SP") else 64
+    for name, words in datagen.adversarial(W)[:6] + [("smooth", datagen.smooth_1d(3 * 16384 // (W // 8) + 77,
+                                                                               np.float32 if W == 32 else np.float64,
+                                                                               seed=2).view(np.uint32 if W == 32 else np.uint64))]:
+        x = torch.from_numpy(words.view(np.int32 if W == 32 else np.int64).copy()).cuda()
+        s = lcf.compress(algo, x)
+        y = lcf.decompress(algo, s)
+        assert torch.equal(x, y), (algo, name)
+        t = s.clone()
+        t[min(40, t.numel() - 1)] ^= 0x5A  # corrupt a size entry / payload byte
+        try:
+            lcf.lcf_decompress(algo, None, t, t.numel(), y, y.numel() * y.element_size())
+        except lcf.LcfError:
+            pass
+    print(algo, "ok")
+torch.cuda.synchronize()

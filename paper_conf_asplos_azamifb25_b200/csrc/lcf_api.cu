@@ -15,6 +15,7 @@ using namespace lcf;
 namespace {
 
 std::atomic<uint64_t> g_launches{0};
+unsigned long long* g_trace_buf = nullptr;  // lcf__trace_compress only
 
 struct Workspace {
   int device = -1;
@@ -194,6 +195,18 @@ size_t lcf_max_compressed_size(lcf_algo_t algo, lcf_dtype_t dtype, size_t in_byt
 
 uint64_t lcf_launch_count(void) { return g_launches.load(); }
 
+// Undocumented diagnostic entry point (not in lcf.h): lcf_compress that also
+// records 8 globaltimer stamps per chunk into d_trace (n_chunks × 8 u64) for the
+// speed codecs' pipeline analysis (scripts/trace_pipeline.py).
+lcf_status_t lcf__trace_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
+                                 size_t out_capacity, unsigned long long* d_trace, void* stream) {
+  g_trace_buf = d_trace;
+  size_t n = 0;
+  lcf_status_t st = lcf_compress(algo, dtype, d_in, in_bytes, d_out, out_capacity, &n, stream);
+  g_trace_buf = nullptr;
+  return st;
+}
+
 lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
                           size_t out_capacity, size_t* out_bytes, void* stream_) {
   cudaStream_t stream = (cudaStream_t)stream_;
@@ -219,6 +232,7 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
   a.header = reinterpret_cast<StreamHeader*>(d_out);
   a.pad_start = static_cast<uint8_t*>(d_out) + kHeaderBytes + 4 * C;
   a.pad_len = (uint32_t)(base - kHeaderBytes - 4 * C);
+  a.trace = g_trace_buf;
   if (C == 0) {
     launch_write_header(a, stream);
     ++g_launches;

@@ -80,8 +80,12 @@ __device__ __forceinline__ void lookback_publish(const LaunchCtx& ctx, uint64_t 
 // Called by a whole warp for chunk c: returns the exclusive prefix of the
 // aggregates of chunks [0, c) and publishes chunk c's inclusive prefix. Lane i
 // inspects chunk c−1−i of a 32-chunk window; the window moves back until an
-// inclusive prefix is found. (A 128-wide window with propagation of the
-// resolved prefixes measured 2.8× slower on B200: scripts/ab_time.py.)
+// inclusive prefix is found. (Measured alternatives, all slower on B200 with
+// scripts/ab_time.py: a 128-wide window, propagation of the resolved prefixes,
+// two storer warps per CTA; the poll back-off (16 ns … 1 µs) does not matter.)
+#ifndef LCF_LB_SLEEP
+#define LCF_LB_SLEEP 64
+#endif
 __device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t c, uint64_t agg) {
   const unsigned lane = threadIdx.x & 31;
   if (c == 0) return 0;
@@ -108,7 +112,7 @@ __device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t
       need = first_incl == 32 ? 0xFFFFFFFFu : ((2u << first_incl) - 1u);
       bad = __ballot_sync(0xFFFFFFFFu, !valid) & need;
       if (!bad) break;
-      __nanosleep(64);
+      __nanosleep(LCF_LB_SLEEP);
     }
     uint64_t v = ((int)lane <= first_incl && idx >= 0) ? (s & ((1ull << 40) - 1)) : 0;
 #pragma unroll

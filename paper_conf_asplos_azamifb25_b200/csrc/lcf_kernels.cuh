@@ -40,7 +40,19 @@ struct EncArgs {
   uint32_t pad_len;
   // DPratio: FCM side inputs (per-word distance, 0 = no match)
   const uint32_t* fcm_dist;
+  // optional pipeline trace (scripts/micro/trace_pipeline.cu): 8 globaltimer
+  // stamps per chunk; nullptr in the library
+  unsigned long long* trace;
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void trace_stamp(const EncArgs& a, uint64_t chunk, int k) {
+  if (a.trace) a.trace[chunk * 8 + k] = gtimer();
+}
 
 struct DecArgs {
   const uint8_t* stream;  // 16-byte aligned

@@ -49,6 +49,7 @@ __device__ __forceinline__ void enc_loader(Sm& S, const EncArgs& a, const Launch
     }
     const uint32_t bytes = chunk_words(a.n_words_total, a.first_chunk + t, CW) * wb;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes;
+    if (lane == 0) trace_stamp(a, t, 0);
     if ((bytes & 15) == 0) {
       if (lane == 0) {
         S.in_chunk[s] = t;
@@ -73,7 +74,9 @@ __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const Launch
     const uint64_t t = S.out_chunk[o];
     if (t == kNoChunk) break;
     const uint32_t len = S.out_len[o], raw = S.out_raw[o];
+    if (lane == 0) trace_stamp(a, t, 5);
     const uint64_t excl = lookback_warp(ctx, t, round16(len));
+    if (lane == 0) trace_stamp(a, t, 6);
     if (lane == 0) {
       tma_store_1d(a.payload + excl, S.out[o], (uint32_t)round16(len));
       tma_store_commit();
@@ -82,6 +85,7 @@ __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const Launch
       if (t == 0)
         for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
       tma_store_wait_read0();  // the slot's bytes have been read by the TMA unit
+      trace_stamp(a, t, 7);
       mbar_arrive(&S.empty_out[o]);
     }
     __syncwarp();

@@ -205,6 +205,7 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
       enc_forward_end<kEncOut, kStorers>(S, it, cw, lane);
       return;
     }
+    if (cw == 0 && lane == 0) trace_stamp(a, t, 1);
     const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, CW);
     const bool full = m == (uint32_t)CW;
     const U* in = reinterpret_cast<const U*>(S.in[s]);
@@ -271,8 +272,12 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
     const uint32_t raw_len = m * (uint32_t)sizeof(U);
     const bool raw = total >= raw_len;  // L104, ties → raw
     const uint32_t len = raw ? raw_len : total;
-    if (cw == 0 && lane == 0) lookback_publish(ctx, t, round16(len));
+    if (cw == 0 && lane == 0) {
+      lookback_publish(ctx, t, round16(len));
+      trace_stamp(a, t, 2);
+    }
     mbar_wait(&S.empty_out[o], pho ^ 1);  // output slot free
+    if (cw == 0 && lane == 0) trace_stamp(a, t, 3);
     uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
     if (cw == 0) {
       if (lane == 0) {
@@ -324,6 +329,7 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
     }
     fence_proxy_async_smem();  // packed bytes → visible to the TMA store
     __syncwarp();
+    if (cw == 0 && lane == 0) trace_stamp(a, t, 4);
     if (lane == 0) mbar_arrive(&S.full_out[o]);
   }
 }

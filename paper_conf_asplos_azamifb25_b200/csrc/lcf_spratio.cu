@@ -135,6 +135,7 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
       enc_forward_end<kROut, 1>(S, it, cw, lane);
       return;
     }
+    if (g == 0) trace_stamp(a, t, 1);
     const uint32_t m = chunk_words(a.n_words_total, a.first_chunk + t, 4096);
     const uint32_t G = m / 32;  // full groups; m mod 32 leftover words are copied (A-9)
     const uint32_t* in = S.in[s];
@@ -149,12 +150,16 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
         A[4 * q] = v.x; A[4 * q + 1] = v.y; A[4 * q + 2] = v.z; A[4 * q + 3] = v.w;
       }
       const uint32_t xprev = g ? in[32 * g - 1] : 0u;
+      // word 32g sits at rotated index 4·kx, kx = (8 − gr) mod 8: its predecessor
+      // is xprev (a select per quad start, so that U stays in registers)
+      const uint32_t kx = (8 - gr) & 7;
       uint32_t U[32];
 #pragma unroll
-      for (int j = 0; j < 32; ++j) U[j] = tcms(A[j] - A[(j + 31) & 31]);
-#pragma unroll
-      for (int k = 0; k < 8; ++k)  // word 32g sits at rotated index (32 − 4gr) mod 32
-        if (((8 - gr) & 7) == (uint32_t)k) U[4 * k] = tcms(A[4 * k] - xprev);
+      for (int j = 0; j < 32; ++j) {
+        uint32_t pre = A[(j + 31) & 31];
+        if ((j & 3) == 0) pre = (uint32_t)(j >> 2) == kx ? xprev : pre;
+        U[j] = tcms(A[j] - pre);
+      }
 #pragma unroll
       for (int i = 0; i < 32; ++i) A[i] = U[31 - i];  // rows reversed → planes MSB-first
       transpose32(A);
@@ -252,8 +257,12 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     const uint32_t raw_len = 4 * m;
     const bool raw = total >= raw_len;  // L104, ties → raw
     const uint32_t len = raw ? raw_len : total;
-    if (cw == 0 && lane == 0) lookback_publish(ctx, t, round16(len));
+    if (cw == 0 && lane == 0) {
+      lookback_publish(ctx, t, round16(len));
+      trace_stamp(a, t, 2);
+    }
     mbar_wait(&S.empty_out[o], pho ^ 1);
+    if (g == 0) trace_stamp(a, t, 3);
     uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
     if (cw == 0 && lane == 0) {
       S.out_chunk[o] = t;
@@ -311,6 +320,7 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     }
     fence_proxy_async_smem();
     __syncwarp();
+    if (g == 0) trace_stamp(a, t, 4);
     if (lane == 0) mbar_arrive(&S.full_out[o]);
     bar_r();  // T, B1, B2 and the scan slots are rewritten by the next chunk
   }

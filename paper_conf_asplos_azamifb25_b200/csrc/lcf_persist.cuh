@@ -65,7 +65,10 @@ __device__ __forceinline__ void enc_loader(Sm& S, const EncArgs& a, const Launch
   }
 }
 
-template <int NO, int NSTORERS, class Sm>
+// kInPlace: the compute warps encode into the chunk's own input stage (S.in),
+// and the storer hands that stage back to the loader (S.empty_in) once the TMA
+// unit has read it — no separate output ring.
+template <int NO, int NSTORERS, class Sm, bool kInPlace = false>
 __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
                                            uint32_t first) {
   for (uint32_t it = first;; it += NSTORERS) {
@@ -78,7 +81,10 @@ __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const Launch
     const uint64_t excl = lookback_warp(ctx, t, round16(len));
     if (lane == 0) trace_stamp(a, t, 6);
     if (lane == 0) {
-      tma_store_1d(a.payload + excl, S.out[o], (uint32_t)round16(len));
+      const void* buf;
+      if constexpr (kInPlace) buf = S.in[o];
+      else buf = S.out[o];
+      tma_store_1d(a.payload + excl, buf, (uint32_t)round16(len));
       tma_store_commit();
       a.table[t] = len | (raw ? kRawFlag : 0u);
       if (t == a.n_chunks - 1) finish_encode(a, excl + round16(len));
@@ -86,7 +92,8 @@ __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const Launch
         for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
       tma_store_wait_read0();  // the slot's bytes have been read by the TMA unit
       trace_stamp(a, t, 7);
-      mbar_arrive(&S.empty_out[o]);
+      if constexpr (kInPlace) mbar_arrive(&S.empty_in[o]);
+      else mbar_arrive(&S.empty_out[o]);
     }
     __syncwarp();
   }

@@ -24,7 +24,11 @@ namespace {
 
 constexpr int kRW = 4;                  // compute warps
 constexpr uint32_t kRT = kRW * 32;      // compute threads: one 32-word group each
-constexpr int kRStages = 2, kROut = 2, kRDecStages = 2, kRDecBatch = 4;
+#ifndef LCF_SPR_STAGES
+#define LCF_SPR_STAGES 2
+#endif
+// encode: kRStages input stages, each also the chunk's output buffer (in place)
+constexpr int kRStages = LCF_SPR_STAGES, kRDecStages = 2, kRDecBatch = 4;
 constexpr int kREncThreads = (2 + kRW) * 32, kRDecThreads = (1 + kRW) * 32;
 constexpr uint32_t kBarR = 1;           // named barrier of the compute warps
 
@@ -95,14 +99,13 @@ __device__ __forceinline__ RZESizes rze_sizes(uint32_t L) {
 }
 
 struct REncSmem {
-  alignas(128) uint32_t in[kRStages][4096];
-  alignas(128) uint32_t out[kROut][(kChunkBytes + 64) / 4];
+  alignas(128) uint32_t in[kRStages][4096];  // raw chunk, then its encoding
   alignas(128) uint32_t T[4096];  // BIT output = RZE input D
   alignas(16) uint8_t B1[2048 + 16];
   alignas(16) uint8_t B2[256 + 16];
-  uint64_t full_in[kRStages], empty_in[kRStages], full_out[kROut], empty_out[kROut];
-  uint64_t in_chunk[kRStages], out_chunk[kROut];
-  uint32_t out_len[kROut], out_raw[kROut];
+  uint64_t full_in[kRStages], empty_in[kRStages], full_out[kRStages];
+  uint64_t in_chunk[kRStages], out_chunk[kRStages];
+  uint32_t out_len[kRStages], out_raw[kRStages];
   uint64_t sc64[2][kRW];
   uint32_t sc32[2][kRW];
   uint32_t b3;  // B3 bytes (≤ 32), kept by warp 0 in registers; B4 here
@@ -128,11 +131,12 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
   const uint32_t g = cw * 32 + lane;  // this thread's group
   for (uint32_t it = 0;; ++it) {
     const uint32_t s = it % kRStages, ph = (it / kRStages) & 1;
-    const uint32_t o = it % kROut, pho = (it / kROut) & 1;
     mbar_wait(&S.full_in[s], ph);
     const uint64_t t = S.in_chunk[s];
-    if (t == kNoChunk) {
-      enc_forward_end<kROut, 1>(S, it, cw, lane);
+    if (t == kNoChunk) {  // the stage is ours: forward the end marker through it
+      if (cw == 0 && lane == 0) S.out_chunk[s] = kNoChunk;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.full_out[s]);
       return;
     }
     if (g == 0) trace_stamp(a, t, 1);
@@ -168,15 +172,13 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     } else if (g == G && (m & 31)) {  // leftover words: DIFFMS, copied unchanged by BIT
       for (uint32_t i = 32 * G; i < m; ++i) S.T[i] = tcms(in[i] - (i ? in[i - 1] : 0u));
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&S.empty_in[s]);
     const RZESizes z = rze_sizes(4 * m);
     const uint32_t NU = (z.L + 15) / 16;  // 16-byte units of D
     if (m < 4096) {  // ragged chunk: zero D beyond L and the bitmap tails
       for (uint32_t i = m + g; i < 4096; i += kRT) S.T[i] = 0;
       for (uint32_t i = g; i < (2048 + 16) / 4; i += kRT) reinterpret_cast<uint32_t*>(S.B1)[i] = 0;
     }
-    bar_r();
+    bar_r();  // the stage has been read: from here on it is the output buffer
 
     // ---- 3. RZE (L144–148): B1 and counts of the units u = g + 128k ----
     uint64_t pk[2] = {0, 0};
@@ -261,29 +263,15 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
       lookback_publish(ctx, t, round16(len));
       trace_stamp(a, t, 2);
     }
-    mbar_wait(&S.empty_out[o], pho ^ 1);
     if (g == 0) trace_stamp(a, t, 3);
-    uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
+    uint8_t* ob = reinterpret_cast<uint8_t*>(S.in[s]);
     if (cw == 0 && lane == 0) {
-      S.out_chunk[o] = t;
-      S.out_len[o] = len;
-      S.out_raw[o] = raw;
+      S.out_chunk[s] = t;
+      S.out_len[s] = len;
+      S.out_raw[s] = raw;
     }
-    if (raw) {
-      const uint4* src = reinterpret_cast<const uint4*>(reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes);
-      for (uint32_t q = g; q < round16(len) / 16; q += kRT) {
-        uint4 val;
-        if (16 * q + 16 <= len) {
-          val = __ldcs(src + q);
-        } else {
-          const uint32_t* s32 = reinterpret_cast<const uint32_t*>(src + q);
-          val.x = s32[0];
-          val.y = 16 * q + 4 < len ? s32[1] : 0u;
-          val.z = 16 * q + 8 < len ? s32[2] : 0u;
-          val.w = 16 * q + 12 < len ? s32[3] : 0u;
-        }
-        reinterpret_cast<uint4*>(ob)[q] = val;
-      }
+    if (raw) {  // the stage still holds the raw chunk: zero its padding
+      if (g < round16(len) - len) ob[len + g] = 0;
     } else {
       // nz(D): non-zero bytes of every unit at its scanned offset
 #pragma unroll
@@ -321,7 +309,7 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     fence_proxy_async_smem();
     __syncwarp();
     if (g == 0) trace_stamp(a, t, 4);
-    if (lane == 0) mbar_arrive(&S.full_out[o]);
+    if (lane == 0) mbar_arrive(&S.full_out[s]);
     bar_r();  // T, B1, B2 and the scan slots are rewritten by the next chunk
   }
 }
@@ -333,17 +321,14 @@ __global__ void __launch_bounds__(kREncThreads) spratio_encode_kernel(EncArgs a,
   if (threadIdx.x == 0) {
     for (int i = 0; i < kRStages; ++i) {
       mbar_init(&S.full_in[i], 1);
-      mbar_init(&S.empty_in[i], kRW);
-    }
-    for (int i = 0; i < kROut; ++i) {
+      mbar_init(&S.empty_in[i], 1);  // released by the storer
       mbar_init(&S.full_out[i], kRW);
-      mbar_init(&S.empty_out[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
   if (warp == 0) enc_loader<kRStages>(S, a, ctx, lane, 4);
-  else if (warp == 1) enc_storer<kROut, 1>(S, a, ctx, lane, 0);
+  else if (warp == 1) enc_storer<kRStages, 1, REncSmem, true>(S, a, ctx, lane, 0);
   else r_enc_compute(S, a, ctx, warp - 2, lane);
 }
 

@@ -28,7 +28,10 @@ constexpr uint32_t kRT = kRW * 32;      // compute threads: one 32-word group ea
 #define LCF_SPR_STAGES 2
 #endif
 // encode: kRStages input stages, each also the chunk's output buffer (in place)
-constexpr int kRStages = LCF_SPR_STAGES, kRDecStages = 2, kRDecBatch = 4;
+#ifndef LCF_SPR_DSTAGES
+#define LCF_SPR_DSTAGES 2
+#endif
+constexpr int kRStages = LCF_SPR_STAGES, kRDecStages = LCF_SPR_DSTAGES, kRDecBatch = 4;
 constexpr int kREncThreads = (2 + kRW) * 32, kRDecThreads = (1 + kRW) * 32;
 constexpr uint32_t kBarR = 1;           // named barrier of the compute warps
 
@@ -113,8 +116,9 @@ struct REncSmem {
 
 struct RDecSmem {
   alignas(128) uint32_t in[kRDecStages][(kChunkBytes + 64) / 4];
-  alignas(128) uint32_t T[4096];
-  alignas(128) uint32_t X[kRT * 33];  // decoded words, 33-word row stride (conflict-free)
+  // T: decoded D (plane-major, 4096 words), then — once every thread holds its
+  // group in registers — the decoded words with a 33-word row stride (X)
+  alignas(128) uint32_t T[kRT * 33];
   alignas(16) uint8_t B1[2048 + 16];
   alignas(16) uint8_t B2[256 + 16];
   uint64_t full_in[kRDecStages], empty_in[kRDecStages];
@@ -500,27 +504,27 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
         tot += tcms_inv(X[i]);
         X[i] = tot;
       }
-    } else if (g == G && (m & 31)) {
-      for (uint32_t i = 32 * G; i < m; ++i) tot += tcms_inv(S.T[i]);
+    } else if (g == G && (m & 31)) {  // leftover words (A-9): DIFFMS⁻¹ only
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if ((uint32_t)i < (m & 31)) tot += tcms_inv(S.T[32 * G + i]);
+        X[i] = tot;
+      }
     }
     uint32_t all;
+    // the scan's barrier also ends every read of T: X overwrites it below
     const uint32_t base = cta_excl_scan<uint32_t>(tot, S.sc32[1], cw, lane, all);
-    if (g < G) {
+    uint32_t* const Xs = S.T;
+    if (g < G || (g == G && (m & 31))) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) S.X[g * 33 + i] = X[i] + base;
-    } else if (g == G && (m & 31)) {
-      uint32_t run = base;
-      for (uint32_t i = 32 * G; i < m; ++i) {
-        run += tcms_inv(S.T[i]);
-        S.X[G * 33 + (i - 32 * G)] = run;
-      }
+      for (int i = 0; i < 32; ++i) Xs[g * 33 + i] = X[i] + base;
     }
     bar_r();
     // coalesced 16-byte stores of words n = 4q .. 4q+3
     for (uint32_t q = g; q < 1024; q += kRT) {
       const uint32_t n = 4 * q;
       if (n >= m) break;
-      const uint32_t* row = S.X + (n >> 5) * 33 + (n & 31);
+      const uint32_t* row = Xs + (n >> 5) * 33 + (n & 31);
       if (n + 4 <= m) {
         __stcs(reinterpret_cast<uint4*>(dst) + q, make_uint4(row[0], row[1], row[2], row[3]));
       } else {

@@ -35,6 +35,7 @@ constexpr int kDOut = LCF_DP_OUT, kDBatch = 4;  // output slots (encode), tiles 
 constexpr int kDEncThreads = (2 + kDW) * 32, kDDecThreads = (1 + kDW) * 32;
 constexpr uint32_t kBarD = 1;
 constexpr uint32_t kTileWords = 2048;
+static_assert(kDT * 8 == kTileWords, "the raw V fallback gives each compute thread 8 words");
 constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
 
 __device__ __forceinline__ void bar_d() { named_bar_sync(kBarD, kDT); }
@@ -138,11 +139,12 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint32_t n = L / 8, tl = L % 8;
   const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
+  const uint32_t R = (n + kDT - 1) / kDT;  // rounds holding words
   if (tid < 65) sc.hist[tid] = 0;
   bar_d();
   // ---- histogram of clz(v_i ⊕ ref_i), warp-aggregated shared atomics ----
 #pragma unroll 1
-  for (uint32_t r = 0; r < 8; ++r) {
+  for (uint32_t r = 0; r < R; ++r) {
     const uint32_t i = tid + kDT * r;
     uint32_t z = 65u;
     if (i < n) z = clz64(sv[i] ^ ((rare && i) ? sv[i - 1] : 0ull));
@@ -273,8 +275,9 @@ __device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8
   const uint64_t hi_base = 24, lo_base = 8ull * (3 + hib);
   const uint32_t wl = 64 - k;
   const uint64_t lmask = wl >= 64 ? ~0ull : ((1ull << wl) - 1);
+  const uint32_t R = (n + kDT - 1) / kDT;  // later rounds hold no words
 #pragma unroll 1
-  for (uint32_t r = 0; r < 8; ++r) {
+  for (uint32_t r = 0; r < R; ++r) {
     const uint32_t i = tid + kDT * r;
     const uint32_t q = r * kDW + warp;
     const uint32_t bal = sc.b1[q];
@@ -447,12 +450,14 @@ __device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t* sh, uint3
 struct DEncSmem {
   alignas(128) uint64_t xin[kTileWords];        // stage: x tile
   alignas(128) uint32_t din[kTileWords];        // stage: FCM distances of the tile
+  alignas(128) uint32_t dcp[kTileWords];        // copy of din: the stage is released after V's DIFFMS
   alignas(128) uint64_t w[kTileWords + 8];      // DIFFMS words of V or Dist
   alignas(128) uint8_t rz[kChunkBytes + 128];   // RAZE output
   alignas(128) uint32_t out[kDOut][(kChunkBytes + 128) / 4];
   uint64_t full_in[1], empty_in[1], full_out[kDOut], empty_out[kDOut];
   uint64_t in_chunk[1], out_chunk[kDOut];
   uint32_t out_len[kDOut], out_raw[kDOut];
+  uint64_t scan[kDW];
   AdaptScratch sc;
 };
 
@@ -508,21 +513,39 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
     for (uint32_t part = 0; part < 2; ++part, ++oit) {  // chunk 2t: V, chunk 2t+1: Dist (A-16)
       const uint64_t c = 2 * t + part;
       // FCM outputs (L170–185) and DIFFMS₆₄ (L187) into w[]
+      uint64_t nzacc = 0;
       for (uint32_t i = tid; i < m; i += kDT) {
-        const uint32_t d = S.din[i], dp = i ? S.din[i - 1] : 0u;
         uint64_t cur, prev;
         if (part == 0) {
+          const uint32_t d = S.din[i], dp = i ? S.din[i - 1] : 0u;
           cur = d ? 0ull : S.xin[i];
           prev = i ? (dp ? 0ull : S.xin[i - 1]) : 0ull;
+          S.dcp[i] = d;
         } else {
-          cur = d;
-          prev = i ? (uint64_t)dp : 0ull;
+          cur = S.dcp[i];
+          prev = i ? (uint64_t)S.dcp[i - 1] : 0ull;
         }
-        S.w[i] = tcms((uint64_t)(cur - prev));
+        const uint64_t wv = tcms((uint64_t)(cur - prev));
+        S.w[i] = wv;
+        nzacc |= wv;
       }
-      bar_d();
       // RAZE then RARE (L189–201)
-      const uint32_t l1 = adaptive_encode(reinterpret_cast<const uint8_t*>(S.w), 8 * m, S.rz, false, S.sc, tid);
+      uint32_t l1;
+      const bool any = bar_d_or(nzacc != 0);
+      // the tile's stage has been read (V's DIFFMS words are in w, the
+      // distances in dcp): hand it back so the next tile loads during this one
+      if (part == 0 && lane == 0) mbar_arrive(&S.empty_in[0]);
+      if (any) {
+        l1 = adaptive_encode(reinterpret_cast<const uint8_t*>(S.w), 8 * m, S.rz, false, S.sc, tid);
+      } else {
+        // all-zero DIFFMS words (e.g. the Dist chunk of a tile without FCM
+        // matches): RAZE's plan is fixed — every clz is 64, so k = 64, B1..B3
+        // are zero and nothing repeats — and the stream is L | k=64 | L3 zero
+        // bytes (FORMAT.md §6.2; the same bytes adaptive_encode writes)
+        const uint32_t L = 8 * m, L3 = (((m + 7) / 8 + 7) / 8 + 7) / 8;
+        if (tid < 3 + L3) S.rz[tid] = tid == 0 ? (uint8_t)L : tid == 1 ? (uint8_t)(L >> 8) : tid == 2 ? 64 : 0;
+        l1 = 3 + L3;
+      }
       // RARE is planned first: the chunk's size — and its aggregate for the
       // look-back of later chunks — is known before an output slot is needed
       const uint32_t l2 = adaptive_plan(S.rz, l1, true, S.sc, tid);
@@ -534,9 +557,28 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       mbar_wait(&S.empty_out[o], pho ^ 1);
       uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       if (raw) {  // the V / Dist words themselves
-        for (uint32_t i = tid; i < m; i += kDT)
-          reinterpret_cast<uint64_t*>(ob)[i] = part == 0 ? (S.din[i] ? 0ull : S.xin[i]) : (uint64_t)S.din[i];
-        if (tid < 2 && (m & 1)) reinterpret_cast<uint64_t*>(ob)[m + tid] = 0;  // round16 pad
+        uint64_t* ow = reinterpret_cast<uint64_t*>(ob);
+        if (part == 0) {  // V = DIFFMS⁻¹(w): words 8·tid .. 8·tid+7, serial run + CTA scan
+          uint64_t run = 0;
+#pragma unroll
+          for (uint32_t j = 0; j < 8; ++j) {
+            const uint32_t i = 8 * tid + j;
+            if (i < m) run += tcms_inv(S.w[i]);
+          }
+          uint64_t all;
+          uint64_t v = cta_scan_u64(run, S.scan, tid, all);
+#pragma unroll
+          for (uint32_t j = 0; j < 8; ++j) {
+            const uint32_t i = 8 * tid + j;
+            if (i < m) {
+              v += tcms_inv(S.w[i]);
+              ow[i] = v;
+            }
+          }
+        } else {
+          for (uint32_t i = tid; i < m; i += kDT) ow[i] = S.dcp[i];
+        }
+        if (tid < 2 && (m & 1)) ow[m + tid] = 0;  // round16 pad
       } else {
         adaptive_emit(S.rz, l1, ob, true, S.sc, tid);
         if (tid < 16 && len + tid < round16(len)) ob[len + tid] = 0;
@@ -550,7 +592,6 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       bar_d();
       if (lane == 0) mbar_arrive(&S.full_out[o]);
     }
-    if (lane == 0) mbar_arrive(&S.empty_in[0]);
   }
 }
 

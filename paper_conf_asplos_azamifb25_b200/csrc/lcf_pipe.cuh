@@ -30,9 +30,29 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+#ifndef LCF_MBAR_HINT
+#define LCF_MBAR_HINT 0
+#endif
+// try_wait with a suspend-time hint (ns): the waiting warp is descheduled until
+// the phase completes or the hint expires, instead of spinning on issue slots.
+__device__ __forceinline__ bool mbar_try_wait_hint(uint64_t* bar, uint32_t parity, uint32_t ns) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2, %3;\n"
+      " selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_addr(bar)), "r"(parity), "r"(ns)
+      : "memory");
+  return ok != 0;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#if LCF_MBAR_HINT
+  while (!mbar_try_wait_hint(bar, parity, LCF_MBAR_HINT)) {
+  }
+#else
   while (!mbar_try_wait(bar, parity)) {
   }
+#endif
 }
 
 // ---- TMA bulk copies (non-tensor, 16-byte granules) ---------------------------

@@ -156,9 +156,11 @@ def kernel_bytes(j):
         return {"speed_encode_u64": io, "speed_decode_u64": io}
     if codec == "SPratio":
         return {"spratio_encode": io, "spratio_decode": io}
-    return {"fcm_hash": 20 * words,                   # x in, 20-bit key + (fold, index) payload out
-            "cub_radix_sort_pairs": 76 * words,       # 3 passes × 12 B in/out + histogram read
-            "fcm_match": 12 * words,                  # sorted keys + payloads in (matches scattered)
+    tiles = -(-words // 16384)
+    return {"fcm_sort_hist": 8 * words,               # x (pass 1) or pass-1 records (pass 2) in
+            "fcm_sort_scan": 8 * 1024 * tiles,        # the tile × digit count matrix, read and rewritten
+            "fcm_sort_scatter": 16 * words,           # 8-byte records (or x) in, records out
+            "fcm_match": 8 * words,                   # sorted records in (x gathered, matches scattered)
             "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
             "dpratio_decode": sb + n}                 # stream in, x out
 

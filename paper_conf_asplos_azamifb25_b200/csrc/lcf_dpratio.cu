@@ -19,7 +19,6 @@
 //   inside the tile are resolved by pointer jumping in shared memory, references
 //   to earlier tiles read the already written output after an acquire on that
 //   tile's completion flag (tiles complete in ticket order, so no cycles).
-#include <cub/cub.cuh>
 
 #include "lcf_persist.cuh"
 
@@ -36,7 +35,6 @@ constexpr int kDEncThreads = (2 + kDW) * 32, kDDecThreads = (1 + kDW) * 32;
 constexpr uint32_t kBarD = 1;
 constexpr uint32_t kTileWords = 2048;
 static_assert(kDT * 8 == kTileWords, "the raw V fallback gives each compute thread 8 words");
-constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
 
 __device__ __forceinline__ void bar_d() { named_bar_sync(kBarD, kDT); }
 __device__ __forceinline__ bool bar_d_or(bool p) {
@@ -46,64 +44,6 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
                : "r"((uint32_t)p), "r"(kBarD), "r"(kDT)
                : "memory");
   return r != 0;
-}
-
-// =============================== FCM encode kernels ===============================
-__global__ void fcm_hash_kernel(const uint64_t* __restrict__ x, uint64_t n, uint32_t* __restrict__ key,
-                                uint64_t* __restrict__ val) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t a = i >= 1 ? x[i - 1] : 0, b = i >= 2 ? x[i - 2] : 0, c = i >= 3 ? x[i - 3] : 0;
-    key[i] = (uint32_t)(((a * FCM_K1) ^ (b * FCM_K2) ^ (c * FCM_K3)) >> 44);
-    // sort payload: the index and a 32-bit fold of x[i]; unequal folds prove
-    // unequal words, so the match kernel gathers x only for likely matches
-    const uint64_t xi = x[i];
-    val[i] = ((uint64_t)(uint32_t)(xi ^ (xi >> 32)) << 32) | (uint32_t)i;
-  }
-}
-
-constexpr int kMatchBlock = 256;
-// One thread per sorted position k: the nearest of the pairs k−1 … k−4 with the
-// same hash and a bitwise-equal word is the match (L174, A-14, A-15). The
-// distance array is pre-zeroed; only matches are scattered.
-__global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
-                                                                const uint32_t* __restrict__ key,
-                                                                const uint64_t* __restrict__ val,
-                                                                uint32_t* __restrict__ dist) {
-  __shared__ uint32_t sk[kMatchBlock + 4];
-  __shared__ uint64_t sv[kMatchBlock + 4];
-  for (uint64_t b0 = blockIdx.x * (uint64_t)kMatchBlock; b0 < n; b0 += (uint64_t)gridDim.x * kMatchBlock) {
-    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {  // sorted window [b0 − 4, b0 + 256)
-      const int64_t k = (int64_t)b0 - 4 + j;
-      const bool in = k >= 0 && (uint64_t)k < n;
-      sk[j] = in ? key[k] : 0xFFFFFFFFu;  // never equals a 20-bit hash
-      sv[j] = in ? val[k] : 0;
-    }
-    __syncthreads();
-    const uint64_t k = b0 + threadIdx.x;
-    if (k < n) {
-      const int j = threadIdx.x + 4;
-      const uint32_t h = sk[j], i = (uint32_t)sv[j], fp = (uint32_t)(sv[j] >> 32);
-      uint32_t d = 0;
-      uint64_t xi = 0;
-      bool have = false;
-#pragma unroll
-      for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
-        if (sk[j - back] == h && (uint32_t)(sv[j - back] >> 32) == fp) {
-          const uint32_t jj = (uint32_t)sv[j - back];
-          if (!have) {
-            xi = x[i];
-            have = true;
-          }
-          if (x[jj] == xi) {
-            d = i - jj;
-            break;
-          }
-        }
-      }
-      if (d) dist[i] = d;
-    }
-    __syncthreads();
-  }
 }
 
 // ============================ RAZE / RARE in shared memory ============================
@@ -826,50 +766,14 @@ __global__ void __launch_bounds__(kDDecThreads) dpratio_decode_kernel(DecArgs a,
 }  // namespace
 
 // ---- host side -------------------------------------------------------------------
-size_t dpratio_fcm_workspace(uint64_t n) {
-  size_t temp = 0;
-  cub::DoubleBuffer<uint32_t> dk(nullptr, nullptr);
-  cub::DoubleBuffer<uint64_t> dv(nullptr, nullptr);
-  cub::DeviceRadixSort::SortPairs(nullptr, temp, dk, dv, (int)n, 0, 20);
-  return 2 * round16(n * 4) + 2 * round16(n * 8) + round16(temp) + 256;
-}
+size_t dpratio_fcm_workspace(uint64_t n) { return fcm_dist_workspace(n); }
 
 int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st) {
   const uint64_t n = a0.n_words_total;
-  uint8_t* p = static_cast<uint8_t*>(ws);
-  uint32_t* key_a = reinterpret_cast<uint32_t*>(p);
-  uint32_t* key_b = reinterpret_cast<uint32_t*>(p + round16(4 * n));
-  uint64_t* val_a = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n));
-  uint64_t* val_b = reinterpret_cast<uint64_t*>(p + 2 * round16(4 * n) + round16(8 * n));
-  void* temp = p + 2 * round16(4 * n) + 2 * round16(8 * n);
-  size_t temp_bytes = ws_bytes - (2 * round16(4 * n) + 2 * round16(8 * n));
   int launches = 0;
   if (n) {
-    const int blocks = (int)umin64((n + 255) / 256, 148 * 16);
-    {
-      KTrace kt("fcm_hash", st);
-      fcm_hash_kernel<<<blocks, 256, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_a, val_a);
-    }
-    ++launches;
-    // (h, i) pairs by the 20 key bits; stable, so equal hashes keep index order
-    cub::DoubleBuffer<uint32_t> dk(key_a, key_b);
-    cub::DoubleBuffer<uint64_t> dv(val_a, val_b);
-    {
-      KTrace kt("cub_radix_sort_pairs", st);
-      cub::DeviceRadixSort::SortPairs(temp, temp_bytes, dk, dv, (int)n, 0, 20, st);
-    }
-    const uint32_t* key_out = dk.Current();
-    const uint64_t* val_out = dv.Current();
-    uint32_t* key_in = dk.Alternate();
-    uint32_t* dist = key_in;  // the unsorted keys are dead after the sort
-    cudaMemsetAsync(dist, 0, 4 * n, st);
-    const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
-    {
-      KTrace kt("fcm_match", st);
-      fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(reinterpret_cast<const uint64_t*>(a0.in), n, key_out,
-                                                        val_out, dist);
-    }
-    ++launches;
+    uint32_t* dist = nullptr;  // FCM distances (L170–185), lcf_fcm.cu
+    launches += launch_fcm_dist(reinterpret_cast<const uint64_t*>(a0.in), n, ws, ws_bytes, st, &dist);
     EncArgs a = a0;
     a.fcm_dist = dist;
     const size_t smem = sizeof(DEncSmem);

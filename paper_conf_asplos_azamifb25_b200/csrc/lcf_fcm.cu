@@ -1,0 +1,386 @@
+// lcf_fcm.cu — the FCM distance array of DPratio (§3.4) on
+// sm_100a, without a library sort.
+//
+// L172–176: hash the three preceding words of every position i, sort the
+// pairs (h, i), and find for i the nearest of the (up to) four preceding pairs
+// in sorted order with the same hash whose word equals x[i]; dist[i] = i − j.
+//
+// The (h, i) order is produced by a two-pass stable LSD radix sort over the two
+// 10-bit digits of the 20-bit hash. Pass 1 reads x itself (the hash is computed
+// on the fly from a warp's 32 consecutive words plus three carried words), so
+// there is no separate hash array. A sort record is one u64:
+//     h (20 bits) | fp (12-bit fingerprint of x[i]) | i (32 bits)
+// and the match kernel gathers x only where fingerprints agree.
+//
+// Each pass is three kernels over tiles of kTile = 16 Ki records, 16 warps per
+// tile, warp w owning records [w·1024, (w+1)·1024) of the tile:
+//   sort_hist    per-tile digit counts (warp-aggregated shared atomics)
+//   sort_scan    per-digit exclusive prefix over tiles (column scan) + totals
+//   sort_scatter per-warp digit counts → per-warp offsets inside the tile's
+//                digit run; then each warp walks its records in order and
+//                ranks equal digits with __match_any_sync → stable scatter
+#include "lcf_kernels.cuh"
+
+namespace lcf {
+namespace {
+
+constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
+constexpr int kDigitBits = 10, kDigits = 1 << kDigitBits;
+constexpr int kSortWarps = 16, kSortThreads = kSortWarps * 32, kWarpRecs = 1024;
+constexpr uint32_t kTile = kSortWarps * kWarpRecs;
+constexpr int kRecHashShift = 44, kRecFpShift = 32;
+constexpr uint64_t kRecIdxMask = 0xFFFFFFFFull;
+constexpr uint32_t kNoDigit = kDigits;  // records past n
+constexpr int kMatchBlock = 256;
+constexpr int kScanWarps = 32, kScanBlocks = kDigits / 32;
+
+__device__ __forceinline__ uint32_t rec_digit(uint64_t rec, int pass) {
+  return pass == 0 ? (uint32_t)(rec >> kRecHashShift) & (kDigits - 1) : (uint32_t)(rec >> (kRecHashShift + kDigitBits));
+}
+
+// Record from x[i] and the high words of the three hash products (only bits
+// 44..63 of the 64-bit hash value are kept: bits 12..31 of its high word).
+__device__ __forceinline__ uint64_t make_rec(uint64_t xi, uint32_t hw, uint64_t i) {
+  const uint64_t h = hw >> 12;  // 20-bit hash (A-14)
+  const uint32_t f = (uint32_t)(xi ^ (xi >> 32));
+  const uint32_t fp = (f ^ (f >> 12) ^ (f >> 24)) & 0xFFFu;
+  return (h << kRecHashShift) | ((uint64_t)fp << kRecFpShift) | i;
+}
+__device__ __forceinline__ uint32_t hi_mul(uint64_t a, uint64_t k) { return (uint32_t)((a * k) >> 32); }
+
+// Lanes of the warp holding the same digit as this lane (valid lanes only):
+// ten ballots, one per digit bit — ALU-pipe votes instead of __match_any_sync,
+// whose long MIO latency serialised the ranking loop.
+__device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
+  uint32_t peers = __ballot_sync(0xFFFFFFFFu, valid);
+#pragma unroll
+  for (int b = 0; b < kDigitBits; ++b) {
+    const bool bit = (d >> b) & 1;
+    const uint32_t bb = __ballot_sync(0xFFFFFFFFu, bit);
+    peers &= bit ? bb : ~bb;
+  }
+  return peers;
+}
+
+// The records of one warp's range in index order, kBatch·32 at a time: all
+// loads of a batch are issued before any record is formed (memory-level
+// parallelism). Pass 0 builds records from x: lane l computes the products
+// x[i]·K1, x[i]·K2, x[i]·K3 of its own word and the hash of position i takes
+// them from lanes l−1, l−2, l−3 (one 32-bit rotation shuffle each); lanes
+// 0..2 use the rotated values of the previous group. Pass 1 reads the
+// records of pass 0.
+constexpr int kBatch = 8;
+template <int PASS>
+struct RecReader {
+  const uint64_t* src;
+  uint64_t n, i0;
+  uint32_t r1p, r2p, r3p;  // previous group's rotated product words (pass 0)
+  uint64_t v[kBatch];
+  __device__ __forceinline__ RecReader(const uint64_t* s, uint64_t n_, uint64_t start, uint32_t lane)
+      : src(s), n(n_), i0(start) {
+    if (PASS == 0) {  // the group before `start`: only its lanes 29..31 matter
+      const int64_t j = (int64_t)start - 32 + (int64_t)lane;
+      const uint64_t y = (lane >= 29 && j >= 0 && (uint64_t)j < n) ? src[j] : 0;
+      rotate(y, lane, r1p, r2p, r3p);
+    }
+  }
+  __device__ __forceinline__ static void rotate(uint64_t y, uint32_t lane, uint32_t& r1, uint32_t& r2,
+                                                uint32_t& r3) {
+    r1 = __shfl_sync(0xFFFFFFFFu, hi_mul(y, FCM_K1), (lane + 31) & 31);
+    r2 = __shfl_sync(0xFFFFFFFFu, hi_mul(y, FCM_K2), (lane + 30) & 31);
+    r3 = __shfl_sync(0xFFFFFFFFu, hi_mul(y, FCM_K3), (lane + 29) & 31);
+  }
+  __device__ __forceinline__ void load(uint32_t lane) {
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      const uint64_t i = i0 + 32 * k + lane;
+      v[k] = i < n ? src[i] : 0;
+    }
+  }
+  // record of group k of the loaded batch (index i0 + 32k + lane)
+  __device__ __forceinline__ uint64_t rec(int k, uint32_t lane, bool& valid) {
+    const uint64_t i = i0 + 32 * k + lane;
+    valid = i < n;
+    if (PASS == 1) return v[k];
+    uint32_t r1, r2, r3;
+    rotate(v[k], lane, r1, r2, r3);
+    const uint32_t a1 = lane >= 1 ? r1 : r1p, a2 = lane >= 2 ? r2 : r2p, a3 = lane >= 3 ? r3 : r3p;
+    r1p = r1;
+    r2p = r2;
+    r3p = r3;
+    return make_rec(v[k], a1 ^ a2 ^ a3, i);
+  }
+  __device__ __forceinline__ void advance() { i0 += 32 * kBatch; }
+};
+
+template <int PASS>
+__global__ void __launch_bounds__(kSortThreads) sort_hist_kernel(const uint64_t* __restrict__ src, uint64_t n,
+                                                                 uint32_t* __restrict__ counts) {
+  __shared__ uint32_t hist[kDigits];
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (uint32_t d = threadIdx.x; d < kDigits; d += kSortThreads) hist[d] = 0;
+  __syncthreads();
+  const uint64_t start = (uint64_t)blockIdx.x * kTile + warp * kWarpRecs;
+  RecReader<PASS> rd(src, n, start, lane);
+  for (int s = 0; s < kWarpRecs / (32 * kBatch); ++s, rd.advance()) {
+    if (rd.i0 >= n) break;  // warp-uniform
+    rd.load(lane);
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      bool valid;
+      const uint64_t rec = rd.rec(k, lane, valid);
+      const uint32_t d = valid ? rec_digit(rec, PASS) : kNoDigit;
+      if (valid) atomicAdd(&hist[d], 1u);
+    }
+  }
+  __syncthreads();
+  for (uint32_t d = threadIdx.x; d < kDigits; d += kSortThreads) counts[(uint64_t)blockIdx.x * kDigits + d] = hist[d];
+}
+
+// counts[t][d] → exclusive prefix over tiles t of digit d; tot[d] = total.
+__global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __restrict__ counts, uint32_t n_tiles,
+                                                                   uint32_t* __restrict__ tot) {
+  __shared__ uint32_t part[kScanWarps][32];
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t d = blockIdx.x * 32 + lane;
+  const uint32_t t0 = (uint32_t)((uint64_t)warp * n_tiles / kScanWarps);
+  const uint32_t t1 = (uint32_t)((uint64_t)(warp + 1) * n_tiles / kScanWarps);
+  uint32_t s = 0;
+  for (uint32_t t = t0; t < t1; ++t) s += counts[(uint64_t)t * kDigits + d];
+  part[warp][lane] = s;
+  __syncthreads();
+  uint32_t run = 0;
+  for (uint32_t w = 0; w < warp; ++w) run += part[w][lane];
+  if (warp == kScanWarps - 1) tot[d] = run + s;
+  for (uint32_t t = t0; t < t1; ++t) {
+    uint32_t* c = counts + (uint64_t)t * kDigits + d;
+    const uint32_t v = *c;
+    *c = run;
+    run += v;
+  }
+}
+
+// Stable scatter of one tile, in kRounds rounds of kRound records; in round r
+// warp w owns records [r·kRound + w·256, +256) of the tile (8 groups of 32, one
+// register batch), so round, warp, group and lane order is index order.
+//   1. per-warp digit counts (packed u16 pairs, shared atomics)
+//   2. per digit: exclusive prefix over the warps; the round's digit starts
+//   3. rank inside the warp (ballot-matched equal digits, lane order) and put
+//      the record at its sorted place in the round's shared stage
+//   4. copy the stage out: record j of digit d goes to run[d] + j − start[d],
+//      so consecutive threads write consecutive positions of a digit run
+constexpr int kRound = kSortWarps * 32 * kBatch;  // 4096 records
+constexpr int kRounds = kTile / kRound;
+static_assert(kRounds * kRound == kTile, "tile = whole rounds");
+struct ScatterSmem {
+  uint64_t stage[kRound];
+  uint32_t wcnt[kSortWarps][kDigits / 2];  // packed u16 pair per word
+  uint32_t run[kDigits];                   // next output position of each digit (tile-wide)
+  uint32_t rstart[kDigits];                // round: first stage slot of each digit
+  uint32_t rtot[kDigits / 2];              // round: packed digit totals
+  uint32_t wsum[kSortWarps];
+};
+
+template <int PASS>
+__global__ void __launch_bounds__(kSortThreads) sort_scatter_kernel(const uint64_t* __restrict__ src, uint64_t n,
+                                                                    const uint32_t* __restrict__ offs,
+                                                                    const uint32_t* __restrict__ tot,
+                                                                    uint64_t* __restrict__ dst) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
+  const uint32_t tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint32_t lt = (1u << lane) - 1u;
+  // block exclusive scan of (a, b) pairs, one pair per thread → (ex_a, ex_a + a)
+  auto pair_scan = [&](uint32_t a, uint32_t b) -> uint32_t {
+    uint32_t x = a + b;
+#pragma unroll
+    for (int k = 1; k < 32; k <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, k);
+      if ((int)lane >= k) x += y;
+    }
+    if (lane == 31) S.wsum[warp] = x;
+    __syncthreads();
+    uint32_t base = 0;
+    for (uint32_t w = 0; w < warp; ++w) base += S.wsum[w];
+    return base + x - a - b;
+  };
+  {  // digit bases (exclusive scan of tot) + this tile's offsets
+    const uint32_t a = tot[2 * tid], b = tot[2 * tid + 1];
+    const uint32_t ex = pair_scan(a, b);
+    const uint32_t* o = offs + (uint64_t)blockIdx.x * kDigits;
+    S.run[2 * tid] = ex + o[2 * tid];
+    S.run[2 * tid + 1] = ex + a + o[2 * tid + 1];
+  }
+  const uint64_t tile0 = (uint64_t)blockIdx.x * kTile;
+  for (int r = 0; r < kRounds; ++r) {
+    const uint64_t r0 = tile0 + (uint64_t)r * kRound;
+    if (r0 >= n) break;  // block-uniform
+    const uint32_t nr = (uint32_t)umin64(kRound, n - r0);
+    // 1. records of this warp's 256 and its digit counts
+    RecReader<PASS> rd(src, n, r0 + warp * 32 * kBatch, lane);
+    rd.load(lane);
+#pragma unroll
+    for (int j = lane; j < kDigits / 2; j += 32) S.wcnt[warp][j] = 0;
+    __syncwarp();
+    uint64_t rec[kBatch];
+    uint32_t dg[kBatch];
+    bool ok[kBatch];
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      rec[k] = rd.rec(k, lane, ok[k]);
+      dg[k] = ok[k] ? rec_digit(rec[k], PASS) : 0u;
+      if (ok[k]) atomicAdd(&S.wcnt[warp][dg[k] >> 1], 1u << (16 * (dg[k] & 1)));
+    }
+    __syncthreads();
+    // 2. digits 2·tid, 2·tid+1: prefix over the warps (packed: sums ≤ 4096 per half)
+    uint32_t tw = 0;
+#pragma unroll
+    for (int w = 0; w < kSortWarps; ++w) {
+      const uint32_t c = S.wcnt[w][tid];
+      S.wcnt[w][tid] = tw;
+      tw += c;
+    }
+    S.rtot[tid] = tw;
+    {
+      const uint32_t a = tw & 0xFFFFu, b = tw >> 16;
+      const uint32_t ex = pair_scan(a, b);  // (contains the barrier that publishes wcnt)
+      S.rstart[2 * tid] = ex;
+      S.rstart[2 * tid + 1] = ex + a;
+    }
+    __syncthreads();
+    // 3. ranks → stage
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      const uint32_t d = dg[k];
+      const uint32_t peers = digit_peers(d, ok[k]);
+      uint32_t* wc = &S.wcnt[warp][d >> 1];
+      const uint32_t sh = 16 * (d & 1);
+      const uint32_t rbase = ok[k] ? (*wc >> sh) & 0xFFFFu : 0u;
+      __syncwarp();
+      if (ok[k]) {
+        S.stage[S.rstart[d] + rbase + __popc(peers & lt)] = rec[k];
+        if (lane == (uint32_t)__ffs(peers) - 1) atomicAdd(wc, (uint32_t)__popc(peers) << sh);
+      }
+      __syncwarp();
+    }
+    __syncthreads();
+    // 4. stage → dst, digit runs contiguous
+    for (uint32_t j = tid; j < nr; j += kSortThreads) {
+      const uint64_t v = S.stage[j];
+      const uint32_t d = rec_digit(v, PASS);
+      dst[S.run[d] + (j - S.rstart[d])] = v;
+    }
+    __syncthreads();
+    {
+      const uint32_t t2 = S.rtot[tid];
+      S.run[2 * tid] += t2 & 0xFFFFu;
+      S.run[2 * tid + 1] += t2 >> 16;
+    }
+    // (the next round's first barrier orders these updates before step 4)
+  }
+}
+
+// One thread per sorted position k: the nearest of the records k−1 … k−4 with
+// the same hash and an equal word is the match (L174, A-14, A-15). Records of
+// one hash are contiguous, so the walk stops at the first other hash. The
+// distance array is pre-zeroed; only matches are scattered.
+__global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
+                                                                const uint64_t* __restrict__ rec,
+                                                                uint32_t* __restrict__ dist) {
+  __shared__ uint64_t sr[kMatchBlock + 4];
+  for (uint64_t b0 = blockIdx.x * (uint64_t)kMatchBlock; b0 < n; b0 += (uint64_t)gridDim.x * kMatchBlock) {
+    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {  // sorted window [b0 − 4, b0 + 256)
+      const int64_t k = (int64_t)b0 - 4 + j;
+      sr[j] = (k >= 0 && (uint64_t)k < n) ? rec[k] : 0;  // padding is never read as a predecessor
+    }
+    __syncthreads();
+    const uint64_t k = b0 + threadIdx.x;
+    if (k < n) {
+      const int j = threadIdx.x + 4;
+      const uint64_t r = sr[j];
+      const uint32_t i = (uint32_t)(r & kRecIdxMask);
+      uint32_t d = 0;
+      uint64_t xi = 0;
+      bool have = false;
+#pragma unroll
+      for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
+        if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
+        const uint64_t rb = sr[j - back];
+        if ((rb >> kRecHashShift) != (r >> kRecHashShift)) break;  // left the hash's run
+        if ((rb >> kRecFpShift) == (r >> kRecFpShift)) {           // same hash and fingerprint
+          const uint32_t jj = (uint32_t)(rb & kRecIdxMask);
+          if (!have) {
+            xi = x[i];
+            have = true;
+          }
+          if (x[jj] == xi) {
+            d = i - jj;
+            break;
+          }
+        }
+      }
+      if (d) dist[i] = d;
+    }
+    __syncthreads();
+  }
+}
+
+uint64_t n_tiles_of(uint64_t n) { return (n + kTile - 1) / kTile; }
+
+}  // namespace
+
+size_t fcm_dist_workspace(uint64_t n) {
+  return 2 * round16(8 * n) + round16(4 * n_tiles_of(n) * kDigits) + 4 * kDigits + 256;
+}
+
+int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
+  (void)ws_bytes;
+  uint8_t* p = static_cast<uint8_t*>(ws);
+  uint64_t* rec_a = reinterpret_cast<uint64_t*>(p);
+  uint64_t* rec_b = reinterpret_cast<uint64_t*>(p + round16(8 * n));
+  const uint64_t T = n_tiles_of(n);
+  uint32_t* counts = reinterpret_cast<uint32_t*>(p + 2 * round16(8 * n));
+  uint32_t* tot = reinterpret_cast<uint32_t*>(p + 2 * round16(8 * n) + round16(4 * T * kDigits));
+  uint32_t* dist = reinterpret_cast<uint32_t*>(rec_a);  // pass-1 records are dead after pass 2
+  *dist_out = dist;
+  if (n == 0) return 0;
+  static const bool init = [] {
+    cudaFuncSetAttribute(sort_scatter_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScatterSmem));
+    cudaFuncSetAttribute(sort_scatter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScatterSmem));
+    return true;
+  }();
+  (void)init;
+  {
+    KTrace kt("fcm_sort_hist", st);
+    sort_hist_kernel<0><<<(unsigned)T, kSortThreads, 0, st>>>(x, n, counts);
+  }
+  {
+    KTrace kt("fcm_sort_scan", st);
+    sort_scan_kernel<<<kScanBlocks, kScanWarps * 32, 0, st>>>(counts, (uint32_t)T, tot);
+  }
+  {
+    KTrace kt("fcm_sort_scatter", st);
+    sort_scatter_kernel<0><<<(unsigned)T, kSortThreads, sizeof(ScatterSmem), st>>>(x, n, counts, tot, rec_a);
+  }
+  {
+    KTrace kt("fcm_sort_hist", st);
+    sort_hist_kernel<1><<<(unsigned)T, kSortThreads, 0, st>>>(rec_a, n, counts);
+  }
+  {
+    KTrace kt("fcm_sort_scan", st);
+    sort_scan_kernel<<<kScanBlocks, kScanWarps * 32, 0, st>>>(counts, (uint32_t)T, tot);
+  }
+  {
+    KTrace kt("fcm_sort_scatter", st);
+    sort_scatter_kernel<1><<<(unsigned)T, kSortThreads, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b);
+  }
+  cudaMemsetAsync(dist, 0, 4 * n, st);
+  {
+    KTrace kt("fcm_match", st);
+    const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
+    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist);
+  }
+  return 7;
+}
+
+}  // namespace lcf

@@ -140,6 +140,10 @@ void launch_speed_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_ch
 void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t st);
 void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st);
 void launch_write_header(const EncArgs& a, cudaStream_t st);
+// FCM distances of n words at x (lcf_fcm.cu): workspace bytes, and the launch
+// (returns the number of kernels; *dist points into ws, n u32 values).
+size_t fcm_dist_workspace(uint64_t n_words);
+int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist);
 size_t dpratio_fcm_workspace(uint64_t n_words);
 int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st);
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);

@@ -70,12 +70,12 @@ __device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
 // 0..2 use the rotated values of the previous group. Pass 1 reads the
 // records of pass 0.
 constexpr int kBatch = 8;
-template <int PASS>
+template <int PASS, int B = kBatch>
 struct RecReader {
   const uint64_t* src;
   uint64_t n, i0;
   uint32_t r1p, r2p, r3p;  // previous group's rotated product words (pass 0)
-  uint64_t v[kBatch];
+  uint64_t v[B];
   __device__ __forceinline__ RecReader(const uint64_t* s, uint64_t n_, uint64_t start, uint32_t lane)
       : src(s), n(n_), i0(start) {
     if (PASS == 0) {  // the group before `start`: only its lanes 29..31 matter
@@ -92,7 +92,7 @@ struct RecReader {
   }
   __device__ __forceinline__ void load(uint32_t lane) {
 #pragma unroll
-    for (int k = 0; k < kBatch; ++k) {
+    for (int k = 0; k < B; ++k) {
       const uint64_t i = i0 + 32 * k + lane;
       v[k] = i < n ? src[i] : 0;
     }
@@ -110,7 +110,7 @@ struct RecReader {
     r3p = r3;
     return make_rec(v[k], a1 ^ a2 ^ a3, i);
   }
-  __device__ __forceinline__ void advance() { i0 += 32 * kBatch; }
+  __device__ __forceinline__ void advance() { i0 += 32 * B; }
 };
 
 template <int PASS>
@@ -169,20 +169,36 @@ __global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __
 //      the record at its sorted place in the round's shared stage
 //   4. copy the stage out: record j of digit d goes to run[d] + j − start[d],
 //      so consecutive threads write consecutive positions of a digit run
-constexpr int kRound = kSortWarps * 32 * kBatch;  // 4096 records
+#ifndef LCF_SCAT_WARPS
+#define LCF_SCAT_WARPS 16
+#endif
+#ifndef LCF_SCAT_BATCH
+#define LCF_SCAT_BATCH 8
+#endif
+#ifndef LCF_SCAT_MINB
+#define LCF_SCAT_MINB 2
+#endif
+#ifndef LCF_SCAT_PREFETCH
+#define LCF_SCAT_PREFETCH 1
+#endif
+constexpr int kSW = LCF_SCAT_WARPS, kST = kSW * 32, kSB = LCF_SCAT_BATCH;
+constexpr int kRound = kST * kSB;  // records per round
+constexpr int kP = kDigits / 2 / kST;  // digit pairs per thread
+static_assert(kP * 2 * kST == kDigits, "digit pairs divide over the threads");
 constexpr int kRounds = kTile / kRound;
 static_assert(kRounds * kRound == kTile, "tile = whole rounds");
 struct ScatterSmem {
   uint64_t stage[kRound];
-  uint32_t wcnt[kSortWarps][kDigits / 2];  // packed u16 pair per word
+  uint32_t wcnt[kSW][kDigits / 2];  // packed u16 pair per word
   uint32_t run[kDigits];                   // next output position of each digit (tile-wide)
   uint32_t rstart[kDigits];                // round: first stage slot of each digit
   uint32_t rtot[kDigits / 2];              // round: packed digit totals
-  uint32_t wsum[kSortWarps];
+  uint32_t wsum[kSW];
+  uint8_t tag[kSW][kDigits];        // per warp: last lane that claimed a digit
 };
 
 template <int PASS>
-__global__ void __launch_bounds__(kSortThreads) sort_scatter_kernel(const uint64_t* __restrict__ src, uint64_t n,
+__global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const uint64_t* __restrict__ src, uint64_t n,
                                                                     const uint32_t* __restrict__ offs,
                                                                     const uint32_t* __restrict__ tot,
                                                                     uint64_t* __restrict__ dst) {
@@ -190,9 +206,14 @@ __global__ void __launch_bounds__(kSortThreads) sort_scatter_kernel(const uint64
   ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
   const uint32_t tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const uint32_t lt = (1u << lane) - 1u;
-  // block exclusive scan of (a, b) pairs, one pair per thread → (ex_a, ex_a + a)
-  auto pair_scan = [&](uint32_t a, uint32_t b) -> uint32_t {
-    uint32_t x = a + b;
+  // Thread tid owns the kP digit pairs [kP·tid, kP·tid + kP), i.e. digits
+  // [2kP·tid, 2kP·tid + 2kP). Block exclusive scan of per-digit values c[]
+  // (in this thread's digit order) → ex[] (contains a __syncthreads).
+  auto digit_scan = [&](const uint32_t (&c)[2 * kP], uint32_t (&ex)[2 * kP]) {
+    uint32_t own = 0;
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) own += c[j];
+    uint32_t x = own;
 #pragma unroll
     for (int k = 1; k < 32; k <<= 1) {
       const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, k);
@@ -200,59 +221,82 @@ __global__ void __launch_bounds__(kSortThreads) sort_scatter_kernel(const uint64
     }
     if (lane == 31) S.wsum[warp] = x;
     __syncthreads();
-    uint32_t base = 0;
+    uint32_t base = x - own;
     for (uint32_t w = 0; w < warp; ++w) base += S.wsum[w];
-    return base + x - a - b;
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) {
+      ex[j] = base;
+      base += c[j];
+    }
   };
   {  // digit bases (exclusive scan of tot) + this tile's offsets
-    const uint32_t a = tot[2 * tid], b = tot[2 * tid + 1];
-    const uint32_t ex = pair_scan(a, b);
+    uint32_t c[2 * kP], ex[2 * kP];
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) c[j] = tot[2 * kP * tid + j];
+    digit_scan(c, ex);
     const uint32_t* o = offs + (uint64_t)blockIdx.x * kDigits;
-    S.run[2 * tid] = ex + o[2 * tid];
-    S.run[2 * tid + 1] = ex + a + o[2 * tid + 1];
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) S.run[2 * kP * tid + j] = ex[j] + o[2 * kP * tid + j];
   }
   const uint64_t tile0 = (uint64_t)blockIdx.x * kTile;
+  // the next round's loads are issued before this round's copy-out (step 4)
+  RecReader<PASS, kSB> rd(src, n, tile0 + warp * 32 * kSB, lane);
+  rd.load(lane);
   for (int r = 0; r < kRounds; ++r) {
     const uint64_t r0 = tile0 + (uint64_t)r * kRound;
     if (r0 >= n) break;  // block-uniform
     const uint32_t nr = (uint32_t)umin64(kRound, n - r0);
-    // 1. records of this warp's 256 and its digit counts
-    RecReader<PASS> rd(src, n, r0 + warp * 32 * kBatch, lane);
-    rd.load(lane);
+    if (!LCF_SCAT_PREFETCH && r > 0) {
+      rd = RecReader<PASS, kSB>(src, n, r0 + warp * 32 * kSB, lane);
+      rd.load(lane);
+    }
+    // 1. this warp's records of the round and its digit counts
 #pragma unroll
     for (int j = lane; j < kDigits / 2; j += 32) S.wcnt[warp][j] = 0;
     __syncwarp();
-    uint64_t rec[kBatch];
-    uint32_t dg[kBatch];
-    bool ok[kBatch];
+    uint64_t rec[kSB];
+    uint32_t dg[kSB];
+    bool ok[kSB];
 #pragma unroll
-    for (int k = 0; k < kBatch; ++k) {
+    for (int k = 0; k < kSB; ++k) {
       rec[k] = rd.rec(k, lane, ok[k]);
       dg[k] = ok[k] ? rec_digit(rec[k], PASS) : 0u;
       if (ok[k]) atomicAdd(&S.wcnt[warp][dg[k] >> 1], 1u << (16 * (dg[k] & 1)));
     }
     __syncthreads();
-    // 2. digits 2·tid, 2·tid+1: prefix over the warps (packed: sums ≤ 4096 per half)
-    uint32_t tw = 0;
-#pragma unroll
-    for (int w = 0; w < kSortWarps; ++w) {
-      const uint32_t c = S.wcnt[w][tid];
-      S.wcnt[w][tid] = tw;
-      tw += c;
-    }
-    S.rtot[tid] = tw;
+    // 2. this thread's digit pairs: prefix over the warps (packed: sums ≤ kRound per half)
     {
-      const uint32_t a = tw & 0xFFFFu, b = tw >> 16;
-      const uint32_t ex = pair_scan(a, b);  // (contains the barrier that publishes wcnt)
-      S.rstart[2 * tid] = ex;
-      S.rstart[2 * tid + 1] = ex + a;
+      uint32_t c[2 * kP], ex[2 * kP];
+#pragma unroll
+      for (int q = 0; q < kP; ++q) {
+        const uint32_t pq = kP * tid + q;
+        uint32_t tw = 0;
+#pragma unroll
+        for (int w = 0; w < kSW; ++w) {
+          const uint32_t v = S.wcnt[w][pq];
+          S.wcnt[w][pq] = tw;
+          tw += v;
+        }
+        S.rtot[pq] = tw;
+        c[2 * q] = tw & 0xFFFFu;
+        c[2 * q + 1] = tw >> 16;
+      }
+      digit_scan(c, ex);  // (its barrier also publishes wcnt)
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) S.rstart[2 * kP * tid + j] = ex[j];
     }
     __syncthreads();
     // 3. ranks → stage
 #pragma unroll
-    for (int k = 0; k < kBatch; ++k) {
+    for (int k = 0; k < kSB; ++k) {
       const uint32_t d = dg[k];
-      const uint32_t peers = digit_peers(d, ok[k]);
+      // equal digits inside the group are detected through a tag per digit
+      // (one of the lanes that share a digit wins the byte store, the others
+      // read another lane id back); only then are the peers matched exactly
+      if (ok[k]) S.tag[warp][d] = (uint8_t)lane;
+      __syncwarp();
+      const bool clash = __any_sync(0xFFFFFFFFu, ok[k] && S.tag[warp][d] != lane);
+      const uint32_t peers = clash ? digit_peers(d, ok[k]) : (1u << lane);
       uint32_t* wc = &S.wcnt[warp][d >> 1];
       const uint32_t sh = 16 * (d & 1);
       const uint32_t rbase = ok[k] ? (*wc >> sh) & 0xFFFFu : 0u;
@@ -263,18 +307,23 @@ __global__ void __launch_bounds__(kSortThreads) sort_scatter_kernel(const uint64
       }
       __syncwarp();
     }
+    if (LCF_SCAT_PREFETCH && r + 1 < kRounds) {
+      rd = RecReader<PASS, kSB>(src, n, r0 + kRound + warp * 32 * kSB, lane);
+      rd.load(lane);
+    }
     __syncthreads();
     // 4. stage → dst, digit runs contiguous
-    for (uint32_t j = tid; j < nr; j += kSortThreads) {
+    for (uint32_t j = tid; j < nr; j += kST) {
       const uint64_t v = S.stage[j];
       const uint32_t d = rec_digit(v, PASS);
       dst[S.run[d] + (j - S.rstart[d])] = v;
     }
     __syncthreads();
-    {
-      const uint32_t t2 = S.rtot[tid];
-      S.run[2 * tid] += t2 & 0xFFFFu;
-      S.run[2 * tid + 1] += t2 >> 16;
+#pragma unroll
+    for (int q = 0; q < kP; ++q) {
+      const uint32_t pq = kP * tid + q, t2 = S.rtot[pq];
+      S.run[2 * pq] += t2 & 0xFFFFu;
+      S.run[2 * pq + 1] += t2 >> 16;
     }
     // (the next round's first barrier orders these updates before step 4)
   }
@@ -360,7 +409,7 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   }
   {
     KTrace kt("fcm_sort_scatter", st);
-    sort_scatter_kernel<0><<<(unsigned)T, kSortThreads, sizeof(ScatterSmem), st>>>(x, n, counts, tot, rec_a);
+    sort_scatter_kernel<0><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(x, n, counts, tot, rec_a);
   }
   {
     KTrace kt("fcm_sort_hist", st);
@@ -372,7 +421,7 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   }
   {
     KTrace kt("fcm_sort_scatter", st);
-    sort_scatter_kernel<1><<<(unsigned)T, kSortThreads, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b);
+    sort_scatter_kernel<1><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b);
   }
   cudaMemsetAsync(dist, 0, 4 * n, st);
   {

@@ -329,34 +329,58 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
   }
 }
 
-// One thread per sorted position k: the nearest of the records k−1 … k−4 with
-// the same hash and an equal word is the match (L174, A-14, A-15). Records of
-// one hash are contiguous, so the walk stops at the first other hash. The
-// distance array is pre-zeroed; only matches are scattered.
+// Thread t covers the kMatchItems sorted positions k = 8t … 8t+7; for each,
+// the nearest of the records k−1 … k−4 with the same hash and an equal word is
+// the match (L174, A-14, A-15). Records of one hash are contiguous, so the walk
+// stops at the first other hash. The 12 records a thread needs come from six
+// 16-byte loads (no shared memory, no barriers). The distance array is
+// pre-zeroed; only matches are scattered.
+constexpr int kMatchItems = 8;
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint64_t* __restrict__ rec,
                                                                 uint32_t* __restrict__ dist) {
-  __shared__ uint64_t sr[kMatchBlock + 4];
-  for (uint64_t b0 = blockIdx.x * (uint64_t)kMatchBlock; b0 < n; b0 += (uint64_t)gridDim.x * kMatchBlock) {
-    for (int j = threadIdx.x; j < kMatchBlock + 4; j += kMatchBlock) {  // sorted window [b0 − 4, b0 + 256)
-      const int64_t k = (int64_t)b0 - 4 + j;
-      sr[j] = (k >= 0 && (uint64_t)k < n) ? rec[k] : 0;  // padding is never read as a predecessor
+  const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
+  for (uint64_t g = blockIdx.x * (uint64_t)kMatchBlock + threadIdx.x; g < groups;
+       g += (uint64_t)gridDim.x * kMatchBlock) {
+    const uint64_t k0 = g * kMatchItems;
+    uint64_t r[4 + kMatchItems];  // records k0−4 … k0+7 (0 outside [0, n): never read as predecessors)
+    if (k0 + kMatchItems <= n) {
+      const ulonglong2* p = reinterpret_cast<const ulonglong2*>(rec + k0);
+#pragma unroll
+      for (int q = 0; q < kMatchItems / 2; ++q) {
+        const ulonglong2 v = p[q];
+        r[4 + 2 * q] = v.x;
+        r[5 + 2 * q] = v.y;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < kMatchItems; ++j) r[4 + j] = k0 + j < n ? rec[k0 + j] : 0;
     }
-    __syncthreads();
-    const uint64_t k = b0 + threadIdx.x;
-    if (k < n) {
-      const int j = threadIdx.x + 4;
-      const uint64_t r = sr[j];
-      const uint32_t i = (uint32_t)(r & kRecIdxMask);
+    if (k0 >= 4) {
+      const ulonglong2* p = reinterpret_cast<const ulonglong2*>(rec + k0 - 4);
+      const ulonglong2 v0 = p[0], v1 = p[1];
+      r[0] = v0.x;
+      r[1] = v0.y;
+      r[2] = v1.x;
+      r[3] = v1.y;
+    } else {
+      r[0] = r[1] = r[2] = r[3] = 0;
+    }
+#pragma unroll
+    for (int j = 0; j < kMatchItems; ++j) {
+      const uint64_t k = k0 + j;
+      if (k >= n) break;
+      const uint64_t rk = r[4 + j];
+      const uint32_t i = (uint32_t)(rk & kRecIdxMask);
       uint32_t d = 0;
       uint64_t xi = 0;
       bool have = false;
 #pragma unroll
       for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
         if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
-        const uint64_t rb = sr[j - back];
-        if ((rb >> kRecHashShift) != (r >> kRecHashShift)) break;  // left the hash's run
-        if ((rb >> kRecFpShift) == (r >> kRecFpShift)) {           // same hash and fingerprint
+        const uint64_t rb = r[4 + j - back];
+        if ((rb >> kRecHashShift) != (rk >> kRecHashShift)) break;  // left the hash's run
+        if ((rb >> kRecFpShift) == (rk >> kRecFpShift)) {           // same hash and fingerprint
           const uint32_t jj = (uint32_t)(rb & kRecIdxMask);
           if (!have) {
             xi = x[i];
@@ -370,7 +394,6 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
       }
       if (d) dist[i] = d;
     }
-    __syncthreads();
   }
 }
 
@@ -426,7 +449,8 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   cudaMemsetAsync(dist, 0, 4 * n, st);
   {
     KTrace kt("fcm_match", st);
-    const int mblocks = (int)umin64((n + kMatchBlock - 1) / kMatchBlock, 148 * 8);
+    const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
+    const int mblocks = (int)umin64((groups + kMatchBlock - 1) / kMatchBlock, 148 * 16);
     fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist);
   }
   return 7;

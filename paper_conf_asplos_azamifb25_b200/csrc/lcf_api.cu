@@ -216,7 +216,7 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
   if (in_bytes % wb || !d_out || !aligned16(d_out) || (in_bytes && (!d_in || !aligned16(d_in))))
     return LCF_ERROR_INVALID_ARGUMENT;
   if (out_capacity < lcf_max_compressed_size(algo, dtype, in_bytes)) return LCF_ERROR_BUFFER_TOO_SMALL;
-  if (algo == LCF_DPRATIO && in_bytes / 8 >= (1ull << 31)) return LCF_ERROR_INVALID_ARGUMENT;  // CUB sort index
+  if (algo == LCF_DPRATIO && in_bytes / 8 >= (1ull << 31)) return LCF_ERROR_INVALID_ARGUMENT;  // 32-bit FCM record index
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;

@@ -418,6 +418,10 @@ __device__ __forceinline__ void d_enc_loader(DEncSmem& S, const EncArgs& a, cons
       return;
     }
     const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
+    if (lane == 0) {
+      trace_stamp(a, 2 * t, 0);
+      trace_stamp(a, 2 * t + 1, 0);
+    }
     const uint64_t* xs = reinterpret_cast<const uint64_t*>(a.in) + t * kTileWords;
     const uint32_t* ds = a.fcm_dist + t * kTileWords;
     if ((m & 3) == 0) {
@@ -452,6 +456,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
     const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
     for (uint32_t part = 0; part < 2; ++part, ++oit) {  // chunk 2t: V, chunk 2t+1: Dist (A-16)
       const uint64_t c = 2 * t + part;
+      if (tid == 0) trace_stamp(a, c, 1);
       // FCM outputs (L170–185) and DIFFMS₆₄ (L187) into w[]
       uint64_t nzacc = 0;
       for (uint32_t i = tid; i < m; i += kDT) {
@@ -492,9 +497,13 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       const uint32_t raw_len = 8 * m;
       const bool raw = l2 >= raw_len;  // L104, ties → raw
       const uint32_t len = raw ? raw_len : l2;
-      if (tid == 0) lookback_publish(ctx, c, round16(len));
+      if (tid == 0) {
+        lookback_publish(ctx, c, round16(len));
+        trace_stamp(a, c, 2);
+      }
       const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
       mbar_wait(&S.empty_out[o], pho ^ 1);
+      if (tid == 0) trace_stamp(a, c, 3);
       uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       if (raw) {  // the V / Dist words themselves
         uint64_t* ow = reinterpret_cast<uint64_t*>(ob);
@@ -530,6 +539,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       }
       fence_proxy_async_smem();
       bar_d();
+      if (tid == 0) trace_stamp(a, c, 4);
       if (lane == 0) mbar_arrive(&S.full_out[o]);
     }
   }

@@ -39,8 +39,12 @@ t0 = t[:, 0].min()
 t = (t - t0) / 1e3  # µs since the first ticket
 names = ["ticket", "data", "published", "slot", "packed", "storer", "lookback", "stored"]
 print(f"{a.codec} {a.config}/{a.field}: {C} chunks, span {t[:, 7].max():.1f} us (first ticket → last store read)")
-for k in range(1, 8):
-    d = t[:, k] - t[:, k - 1]
-    print(f"  {names[k - 1]:>9s} → {names[k]:<9s}: median {np.median(d):7.2f} us  p90 {np.percentile(d, 90):7.2f}  max {d.max():7.2f}")
+groups = [("all", t)] if a.codec != "DPratio" else [("V chunks", t[0::2]), ("Dist chunks", t[1::2])]
+for label, tg in groups:
+    if len(groups) > 1:
+        print(f" {label}:")
+    for k in range(1, 8):
+        d = tg[:, k] - tg[:, k - 1]
+        print(f"  {names[k - 1]:>9s} → {names[k]:<9s}: median {np.median(d):7.2f} us  p90 {np.percentile(d, 90):7.2f}  max {d.max():7.2f}")
 for q in (0, 0.1, 0.5, 0.9, 1.0):
     print(f"  ticket time quantile {q:.1f}: {np.quantile(t[:, 0], q):7.2f} us; stored: {np.quantile(t[:, 7], q):7.2f} us")

@@ -53,6 +53,8 @@ struct AdaptScratch {
   uint32_t b1[64];      // B1 bitmap words (n ≤ 2048 bits)
   uint32_t c1m[32], off1[32], b2[32];  // encoder plan → emit: warp 0's B2 bits, nr(B1) offsets
   uint32_t k, flag, s1, s2, nr1, b3;
+  uint32_t wtot[kDW];                   // encoder: set words per warp
+  uint16_t rank0[kDT];                  // encoder: set words before thread t's 8 words
 };
 
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
@@ -68,26 +70,82 @@ __device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, 
   return w >= 64 ? v : v & ((1ull << w) - 1);
 }
 
-// Encode L bytes at src (8-byte aligned) with RAZE (rare = false, L189) or RARE
-// (rare = true, L195) into dst (16-byte aligned, ≥ L + 3 + 32 bytes). All kDT
-// compute threads call it; returns the output length (FORMAT.md §6.2–6.3).
-// Word i = tid + 256·r (r = 0..7); the rounds are not unrolled and re-read the
-// words from shared memory, which keeps the code small (I-cache) and the
-// register count low (occupancy).
+// Words 8·tid … 8·tid+7 of sv with 16-byte shared loads; quad q of thread t is
+// read in slot q ^ ((t >> 1) & 3), which spreads the eight threads of a
+// wavefront over distinct banks. Words at or past n are returned as 0. sv must
+// be 16-byte aligned with readable slack up to word 8·kDT.
+__device__ __forceinline__ void load8(const uint64_t* sv, uint32_t n, uint32_t tid, uint64_t (&v)[8]) {
+  const uint32_t s = (tid >> 1) & 3;
+  ulonglong2 ld[4];
+#pragma unroll
+  for (uint32_t q = 0; q < 4; ++q) ld[q] = reinterpret_cast<const ulonglong2*>(sv)[4 * tid + (q ^ s)];
+#pragma unroll
+  for (uint32_t q = 0; q < 4; ++q) {
+    const ulonglong2 x = s == 0 ? ld[q] : s == 1 ? ld[q ^ 1] : s == 2 ? ld[q ^ 2] : ld[q ^ 3];
+    v[2 * q] = 8 * tid + 2 * q < n ? x.x : 0ull;
+    v[2 * q + 1] = 8 * tid + 2 * q + 1 < n ? x.y : 0ull;
+  }
+}
+
+// LSB-first bit writer for one thread's contiguous run of fields in a u32
+// buffer. The run's first and last words may be shared with the neighbouring
+// runs (atomicOr into a zeroed buffer); the words in between belong to this
+// thread alone (plain stores).
+struct BitWriter {
+  uint32_t* buf;
+  uint32_t widx, nb;  // current word, pending bits in acc (< 32 between puts)
+  uint64_t acc;
+  bool first;
+  __device__ __forceinline__ BitWriter(uint32_t* b, uint64_t off)
+      : buf(b), widx((uint32_t)(off >> 5)), nb((uint32_t)(off & 31)), acc(0), first(true) {}
+  __device__ __forceinline__ void emit(uint32_t w) {
+    if (first) atomicOr(buf + widx, w);
+    else buf[widx] = w;
+    first = false;
+    ++widx;
+  }
+  // append the low w bits of f (f < 2^w, 1 ≤ w ≤ 64)
+  __device__ __forceinline__ void put(uint64_t f, uint32_t w) {
+    const uint64_t carry = nb ? f >> (64 - nb) : 0ull;  // bits beyond the 64-bit accumulator
+    acc |= f << nb;
+    nb += w;
+    if (nb >= 32) {
+      emit((uint32_t)acc);
+      acc = (acc >> 32) | (carry << 32);
+      nb -= 32;
+      if (nb >= 32) {
+        emit((uint32_t)acc);
+        acc >>= 32;
+        nb -= 32;
+      }
+    }
+  }
+  __device__ __forceinline__ void finish() {
+    if (nb) atomicOr(buf + widx, (uint32_t)acc);
+  }
+};
+
+// Encode L bytes at src (16-byte aligned, zero-safe slack to 16 KiB) with RAZE
+// (rare = false, L189) or RARE (rare = true, L195) into dst (16-byte aligned,
+// ≥ L + 3 + 32 bytes). All kDT compute threads call it; returns the output
+// length (FORMAT.md §6.2–6.3). Thread t owns words 8t … 8t+7 (n ≤ 2048): its
+// B1 bits are B1 byte t, and its HI and LO fields are contiguous bit runs.
 __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, bool rare, AdaptScratch& sc,
                                                uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint32_t n = L / 8, tl = L % 8;
   const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
-  const uint32_t R = (n + kDT - 1) / kDT;  // rounds holding words
   if (tid < 65) sc.hist[tid] = 0;
+  uint64_t v[8];
+  load8(sv, n, tid, v);
+  const uint32_t i0 = 8 * tid;
+  const uint64_t p = (rare && i0 >= 1 && i0 - 1 < n) ? sv[i0 - 1] : 0ull;  // RARE reference of word i0
   bar_d();
   // ---- histogram of clz(v_i ⊕ ref_i), warp-aggregated shared atomics ----
-#pragma unroll 1
-  for (uint32_t r = 0; r < R; ++r) {
-    const uint32_t i = tid + kDT * r;
-    uint32_t z = 65u;
-    if (i < n) z = clz64(sv[i] ^ ((rare && i) ? sv[i - 1] : 0ull));
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint64_t ref = rare ? (j ? v[j - 1] : p) : 0ull;
+    const uint32_t z = i0 + j < n ? clz64(v[j] ^ ref) : 65u;
     const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
     if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
   }
@@ -111,36 +169,36 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   bar_d();
   const uint32_t k = sc.k;
   const uint32_t sh = 64 - k;  // top(v) = v >> sh (k = 64: sh = 0)
-  // ---- B1 (warp ballots are the B1 words) and per-(round, warp) counts ----
-#pragma unroll 1
-  for (uint32_t r = 0; r < 8; ++r) {
-    const uint32_t i = tid + kDT * r;
-    bool set = false;
-    if (i < n) {
-      const uint64_t ref = (rare && i) ? sv[i - 1] : 0ull;
-      set = (sv[i] >> sh) != (ref >> sh);
-    }
-    const uint32_t bal = __ballot_sync(0xFFFFFFFFu, set);
-    if (lane == 0) {
-      sc.b1[r * kDW + warp] = bal;
-      sc.cnt[r * kDW + warp] = __popc(bal);
-    }
+  // ---- B1 byte t = this thread's set bits; ranks of the set words ----
+  uint32_t byte = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint64_t ref = rare ? (j ? v[j - 1] : p) : 0ull;
+    if (i0 + j < n && (v[j] >> sh) != (ref >> sh)) byte |= 1u << j;
   }
+  reinterpret_cast<uint8_t*>(sc.b1)[tid] = (uint8_t)byte;
+  const uint32_t c = __popc(byte);
+  uint32_t x = c;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+    if ((int)lane >= d) x += y;
+  }
+  if (lane == 31) sc.wtot[warp] = x;
   bar_d();
+  {
+    uint32_t base = 0;
+#pragma unroll
+    for (uint32_t w = 0; w < kDW; ++w)
+      if (w < warp) base += sc.wtot[w];
+    sc.rank0[tid] = (uint16_t)(base + x - c);
+  }
   uint32_t nr1 = 0, b2 = 0, b3 = 0, c1m = 0, off1 = 0, b1w0 = 0, b1w1 = 0;
   const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
   if (warp == 0) {
-    // prefix of the 64 per-(round, warp) counts
-    const uint32_t a0 = sc.cnt[2 * lane], a1 = sc.cnt[2 * lane + 1];
-    uint32_t s = a0 + a1;
+    uint32_t nset = 0;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, d);
-      if ((int)lane >= d) s += y;
-    }
-    sc.cnt[2 * lane] = s - a0 - a1;
-    sc.cnt[2 * lane + 1] = s - a1;
-    const uint32_t nset = __shfl_sync(0xFFFFFFFFu, s, 31);
+    for (uint32_t w = 0; w < kDW; ++w) nset += sc.wtot[w];
     // B1 → B2 (lane: B1 bytes [8·lane, 8·lane+8) = words 2·lane, 2·lane+1)
     b1w0 = sc.b1[2 * lane];
     b1w1 = sc.b1[2 * lane + 1];
@@ -152,14 +210,14 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
       if (cur != pre && 8 * lane + j < L1) c1m |= 1u << j;
     }
     b2 = c1m;  // B2 byte `lane`
-    uint32_t x = __popc(c1m);
+    uint32_t y = __popc(c1m);
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
-      if ((int)lane >= d) x += y;
+      const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, y, d);
+      if ((int)lane >= d) y += o;
     }
-    off1 = x - __popc(c1m);
-    nr1 = __shfl_sync(0xFFFFFFFFu, x, 31);
+    off1 = y - __popc(c1m);
+    nr1 = __shfl_sync(0xFFFFFFFFu, y, 31);
     const uint32_t pb2 = __shfl_up_sync(0xFFFFFFFFu, b2, 1);
     b3 = __ballot_sync(0xFFFFFFFFu, lane < L2 && b2 != (lane ? pb2 : 0u));
     const uint32_t nr2 = __popc(b3);
@@ -191,6 +249,7 @@ __device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8
   const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
   (void)L1;
   (void)L2;
+  (void)rare;
   const bool bypass = sc.flag;
   const uint32_t total = sc.s1, hib = sc.s2, nr1 = sc.nr1, b3 = sc.b3;
   if (bypass) {  // dst[3 + j] = src[j], one funnel shift per output word
@@ -210,26 +269,29 @@ __device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8
   }
   uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
   for (uint32_t j = tid; j < (total + 7) / 4 + 1; j += kDT) dw[j] = 0;
+  uint64_t v[8];
+  load8(sv, n, tid, v);
+  const uint32_t i0 = 8 * tid;
+  const uint32_t byte = reinterpret_cast<const uint8_t*>(sc.b1)[tid];
+  const uint32_t rank0 = sc.rank0[tid];
   bar_d();
   // ---- HI: top fields of the set words (rank order), LO: low fields of all words ----
   const uint64_t hi_base = 24, lo_base = 8ull * (3 + hib);
   const uint32_t wl = 64 - k;
   const uint64_t lmask = wl >= 64 ? ~0ull : ((1ull << wl) - 1);
-  const uint32_t R = (n + kDT - 1) / kDT;  // later rounds hold no words
-#pragma unroll 1
-  for (uint32_t r = 0; r < R; ++r) {
-    const uint32_t i = tid + kDT * r;
-    const uint32_t q = r * kDW + warp;
-    const uint32_t bal = sc.b1[q];
-    const uint64_t v = i < n ? sv[i] : 0ull;
-    if (bal) {  // a warp without set words has nothing to emit
-      const bool set = (bal >> lane) & 1;
-      const uint32_t rank = sc.cnt[q] + __popc(bal & ((1u << lane) - 1));
-      emit_bits_warp(dw, hi_base + (uint64_t)rank * k, set ? k : 0, set ? (v >> sh) : 0, 0, true);
-    }
-    if (wl)
-      emit_bits_warp(dw, lo_base + (uint64_t)i * wl, i < n ? wl : 0, v & lmask, 0, true,
-                     wl >= 32 && kDT * r + 32 * warp + 31 < n);
+  if (byte) {
+    BitWriter bw(dw, hi_base + (uint64_t)rank0 * k);
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if ((byte >> j) & 1) bw.put(v[j] >> sh, k);
+    bw.finish();
+  }
+  if (wl && i0 < n) {
+    BitWriter bw(dw, lo_base + (uint64_t)i0 * wl);
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (i0 + j < n) bw.put(v[j] & lmask, wl);
+    bw.finish();
   }
   bar_d();
   // ---- header, tail bytes, nr(B1), nr(B2), B3 ----

@@ -47,6 +47,11 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
 }
 
 // ============================ RAZE / RARE in shared memory ============================
+// clz histogram: plain shared atomics (1, measured fastest: the hardware
+// serialises equal bins within a warp cheaply) or match-aggregated ones (0)
+#ifndef LCF_HIST_MODE
+#define LCF_HIST_MODE 1
+#endif
 struct AdaptScratch {
   uint32_t hist[65];
   uint32_t cnt[64];     // per (round, warp) set counts → exclusive prefix
@@ -141,13 +146,17 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   const uint32_t i0 = 8 * tid;
   const uint64_t p = (rare && i0 >= 1 && i0 - 1 < n) ? sv[i0 - 1] : 0ull;  // RARE reference of word i0
   bar_d();
-  // ---- histogram of clz(v_i ⊕ ref_i), warp-aggregated shared atomics ----
+  // ---- histogram of clz(v_i ⊕ ref_i) ----
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
     const uint64_t ref = rare ? (j ? v[j - 1] : p) : 0ull;
     const uint32_t z = i0 + j < n ? clz64(v[j] ^ ref) : 65u;
-    const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
-    if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
+    if (LCF_HIST_MODE == 0) {
+      const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
+      if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
+    } else {
+      if (z <= 64) atomicAdd(&sc.hist[z], 1u);
+    }
   }
   bar_d();
   // ---- k* = smallest argmin of est(k) = k·nz(k) + (64−k)·n, k ∈ 1..64 (A-17, A-18) ----

@@ -16,6 +16,7 @@ namespace {
 
 std::atomic<uint64_t> g_launches{0};
 unsigned long long* g_trace_buf = nullptr;  // lcf__trace_compress only
+unsigned long long* g_trace_dec = nullptr;  // lcf__trace_decompress only
 
 struct Workspace {
   int device = -1;
@@ -207,6 +208,17 @@ lcf_status_t lcf__trace_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void*
   return st;
 }
 
+// Diagnostic twin of lcf_decompress (not in lcf.h): DPratio decode kernels
+// record 8 globaltimer stamps per tile into d_trace (n_tiles × 8 u64).
+lcf_status_t lcf__trace_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes,
+                                   void* d_out, size_t out_capacity, unsigned long long* d_trace, void* stream) {
+  g_trace_dec = d_trace;
+  size_t n = 0;
+  lcf_status_t st = lcf_decompress(algo, dtype, d_in, in_bytes, d_out, out_capacity, &n, stream);
+  g_trace_dec = nullptr;
+  return st;
+}
+
 lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
                           size_t out_capacity, size_t* out_bytes, void* stream_) {
   cudaStream_t stream = (cudaStream_t)stream_;
@@ -288,6 +300,7 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
   if (algo == LCF_DPRATIO)
     if (lcf_status_t s = grow(ws->tile_flag, ws->tile_cap, grid / 2 + 1, stream, true)) return s;
   DecArgs a{};
+  a.trace = g_trace_dec;
   a.stream = static_cast<const uint8_t*>(d_in);
   a.stream_bytes = in_bytes;
   a.out = static_cast<uint8_t*>(d_out);

@@ -638,7 +638,7 @@ __global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a,
 // =================================== decode ======================================
 struct DDecSmem {
   alignas(128) uint8_t in[2][kChunkBytes + 128];  // stage: V and Dist payloads of a tile
-  alignas(128) uint8_t rz[kChunkBytes + 128];     // RARE⁻¹ output (RAZE stream)
+  alignas(128) uint8_t rz[2][kChunkBytes + 128];  // RARE⁻¹ outputs (RAZE streams) of V and Dist
   alignas(128) uint64_t V[kTileWords + 8];        // V, then the decoded tile in place
   alignas(128) uint64_t D[kTileWords + 8];
   int32_t pj[2][kDT];                             // pointer jumping: target (−1 done)
@@ -702,8 +702,10 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
       const uint32_t r0 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j), r1 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j + 1);
       const bool b0 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j), b1 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j + 1);
       const uint64_t e0 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j), e1 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j + 1);
+      if (lane == 0) trace_stamp(a, tb + j, 0);
       mbar_wait(&S.empty_in[0], (it & 1) ^ 1);
       if (lane == 0) {
+        trace_stamp(a, tb + j, 1);
         const bool bb = b0 || b1;
         if (bb) record_error(ctx, DERR_CORRUPT);
         S.tile[0] = tb + j;
@@ -723,18 +725,47 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
   }
 }
 
-// One chunk of a tile: RARE⁻¹ → RAZE⁻¹ → DIFFMS⁻¹ into arr[0..m). Returns false
-// if malformed.
-__device__ __forceinline__ bool d_decode_chunk(DDecSmem& S, const uint8_t* pay, uint32_t len, bool raw, uint32_t m,
-                                               uint64_t* arr, uint32_t tid) {
+// One chunk of a tile in two steps, so that the tile's payload stage can be
+// released between them. Step 1 reads the payload: RARE⁻¹ into rz (returns its
+// length), or a raw chunk straight into arr (returns kRawDone; *nz = any
+// non-zero word). Step 2: RAZE⁻¹ into arr and DIFFMS⁻¹ in place (*nz = any
+// non-zero result). Both return −1 / false if malformed.
+constexpr int kRawDone = -2;
+__device__ __forceinline__ int d_decode_step1(DDecSmem& S, const uint8_t* pay, uint32_t len, bool raw, uint32_t m,
+                                              uint8_t* rz, uint64_t* arr, bool& nz, uint32_t tid) {
   if (raw) {
-    for (uint32_t i = tid; i < m; i += kDT) arr[i] = reinterpret_cast<const uint64_t*>(pay)[i];
-    bar_d();
-    return true;
+    uint64_t acc = 0;
+    for (uint32_t i = tid; i < m; i += kDT) {
+      const uint64_t w = reinterpret_cast<const uint64_t*>(pay)[i];
+      arr[i] = w;
+      acc |= w;
+    }
+    nz = bar_d_or(acc != 0);
+    return kRawDone;
   }
-  const int l1 = adaptive_decode(pay, len, S.rz, kChunkBytes + 3, true, S.sc, tid);
+  return adaptive_decode(pay, len, rz, kChunkBytes + 3, true, S.sc, tid);
+}
+__device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_t* rz, uint32_t m, uint64_t* arr,
+                                               bool& nz, bool want_zeros, uint32_t tid) {
+  if (l1 == kRawDone) return true;
   if (l1 < 0) return false;
-  const int l0 = adaptive_decode(S.rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, S.sc, tid);
+  {  // the RAZE stream of an all-zero chunk: k = 64 and nothing but the B3
+     // bytes, which a valid stream then has all zero (any set B3 bit would
+     // claim nr(B2) bytes that are not there) — the encoder's fixed stream
+    const uint32_t L = rz[0] | ((uint32_t)rz[1] << 8), n = L / 8;
+    const uint32_t L3 = (((n + 7) / 8 + 7) / 8 + 7) / 8;
+    if (l1 >= 3 && rz[2] == 64 && L == 8 * m && (uint32_t)l1 == 3 + L3) {
+      bool z = true;
+      for (uint32_t j = 0; j < L3; ++j) z = z && rz[3 + j] == 0;
+      if (!z) return false;
+      if (want_zeros)
+        for (uint32_t i = tid; i < m; i += kDT) arr[i] = 0;  // DIFFMS⁻¹ of zeros
+      nz = false;
+      bar_d();
+      return true;
+    }
+  }
+  const int l0 = adaptive_decode(rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, S.sc, tid);
   if (l0 != (int)(8 * m)) return false;
   // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8), moved as 16-byte pairs
   uint64_t v[8], run = 0;
@@ -747,13 +778,16 @@ __device__ __forceinline__ bool d_decode_chunk(DDecSmem& S, const uint8_t* pay, 
   }
   uint64_t tot;
   uint64_t acc = cta_scan_u64(run, S.scan, tid, tot);
+  uint64_t any = 0;
 #pragma unroll
   for (int j = 0; j < 8; j += 2) {
     const uint64_t a0 = acc + v[j], a1 = a0 + v[j + 1];
     acc = a1;
     reinterpret_cast<ulonglong2*>(arr)[4 * tid + j / 2] = make_ulonglong2(a0, a1);  // words ≥ m: scratch
+    if (8 * tid + j < m) any |= a0;
+    if (8 * tid + j + 1 < m) any |= a1;
   }
-  bar_d();
+  nz = bar_d_or(any != 0);
   return true;
 }
 
@@ -762,21 +796,53 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
   const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / 8;
   uint64_t* out = reinterpret_cast<uint64_t*>(a.out);
+  // The decoded tile leaves S.V by a TMA bulk store issued by thread 0; its
+  // completion (and the tile's flag) is awaited only before S.V is written
+  // again, or at exit.
+  uint64_t pending = kNoChunk;
+  auto finish_pending = [&]() {
+    if (tid == 0 && pending != kNoChunk) {
+      tma_store_wait_all0();
+      __threadfence();
+      st_release_u32(a.tile_flag + pending, ctx.epoch);
+      trace_stamp(a, pending, 7);
+    }
+    pending = kNoChunk;
+  };
   for (uint32_t it = 0;; ++it) {
     mbar_wait(&S.full_in[0], it & 1);
     const uint64_t t = S.tile[0];
-    if (t == kNoChunk) return;
+    if (t == kNoChunk) {
+      finish_pending();
+      return;
+    }
     const uint32_t fl = S.flags[0];
     const uint32_t m = (uint32_t)umin64(kTileWords, n_words - t * kTileWords);
-    bool ok = !(fl & 4);
-    if (ok) ok = d_decode_chunk(S, S.in[0], S.len[0][0], fl & 1, m, S.V, tid);
-    if (ok) ok = d_decode_chunk(S, S.in[1], S.len[0][1], (fl >> 1) & 1, m, S.D, tid);
+    if (tid == 0) trace_stamp(a, t, 2);
+    bool ok = !(fl & 4), nzV = false, nzD = false;
+    int l1V = -1, l1D = -1;
+    if (fl & 1) {  // a raw V chunk is copied into S.V right away
+      finish_pending();
+      bar_d();
+    }
+    if (ok) {
+      l1V = d_decode_step1(S, S.in[0], S.len[0][0], fl & 1, m, S.rz[0], S.V, nzV, tid);
+      l1D = d_decode_step1(S, S.in[1], S.len[0][1], (fl >> 1) & 1, m, S.rz[1], S.D, nzD, tid);
+    }
+    // both payloads have been read (RARE⁻¹ outputs in rz, raw chunks in V / D):
+    // the loader may fetch the next tile while this one finishes
     __syncwarp();
     if (lane == 0) mbar_arrive(&S.empty_in[0]);
+    if (tid == 0) trace_stamp(a, t, 3);
+    finish_pending();  // (step 2 writes S.V only after its first barrier)
+    if (ok) ok = d_decode_step2(S, l1V, S.rz[0], m, S.V, nzV, true, tid);
+    if (tid == 0) trace_stamp(a, t, 4);
+    if (ok) ok = d_decode_step2(S, l1D, S.rz[1], m, S.D, nzD, false, tid);  // (D unread if all zero)
+    if (tid == 0) trace_stamp(a, t, 5);
     // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
     const uint64_t t0 = t * kTileWords;
     bool bad = !ok;
-    if (ok) {
+    if (ok && nzD) {  // (no distances: x = V as it stands)
       for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
         const uint32_t li = b + tid;
         int32_t p = -1;
@@ -819,14 +885,21 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
         bar_d();
       }
     }
+    if (tid == 0) trace_stamp(a, t, 6);
+    fence_proxy_async_smem();  // S.V (generic-proxy writes) → the bulk store
     if (bar_d_or(bad)) {
       if (tid == 0) record_error(ctx, DERR_CORRUPT);
-    } else {
+    } else if (m % 2 == 0) {
+      if (tid == 0) {
+        tma_store_1d(out + t0, S.V, 8 * m);
+        tma_store_commit();
+      }
+    } else {  // ragged last tile: thread stores
       for (uint32_t i = tid; i < m; i += kDT) __stcs(out + t0 + i, S.V[i]);
+      __threadfence();
+      bar_d();
     }
-    __threadfence();
-    bar_d();
-    if (tid == 0) st_release_u32(a.tile_flag + t, ctx.epoch);  // tile complete (also when malformed)
+    pending = t;  // tile complete (also when malformed) once thread 0 has waited
   }
 }
 

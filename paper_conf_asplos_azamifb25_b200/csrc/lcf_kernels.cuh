@@ -50,7 +50,8 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-__device__ __forceinline__ void trace_stamp(const EncArgs& a, uint64_t chunk, int k) {
+template <class Args>
+__device__ __forceinline__ void trace_stamp(const Args& a, uint64_t chunk, int k) {
   if (a.trace) a.trace[chunk * 8 + k] = gtimer();
 }
 
@@ -61,6 +62,7 @@ struct DecArgs {
   uint64_t out_capacity;
   uint32_t algo, word_bytes;
   uint32_t* tile_flag;    // DPratio: per-tile completion (epoch) flags
+  unsigned long long* trace;  // lcf__trace_decompress only: 8 globaltimer stamps per chunk / tile
 };
 
 struct DecChunk {

@@ -12,9 +12,9 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/
 # full sets on the bench's fields (CESM T for SP codecs, Miranda density for DP)
 for spec in "SPspeed cesm_1800x3600_f32 T speed_" "SPratio cesm_1800x3600_f32 T spratio_" \
             "DPspeed miranda_256x384x384_f64 density speed_" \
-            "DPratio miranda_256x384x384_f64 density fcm_|dpratio_"; do
+            "DPratio miranda_256x384x384_f64 density sort_|fcm_|dpratio_"; do
   set -- $spec
-  ncu --set full --clock-control none --import-source on -k "regex:$4" -c 6 -o $OUT/full_$1 \
+  ncu --set full --clock-control none --import-source on -k "regex:$4" -c 10 -o $OUT/full_$1 \
       python scripts/run_codec.py --codec $1 --config $2 --field $3 --reps 1 > $OUT/ncu_$1.log 2>&1
 done
 ls -la $OUT

@@ -16,6 +16,10 @@ os.makedirs("profiles", exist_ok=True)
 
 
 def short(name):
+    for k, v in (("sort_hist_kernel", "fcm_sort_hist"), ("sort_scan_kernel", "fcm_sort_scan"),
+                 ("sort_scatter_kernel", "fcm_sort_scatter")):
+        if k in name:
+            return v
     for k in ("speed_encode_kernel<unsigned int>", "speed_encode_kernel<unsigned long>",
               "speed_decode_kernel<unsigned int>", "speed_decode_kernel<unsigned long>",
               "spratio_encode_kernel", "spratio_decode_kernel", "dpratio_encode_kernel", "dpratio_decode_kernel",

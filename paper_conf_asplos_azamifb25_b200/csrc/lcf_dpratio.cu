@@ -561,6 +561,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         const uint32_t L = 8 * m, L3 = (((m + 7) / 8 + 7) / 8 + 7) / 8;
         if (tid < 3 + L3) S.rz[tid] = tid == 0 ? (uint8_t)L : tid == 1 ? (uint8_t)(L >> 8) : tid == 2 ? 64 : 0;
         l1 = 3 + L3;
+        bar_d();  // adaptive_plan reads its input before its first barrier
       }
       // RARE is planned first: the chunk's size — and its aggregate for the
       // look-back of later chunks — is known before an output slot is needed

@@ -26,3 +26,9 @@ for algo in ("SPspeed", "SPratio", "DPspeed", "DPratio"):
             pass
     print(algo, "ok")
 torch.cuda.synchronize()
+# multi-tile DPratio (several FCM sort tiles, rounds and decode tiles)
+x = datagen.field("miranda_256x384x384_f64", "density", device="cuda", shape=(2, 384, 384)).reshape(-1).view(torch.int64)
+s = lcf.compress("DPratio", x)
+assert torch.equal(lcf.decompress("DPratio", s), x)
+print("DPratio slab ok")
+torch.cuda.synchronize()

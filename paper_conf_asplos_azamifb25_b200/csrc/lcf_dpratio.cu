@@ -79,7 +79,19 @@ __device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, 
 // read in slot q ^ ((t >> 1) & 3), which spreads the eight threads of a
 // wavefront over distinct banks. Words at or past n are returned as 0. sv must
 // be 16-byte aligned with readable slack up to word 8·kDT.
+#ifndef LCF_LOAD8_SWZ
+#define LCF_LOAD8_SWZ 0
+#endif
 __device__ __forceinline__ void load8(const uint64_t* sv, uint32_t n, uint32_t tid, uint64_t (&v)[8]) {
+  if (!LCF_LOAD8_SWZ) {  // plain 16-byte loads (4-way bank conflicts per quarter warp)
+#pragma unroll
+    for (uint32_t q = 0; q < 4; ++q) {
+      const ulonglong2 x = reinterpret_cast<const ulonglong2*>(sv)[4 * tid + q];
+      v[2 * q] = 8 * tid + 2 * q < n ? x.x : 0ull;
+      v[2 * q + 1] = 8 * tid + 2 * q + 1 < n ? x.y : 0ull;
+    }
+    return;
+  }
   const uint32_t s = (tid >> 1) & 3;
   ulonglong2 ld[4];
 #pragma unroll
@@ -140,12 +152,12 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint32_t n = L / 8, tl = L % 8;
   const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
-  if (tid < 65) sc.hist[tid] = 0;
+  // (the input was completed before a barrier of the caller; sc.hist is zero:
+  // zeroed at kernel start and again by warp 0 right after reading it)
   uint64_t v[8];
   load8(sv, n, tid, v);
   const uint32_t i0 = 8 * tid;
   const uint64_t p = (rare && i0 >= 1 && i0 - 1 < n) ? sv[i0 - 1] : 0ull;  // RARE reference of word i0
-  bar_d();
   // ---- histogram of clz(v_i ⊕ ref_i) ----
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
@@ -162,6 +174,9 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   // ---- k* = smallest argmin of est(k) = k·nz(k) + (64−k)·n, k ∈ 1..64 (A-17, A-18) ----
   if (warp == 0) {
     const uint32_t c0 = sc.hist[2 * lane], c1 = sc.hist[2 * lane + 1];
+    sc.hist[2 * lane] = 0;  // ready for the next plan (its atomics follow several barriers)
+    sc.hist[2 * lane + 1] = 0;
+    if (lane == 0) sc.hist[64] = 0;
     uint32_t s = c0 + c1;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -302,24 +317,23 @@ __device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8
       if (i0 + j < n) bw.put(v[j] & lmask, wl);
     bw.finish();
   }
-  bar_d();
-  // ---- header, tail bytes, nr(B1), nr(B2), B3 ----
+  // ---- header, tail bytes, nr(B1), nr(B2), B3: byte ORs into the zeroed
+  // words, concurrent with the bit writers (whose edge words they may share) ----
+  auto put_byte = [&](uint32_t pos, uint32_t val) {
+    atomicOr(dw + (pos >> 2), (val & 0xFFu) << (8 * (pos & 3)));
+  };
   const uint32_t after = 3 + hib + (n * wl + 7) / 8;
-  if (tid == 0) {
-    dst[0] = (uint8_t)L;
-    dst[1] = (uint8_t)(L >> 8);
-    dst[2] = (uint8_t)k;
-  }
-  if (tid < tl) dst[after + tid] = src[8 * n + tid];
+  if (tid == 0) atomicOr(dw, (L & 0xFFFFu) | (k << 16));
+  if (tid < tl) put_byte(after + tid, src[8 * n + tid]);
   if (warp == 0) {
     const uint32_t c1m = sc.c1m[lane], b2 = sc.b2[lane];
     const uint32_t b1w0 = sc.b1[2 * lane], b1w1 = sc.b1[2 * lane + 1];
     uint32_t p = after + tl + sc.off1[lane];
 #pragma unroll
     for (int j = 0; j < 8; ++j)
-      if ((c1m >> j) & 1) dst[p++] = (uint8_t)((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
-    if ((b3 >> lane) & 1) dst[after + tl + nr1 + __popc(b3 & ((1u << lane) - 1))] = (uint8_t)b2;
-    if (lane < L3) dst[total - L3 + lane] = (uint8_t)(b3 >> (8 * lane));
+      if ((c1m >> j) & 1) put_byte(p++, (j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
+    if ((b3 >> lane) & 1) put_byte(after + tl + nr1 + __popc(b3 & ((1u << lane) - 1)), b2);
+    if (lane < L3) put_byte(total - L3 + lane, b3 >> (8 * lane));
   }
   bar_d();
 }
@@ -621,6 +635,7 @@ __global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a,
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (uint32_t i = threadIdx.x; i < 65; i += blockDim.x) S.sc.hist[i] = 0;  // adaptive_plan's invariant
   if (threadIdx.x == 0) {
     mbar_init(&S.full_in[0], 1);
     mbar_init(&S.empty_in[0], kDW);

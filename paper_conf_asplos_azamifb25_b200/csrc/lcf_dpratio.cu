@@ -483,6 +483,8 @@ struct DEncSmem {
   uint64_t in_chunk[1], out_chunk[kDOut];
   uint32_t out_len[kDOut], out_raw[kDOut];
   uint64_t scan[kDW];
+  alignas(16) uint8_t zc[64];  // the Dist chunk of a full tile without distances: its stream, once made
+  uint32_t zlen;               // (0 = not yet)
   AdaptScratch sc;
 };
 
@@ -539,11 +541,35 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       return;
     }
     const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
+    bool dist_zero = false;  // the tile has no FCM match (set by part 0)
     for (uint32_t part = 0; part < 2; ++part, ++oit) {  // chunk 2t: V, chunk 2t+1: Dist (A-16)
       const uint64_t c = 2 * t + part;
       if (tid == 0) trace_stamp(a, c, 1);
+      const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
+      const bool cacheable = part == 1 && dist_zero && m == kTileWords;
+      if (cacheable && S.zlen) {  // the fixed stream of an all-zero Dist chunk, made once per CTA
+        const uint32_t len = S.zlen;
+        if (tid == 0) {
+          lookback_publish(ctx, c, round16(len));
+          trace_stamp(a, c, 2);
+        }
+        mbar_wait(&S.empty_out[o], pho ^ 1);
+        if (tid < round16(len) / 4) S.out[o][tid] = reinterpret_cast<const uint32_t*>(S.zc)[tid];
+        if (tid == 0) {
+          S.out_chunk[o] = c;
+          S.out_len[o] = len;
+          S.out_raw[o] = 0;
+          trace_stamp(a, c, 3);
+        }
+        fence_proxy_async_smem();
+        bar_d();
+        if (tid == 0) trace_stamp(a, c, 4);
+        if (lane == 0) mbar_arrive(&S.full_out[o]);
+        continue;
+      }
       // FCM outputs (L170–185) and DIFFMS₆₄ (L187) into w[]
       uint64_t nzacc = 0;
+      uint32_t dor = 0;
       for (uint32_t i = tid; i < m; i += kDT) {
         uint64_t cur, prev;
         if (part == 0) {
@@ -551,6 +577,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
           cur = d ? 0ull : S.xin[i];
           prev = i ? (dp ? 0ull : S.xin[i - 1]) : 0ull;
           S.dcp[i] = d;
+          dor |= d;
         } else {
           cur = S.dcp[i];
           prev = i ? (uint64_t)S.dcp[i - 1] : 0ull;
@@ -562,6 +589,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       // RAZE then RARE (L189–201)
       uint32_t l1;
       const bool any = bar_d_or(nzacc != 0);
+      if (part == 0) dist_zero = !bar_d_or(dor != 0);
       // the tile's stage has been read (V's DIFFMS words are in w, the
       // distances in dcp): hand it back so the next tile loads during this one
       if (part == 0 && lane == 0) mbar_arrive(&S.empty_in[0]);
@@ -587,7 +615,6 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         lookback_publish(ctx, c, round16(len));
         trace_stamp(a, c, 2);
       }
-      const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
       mbar_wait(&S.empty_out[o], pho ^ 1);
       if (tid == 0) trace_stamp(a, c, 3);
       uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
@@ -617,6 +644,11 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       } else {
         adaptive_emit(S.rz, l1, ob, true, S.sc, tid);
         if (tid < 16 && len + tid < round16(len)) ob[len + tid] = 0;
+        if (cacheable && round16(len) <= sizeof(S.zc)) {  // remember it (read after later barriers)
+          bar_d();
+          if (tid < round16(len)) S.zc[tid] = ob[tid];
+          if (tid == 0) S.zlen = len;
+        }
       }
       if (tid == 0) {
         S.out_chunk[o] = c;
@@ -636,6 +668,7 @@ __global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a,
   DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   for (uint32_t i = threadIdx.x; i < 65; i += blockDim.x) S.sc.hist[i] = 0;  // adaptive_plan's invariant
+  if (threadIdx.x == 0) S.zlen = 0;
   if (threadIdx.x == 0) {
     mbar_init(&S.full_in[0], 1);
     mbar_init(&S.empty_in[0], kDW);

@@ -137,6 +137,22 @@ def test_miranda_subvolume_parity(L, orc, algo, field):
     check_parity(L, orc, algo, x.cpu().numpy().view(np.uint64), f"miranda/{field}")
 
 
+def test_dpratio_mixed_match_tiles(L, orc):
+    """Tiles with and without FCM matches interleaved (the encoder's all-zero
+    Dist fast path and its per-CTA cached stream alternate with the general
+    path), plus a ragged last tile."""
+    if "DPratio" not in algos_available(L):
+        pytest.skip("DPratio not built")
+    x = datagen.field("miranda_256x384x384_f64", "density", shape=(2, 384, 384)).numpy().reshape(-1).view(np.uint64)
+    x = x[: 2048 * 100 + 777].copy()
+    T = 2048
+    for t in range(3, 100, 3):  # every third tile repeats an earlier stretch: matches
+        src = (t - 3) * T + 100
+        x[t * T: t * T + 1500] = x[src: src + 1500]
+    x[50 * T + 10: 50 * T + 20] = x[50 * T + 9]  # a short constant run inside a matching-free tile
+    check_parity(L, orc, "DPratio", x, "mixed_match_tiles")
+
+
 def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
     """Full-size check: GPU stream vs oracle on a sample of chunks (compress_chunks)."""
     s = L.compress(algo, x_dev)

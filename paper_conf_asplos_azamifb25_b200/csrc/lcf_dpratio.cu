@@ -47,19 +47,10 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
 }
 
 // ============================ RAZE / RARE in shared memory ============================
-// clz histogram: plain shared atomics (1, measured fastest: the hardware
-// serialises equal bins within a warp cheaply) or match-aggregated ones (0)
-#ifndef LCF_HIST_MODE
-#define LCF_HIST_MODE 1
-#endif
-struct AdaptScratch {
-  uint32_t hist[65];
-  uint32_t cnt[64];     // per (round, warp) set counts → exclusive prefix
-  uint32_t b1[64];      // B1 bitmap words (n ≤ 2048 bits)
-  uint32_t c1m[32], off1[32], b2[32];  // encoder plan → emit: warp 0's B2 bits, nr(B1) offsets
-  uint32_t k, flag, s1, s2, nr1, b3;
-  uint32_t wtot[kDW];                   // encoder: set words per warp
-  uint16_t rank0[kDT];                  // encoder: set words before thread t's 8 words
+struct AdaptScratch {  // decoder
+  uint32_t cnt[64];    // set words before each B1 word
+  uint32_t b1[64];     // B1 bitmap words (n ≤ 2048 bits)
+  uint32_t flag, s2;
 };
 
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
@@ -107,99 +98,146 @@ __device__ __forceinline__ void load8(const uint64_t* sv, uint32_t n, uint32_t t
 // LSB-first bit writer for one thread's contiguous run of fields in a u32
 // buffer. The run's first and last words may be shared with the neighbouring
 // runs (atomicOr into a zeroed buffer); the words in between belong to this
-// thread alone (plain stores).
+// thread alone (plain stores). The pending partial word is 32 bits wide: a
+// field of up to 64 bits completes at most two words, formed by funnel shifts.
 struct BitWriter {
   uint32_t* buf;
-  uint32_t widx, nb;  // current word, pending bits in acc (< 32 between puts)
-  uint64_t acc;
-  bool first;
+  uint32_t widx, w0, nb, pw;  // current word, first word, pending bits (< 32), pending word
   __device__ __forceinline__ BitWriter(uint32_t* b, uint64_t off)
-      : buf(b), widx((uint32_t)(off >> 5)), nb((uint32_t)(off & 31)), acc(0), first(true) {}
-  __device__ __forceinline__ void emit(uint32_t w) {
-    if (first) atomicOr(buf + widx, w);
+      : buf(b), widx((uint32_t)(off >> 5)), w0((uint32_t)(off >> 5)), nb((uint32_t)(off & 31)), pw(0) {}
+  __device__ __forceinline__ void out(uint32_t w) {
+    if (widx == w0) atomicOr(buf + widx, w);
     else buf[widx] = w;
-    first = false;
     ++widx;
   }
   // append the low w bits of f (f < 2^w, 1 ≤ w ≤ 64)
   __device__ __forceinline__ void put(uint64_t f, uint32_t w) {
-    const uint64_t carry = nb ? f >> (64 - nb) : 0ull;  // bits beyond the 64-bit accumulator
-    acc |= f << nb;
-    nb += w;
-    if (nb >= 32) {
-      emit((uint32_t)acc);
-      acc = (acc >> 32) | (carry << 32);
-      nb -= 32;
-      if (nb >= 32) {
-        emit((uint32_t)acc);
-        acc >>= 32;
-        nb -= 32;
+    const uint32_t flo = (uint32_t)f, fhi = (uint32_t)(f >> 32);
+    const uint32_t o0 = pw | (flo << nb);              // bits 0..31 of pw | f << nb
+    const uint32_t o1 = __funnelshift_l(flo, fhi, nb);  // bits 32..63
+    const uint32_t o2 = __funnelshift_l(fhi, 0u, nb);   // bits 64..95
+    const uint32_t e = nb + w;
+    if (e >= 32) {
+      out(o0);
+      if (e >= 64) {
+        out(o1);
+        pw = o2;
+      } else {
+        pw = o1;
       }
+    } else {
+      pw = o0;
     }
+    nb = e & 31;
   }
   __device__ __forceinline__ void finish() {
-    if (nb) atomicOr(buf + widx, (uint32_t)acc);
+    if (nb) atomicOr(buf + widx, pw);
   }
 };
 
-// Encode L bytes at src (16-byte aligned, zero-safe slack to 16 KiB) with RAZE
-// (rare = false, L189) or RARE (rare = true, L195) into dst (16-byte aligned,
-// ≥ L + 3 + 32 bytes). All kDT compute threads call it; returns the output
-// length (FORMAT.md §6.2–6.3). Thread t owns words 8t … 8t+7 (n ≤ 2048): its
-// B1 bits are B1 byte t, and its HI and LO fields are contiguous bit runs.
-__device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, bool rare, AdaptScratch& sc,
-                                               uint32_t tid) {
+// ---------------------------- RAZE / RARE encoder ----------------------------
+// Thread t owns words 8t … 8t+7 of the stage's input (n ≤ 2048 words), held in
+// registers: its B1 bits are B1 byte t, and its HI and LO fields are contiguous
+// bit runs. A plan takes two CTA barriers; everything after the second one
+// (the k choice, B2, B3, the section sizes) is computed redundantly by every
+// warp from shared data, so no warp waits on another's serial work.
+#ifndef LCF_HISTW
+#define LCF_HISTW 0
+#endif
+struct EncScratch {
+  uint32_t hist[2][66];  // clz histograms, alternating per plan; [65]: the tile has an FCM distance
+  uint32_t b1[64];       // B1 bitmap; byte t = thread t's words
+  uint32_t wtot[kDW];    // set words per warp
+};
+
+struct APlan {
+  uint32_t n, tl, k, byte, rank0, c1m, off1, nr1, b3, hib, total;
+  bool bypass, allzero, anyd;
+};
+
+// Plan of RAZE (RARE = false, L189) or RARE (RARE = true, L195) over the L-byte
+// input whose words 8·tid … 8·tid+7 are v (0 at or past n = L/8) and whose
+// word 8·tid − 1 is p (RARE's reference of v[0]; 0 for tid 0). Before its first
+// barrier it also zeroes the other histogram and `zn` 16-byte words at zp.
+// `dflag`: this thread saw an FCM distance (reported as anyd). A-17, A-18.
+template <bool RARE>
+__device__ __forceinline__ APlan a_plan(const uint64_t (&v)[8], uint64_t p, uint32_t L, EncScratch& sc,
+                                        uint32_t par, uint32_t tid, bool dflag, uint4* zp, uint32_t zn) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
-  const uint32_t n = L / 8, tl = L % 8;
-  const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
-  // (the input was completed before a barrier of the caller; sc.hist is zero:
-  // zeroed at kernel start and again by warp 0 right after reading it)
-  uint64_t v[8];
-  load8(sv, n, tid, v);
-  const uint32_t i0 = 8 * tid;
-  const uint64_t p = (rare && i0 >= 1 && i0 - 1 < n) ? sv[i0 - 1] : 0ull;  // RARE reference of word i0
-  // ---- histogram of clz(v_i ⊕ ref_i) ----
+  APlan P;
+  P.n = L / 8;
+  P.tl = L % 8;
+  const uint32_t n = P.n, i0 = 8 * tid;
+  uint32_t* H = sc.hist[par];
+#if LCF_HISTW
+  {  // counts of z ∈ [b, b+6) (b = the warp's smallest z) are summed in packed
+     // 10-bit fields over the warp, one shared atomic per bin; others directly
+    uint32_t z[8], zmin = 65;
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const uint64_t ref = rare ? (j ? v[j - 1] : p) : 0ull;
-    const uint32_t z = i0 + j < n ? clz64(v[j] ^ ref) : 65u;
-    if (LCF_HIST_MODE == 0) {
-      const uint32_t peers = __match_any_sync(0xFFFFFFFFu, z);
-      if (z <= 64 && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&sc.hist[z], (uint32_t)__popc(peers));
-    } else {
-      if (z <= 64) atomicAdd(&sc.hist[z], 1u);
+    for (int j = 0; j < 8; ++j) {
+      const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
+      z[j] = i0 + j < n ? clz64(v[j] ^ ref) : 65u;
+      zmin = min(zmin, z[j]);
+    }
+    const uint32_t b = __reduce_min_sync(0xFFFFFFFFu, zmin);
+    uint32_t pk0 = 0, pk1 = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const uint32_t dz = z[j] - b;
+      if (dz < 3) pk0 += 1u << (10 * dz);
+      else if (dz < 6) pk1 += 1u << (10 * (dz - 3));
+      else if (z[j] <= 64) atomicAdd(&H[z[j]], 1u);
+    }
+    pk0 = __reduce_add_sync(0xFFFFFFFFu, pk0);
+    pk1 = __reduce_add_sync(0xFFFFFFFFu, pk1);
+    if (lane < 6) {
+      const uint32_t cnt = ((lane < 3 ? pk0 : pk1) >> (10 * (lane % 3))) & 1023u;
+      if (cnt && b + lane <= 64) atomicAdd(&H[b + lane], cnt);
     }
   }
-  bar_d();
-  // ---- k* = smallest argmin of est(k) = k·nz(k) + (64−k)·n, k ∈ 1..64 (A-17, A-18) ----
-  if (warp == 0) {
-    const uint32_t c0 = sc.hist[2 * lane], c1 = sc.hist[2 * lane + 1];
-    sc.hist[2 * lane] = 0;  // ready for the next plan (its atomics follow several barriers)
-    sc.hist[2 * lane + 1] = 0;
-    if (lane == 0) sc.hist[64] = 0;
-    uint32_t s = c0 + c1;
+#else
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, d);
-      if ((int)lane >= d) s += y;
-    }
+  for (int j = 0; j < 8; ++j) {
+    const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
+    if (i0 + j < n) atomicAdd(&H[clz64(v[j] ^ ref)], 1u);
+  }
+#endif
+  if (__any_sync(0xFFFFFFFFu, dflag) && lane == 0) atomicOr(&H[65], 1u);
+  if (tid < 66) sc.hist[par ^ 1][tid] = 0;  // read by the previous plan before a later barrier
+  for (uint32_t j = tid; j < zn; j += kDT) zp[j] = make_uint4(0, 0, 0, 0);
+  bar_d();
+  // ---- k* = smallest argmin of est(k) = k·nz(k) + (64−k)·n, k ∈ 1..64 (every warp) ----
+  const uint32_t c0 = H[2 * lane], c1 = H[2 * lane + 1];
+  P.allzero = H[64] == n;
+  P.anyd = H[65] != 0;
+  uint32_t s = c0 + c1;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, d);
+    if ((int)lane >= d) s += y;
+  }
+  {
     const uint32_t before = s - c0 - c1;
     const uint32_t kA = 2 * lane + 1, kB = 2 * lane + 2;  // nz(kA) = before + c0, nz(kB) = s
     const uint32_t eA = kA * (before + c0) + (64 - kA) * n, eB = kB * s + (64 - kB) * n;
     const uint32_t keyA = (eA << 7) | kA, keyB = (eB << 7) | kB;
     const uint32_t best = __reduce_min_sync(0xFFFFFFFFu, keyA < keyB ? keyA : keyB);
-    if (lane == 0) sc.k = best & 127;
+    P.k = best & 127;
+    // the fields alone (est(k*) bits) already reach the bypass size: bypass,
+    // whatever the bitmaps add (A-23)
+    P.bypass = 3 + ((best >> 7) + 7) / 8 + P.tl + ((((n + 7) / 8 + 7) / 8 + 7) / 8) >= 3 + L;
   }
-  bar_d();
-  const uint32_t k = sc.k;
-  const uint32_t sh = 64 - k;  // top(v) = v >> sh (k = 64: sh = 0)
+  if (!RARE && P.allzero) return P;  // the caller writes the fixed stream
+  if (P.bypass) return P;
+  const uint32_t k = P.k, sh = 64 - k;  // top(v) = v >> sh (k = 64: sh = 0)
   // ---- B1 byte t = this thread's set bits; ranks of the set words ----
   uint32_t byte = 0;
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
-    const uint64_t ref = rare ? (j ? v[j - 1] : p) : 0ull;
+    const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
     if (i0 + j < n && (v[j] >> sh) != (ref >> sh)) byte |= 1u << j;
   }
+  P.byte = byte;
   reinterpret_cast<uint8_t*>(sc.b1)[tid] = (uint8_t)byte;
   const uint32_t c = __popc(byte);
   uint32_t x = c;
@@ -210,139 +248,113 @@ __device__ __noinline__ uint32_t adaptive_plan(const uint8_t* src, uint32_t L, b
   }
   if (lane == 31) sc.wtot[warp] = x;
   bar_d();
-  {
-    uint32_t base = 0;
+  uint32_t base = 0, nset = 0;
 #pragma unroll
-    for (uint32_t w = 0; w < kDW; ++w)
-      if (w < warp) base += sc.wtot[w];
-    sc.rank0[tid] = (uint16_t)(base + x - c);
+  for (uint32_t w = 0; w < kDW; ++w) {
+    const uint32_t t = sc.wtot[w];
+    base += w < warp ? t : 0u;
+    nset += t;
   }
-  uint32_t nr1 = 0, b2 = 0, b3 = 0, c1m = 0, off1 = 0, b1w0 = 0, b1w1 = 0;
+  P.rank0 = base + x - c;
+  // ---- B1 → B2 → B3 (lane l: B1 bytes [8l, 8l+8) = words 2l, 2l+1 → B2 byte l) ----
   const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
-  if (warp == 0) {
-    uint32_t nset = 0;
+  const uint32_t b1w0 = sc.b1[2 * lane], b1w1 = sc.b1[2 * lane + 1];
+  const uint32_t prevb = __shfl_up_sync(0xFFFFFFFFu, b1w1 >> 24, 1);
+  uint32_t c1m = 0;
 #pragma unroll
-    for (uint32_t w = 0; w < kDW; ++w) nset += sc.wtot[w];
-    // B1 → B2 (lane: B1 bytes [8·lane, 8·lane+8) = words 2·lane, 2·lane+1)
-    b1w0 = sc.b1[2 * lane];
-    b1w1 = sc.b1[2 * lane + 1];
-    const uint32_t prevb = __shfl_up_sync(0xFFFFFFFFu, b1w1 >> 24, 1);
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const uint32_t cur = ((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3))) & 0xFF;
-      const uint32_t pre = j ? (((j - 1) < 4 ? b1w0 : b1w1) >> (8 * ((j - 1) & 3))) & 0xFF : (lane ? prevb : 0u);
-      if (cur != pre && 8 * lane + j < L1) c1m |= 1u << j;
-    }
-    b2 = c1m;  // B2 byte `lane`
-    uint32_t y = __popc(c1m);
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, y, d);
-      if ((int)lane >= d) y += o;
-    }
-    off1 = y - __popc(c1m);
-    nr1 = __shfl_sync(0xFFFFFFFFu, y, 31);
-    const uint32_t pb2 = __shfl_up_sync(0xFFFFFFFFu, b2, 1);
-    b3 = __ballot_sync(0xFFFFFFFFu, lane < L2 && b2 != (lane ? pb2 : 0u));
-    const uint32_t nr2 = __popc(b3);
-    const uint32_t hib = (nset * k + 7) / 8, lob = (n * (64 - k) + 7) / 8;
-    const uint32_t total = 3 + hib + lob + tl + nr1 + nr2 + L3;
-    if (lane == 0) {
-      sc.flag = total >= 3 + L;  // bypass (A-23)
-      sc.s1 = total;
-      sc.s2 = hib;
-      sc.nr1 = nr1;
-      sc.b3 = b3;
-    }
-    sc.c1m[lane] = c1m;
-    sc.off1[lane] = off1;
-    sc.b2[lane] = b2;
+  for (int j = 0; j < 8; ++j) {
+    const uint32_t cur = ((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3))) & 0xFF;
+    const uint32_t pre = j ? (((j - 1) < 4 ? b1w0 : b1w1) >> (8 * ((j - 1) & 3))) & 0xFF : (lane ? prevb : 0u);
+    if (cur != pre && 8 * lane + j < L1) c1m |= 1u << j;
   }
-  bar_d();
-  return sc.flag ? 3 + L : sc.s1;
+  uint32_t y = __popc(c1m);
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, y, d);
+    if ((int)lane >= d) y += o;
+  }
+  P.c1m = c1m;  // B2 byte `lane`
+  P.off1 = y - __popc(c1m);
+  P.nr1 = __shfl_sync(0xFFFFFFFFu, y, 31);
+  const uint32_t pb2 = __shfl_up_sync(0xFFFFFFFFu, c1m, 1);
+  P.b3 = __ballot_sync(0xFFFFFFFFu, lane < L2 && c1m != (lane ? pb2 : 0u));
+  P.hib = (nset * k + 7) / 8;
+  const uint32_t lob = (n * (64 - k) + 7) / 8;
+  P.total = 3 + P.hib + lob + P.tl + P.nr1 + __popc(P.b3) + L3;
+  P.bypass = P.total >= 3 + L;  // A-23
+  return P;
 }
 
-// Second half of RAZE/RARE: writes the planned output (adaptive_plan must have
-// run on the same input just before).
-__device__ __noinline__ void adaptive_emit(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
-                                           AdaptScratch& sc, uint32_t tid) {
+// Writes the planned (non-bypass) stream into dst, which is zero over its
+// first P.total bytes: fields by per-thread bit writers, the header, tail,
+// nr(B1), nr(B2) and B3 bytes as byte ORs. `tail` = the input's last L mod 8
+// bytes. No barrier: the caller orders dst's readers after it.
+__device__ __forceinline__ void a_emit(const uint64_t (&v)[8], const APlan& P, uint32_t L, const uint8_t* tail,
+                                       uint8_t* dst, const EncScratch& sc, uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
-  const uint32_t n = L / 8, tl = L % 8;
-  const uint64_t* sv = reinterpret_cast<const uint64_t*>(src);
-  const uint32_t k = sc.k, sh = 64 - k;
-  const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
-  (void)L1;
-  (void)L2;
-  (void)rare;
-  const bool bypass = sc.flag;
-  const uint32_t total = sc.s1, hib = sc.s2, nr1 = sc.nr1, b3 = sc.b3;
-  if (bypass) {  // dst[3 + j] = src[j], one funnel shift per output word
-    const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
-    uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
-    const uint32_t nw = (L + 3 + 3) / 4;
-    for (uint32_t w = tid; w < nw; w += kDT) {
-      const uint32_t lo = w ? sw[w - 1] : 0u;
-      const uint32_t hi = 4 * w < L ? sw[w] : 0u;
-      uint32_t val = w ? __funnelshift_r(lo, hi, 8) : ((L & 0xFFFFu) | (hi << 24));
-      const uint32_t keep = 3 + L - 4 * w;  // bytes of this word inside the output
-      if (keep < 4) val &= (1u << (8 * keep)) - 1u;
-      dw[w] = val;
-    }
-    bar_d();
-    return;
-  }
+  const uint32_t n = P.n, tl = P.tl, k = P.k, sh = 64 - k, wl = 64 - k, i0 = 8 * tid;
   uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
-  for (uint32_t j = tid; j < (total + 7) / 4 + 1; j += kDT) dw[j] = 0;
-  uint64_t v[8];
-  load8(sv, n, tid, v);
-  const uint32_t i0 = 8 * tid;
-  const uint32_t byte = reinterpret_cast<const uint8_t*>(sc.b1)[tid];
-  const uint32_t rank0 = sc.rank0[tid];
-  bar_d();
   // ---- HI: top fields of the set words (rank order), LO: low fields of all words ----
-  const uint64_t hi_base = 24, lo_base = 8ull * (3 + hib);
-  const uint32_t wl = 64 - k;
-  const uint64_t lmask = wl >= 64 ? ~0ull : ((1ull << wl) - 1);
-  if (byte) {
-    BitWriter bw(dw, hi_base + (uint64_t)rank0 * k);
+  if (P.byte) {
+    BitWriter bw(dw, 24 + (uint64_t)P.rank0 * k);
 #pragma unroll
     for (int j = 0; j < 8; ++j)
-      if ((byte >> j) & 1) bw.put(v[j] >> sh, k);
+      if ((P.byte >> j) & 1) bw.put(v[j] >> sh, k);
     bw.finish();
   }
   if (wl && i0 < n) {
-    BitWriter bw(dw, lo_base + (uint64_t)i0 * wl);
+    const uint64_t lmask = (1ull << wl) - 1;  // wl ≤ 63
+    BitWriter bw(dw, 8ull * (3 + P.hib) + (uint64_t)i0 * wl);
 #pragma unroll
     for (int j = 0; j < 8; ++j)
       if (i0 + j < n) bw.put(v[j] & lmask, wl);
     bw.finish();
   }
-  // ---- header, tail bytes, nr(B1), nr(B2), B3: byte ORs into the zeroed
-  // words, concurrent with the bit writers (whose edge words they may share) ----
-  auto put_byte = [&](uint32_t pos, uint32_t val) {
-    atomicOr(dw + (pos >> 2), (val & 0xFFu) << (8 * (pos & 3)));
-  };
-  const uint32_t after = 3 + hib + (n * wl + 7) / 8;
+  auto put_byte = [&](uint32_t pos, uint32_t val) { atomicOr(dw + (pos >> 2), (val & 0xFFu) << (8 * (pos & 3))); };
+  const uint32_t after = 3 + P.hib + (n * wl + 7) / 8;
   if (tid == 0) atomicOr(dw, (L & 0xFFFFu) | (k << 16));
-  if (tid < tl) put_byte(after + tid, src[8 * n + tid]);
-  if (warp == 0) {
-    const uint32_t c1m = sc.c1m[lane], b2 = sc.b2[lane];
+  if (tid < tl) put_byte(after + tid, tail[tid]);
+  if (warp == kDW - 1) {  // nr(B1), nr(B2), B3
+    const uint32_t L3 = (((n + 7) / 8 + 7) / 8 + 7) / 8;
     const uint32_t b1w0 = sc.b1[2 * lane], b1w1 = sc.b1[2 * lane + 1];
-    uint32_t p = after + tl + sc.off1[lane];
+    uint32_t q = after + tl + P.off1;
 #pragma unroll
     for (int j = 0; j < 8; ++j)
-      if ((c1m >> j) & 1) put_byte(p++, (j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
-    if ((b3 >> lane) & 1) put_byte(after + tl + nr1 + __popc(b3 & ((1u << lane) - 1)), b2);
-    if (lane < L3) put_byte(total - L3 + lane, b3 >> (8 * lane));
+      if ((P.c1m >> j) & 1) put_byte(q++, (j < 4 ? b1w0 : b1w1) >> (8 * (j & 3)));
+    if ((P.b3 >> lane) & 1) put_byte(after + tl + P.nr1 + __popc(P.b3 & ((1u << lane) - 1)), P.c1m);
+    if (lane < L3) put_byte(P.total - L3 + lane, P.b3 >> (8 * lane));
   }
-  bar_d();
 }
 
-__device__ __forceinline__ uint32_t adaptive_encode(const uint8_t* src, uint32_t L, uint8_t* dst, bool rare,
-                                                    AdaptScratch& sc, uint32_t tid) {
-  const uint32_t len = adaptive_plan(src, L, rare, sc, tid);
-  adaptive_emit(src, L, dst, rare, sc, tid);
-  return len;
+// RAZE bypass from registers (A-23): u16 L ‖ u8 0 ‖ the input words, into a
+// zeroed dst.
+__device__ __forceinline__ void a_emit_bypass_regs(const uint64_t (&v)[8], uint32_t n, uint8_t* dst, uint32_t tid) {
+  uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
+  const uint32_t i0 = 8 * tid;
+  if (tid == 0) atomicOr(dw, (8 * n) & 0xFFFFu);
+  if (i0 < n) {
+    BitWriter bw(dw, 24 + 64ull * i0);
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (i0 + j < n) bw.put(v[j], 64);
+    bw.finish();
+  }
+}
+
+// RARE bypass from shared memory: dst[0..3) = u16 L ‖ u8 0, dst[3 + j] = src[j],
+// one funnel shift per output word (whole words written; the last is masked).
+__device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t L, uint8_t* dst, uint32_t tid) {
+  const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
+  uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
+  const uint32_t nw = (L + 3 + 3) / 4;
+  for (uint32_t w = tid; w < nw; w += kDT) {
+    const uint32_t lo = w ? sw[w - 1] : 0u;
+    const uint32_t hi = 4 * w < L ? sw[w] : 0u;
+    uint32_t val = w ? __funnelshift_r(lo, hi, 8) : ((L & 0xFFFFu) | (hi << 24));
+    const uint32_t keep = 3 + L - 4 * w;  // bytes of this word inside the output
+    if (keep < 4) val &= (1u << (8 * keep)) - 1u;
+    dw[w] = val;
+  }
 }
 
 // Decode a RAZE/RARE stream of `len` bytes at src (16-byte aligned, ≥ 16 bytes
@@ -475,17 +487,15 @@ __device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t* sh, uint3
 struct DEncSmem {
   alignas(128) uint64_t xin[kTileWords];        // stage: x tile
   alignas(128) uint32_t din[kTileWords];        // stage: FCM distances of the tile
-  alignas(128) uint32_t dcp[kTileWords];        // copy of din: the stage is released after V's DIFFMS
-  alignas(128) uint64_t w[kTileWords + 8];      // DIFFMS words of V or Dist
-  alignas(128) uint8_t rz[kChunkBytes + 128];   // RAZE output
-  alignas(128) uint32_t out[kDOut][(kChunkBytes + 128) / 4];
+  alignas(128) uint8_t rz[kChunkBytes + 128];   // RAZE output (zero past what the last RAZE wrote)
+  alignas(128) uint32_t out[kDOut][(kChunkBytes + 128) / 4];  // output slots (handed back zeroed)
   uint64_t full_in[1], empty_in[1], full_out[kDOut], empty_out[kDOut];
   uint64_t in_chunk[1], out_chunk[kDOut];
   uint32_t out_len[kDOut], out_raw[kDOut];
   uint64_t scan[kDW];
   alignas(16) uint8_t zc[64];  // the Dist chunk of a full tile without distances: its stream, once made
   uint32_t zlen;               // (0 = not yet)
-  AdaptScratch sc;
+  EncScratch sc;
 };
 
 __device__ __forceinline__ void d_enc_loader(DEncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane) {
@@ -532,7 +542,10 @@ __device__ __forceinline__ void d_enc_loader(DEncSmem& S, const EncArgs& a, cons
 
 __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
-  uint32_t oit = 0;  // output-slot iteration (two chunks per tile)
+  const uint32_t i0 = 8 * tid;
+  uint32_t oit = 0;       // output-slot iteration (two chunks per tile)
+  uint32_t par = 0;       // histogram parity
+  uint32_t rz_used = 0;   // bytes of S.rz written by the last RAZE (re-zeroed by the next plan)
   for (uint32_t it = 0;; ++it) {
     mbar_wait(&S.full_in[0], it & 1);
     const uint64_t t = S.in_chunk[0];
@@ -541,11 +554,49 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       return;
     }
     const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
-    bool dist_zero = false;  // the tile has no FCM match (set by part 0)
+    // ---- FCM outputs (L170–185) and DIFFMS₆₄ (L187) of V in registers: words 8·tid … 8·tid+7 ----
+    uint64_t w[8];
+    uint32_t d[8], dprev = 0, dor = 0;
+    {
+      uint64_t x[8];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const ulonglong2 xx = reinterpret_cast<const ulonglong2*>(S.xin)[4 * tid + q];
+        x[2 * q] = xx.x;
+        x[2 * q + 1] = xx.y;
+      }
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const uint4 dd = reinterpret_cast<const uint4*>(S.din)[2 * tid + q];
+        d[4 * q] = dd.x;
+        d[4 * q + 1] = dd.y;
+        d[4 * q + 2] = dd.z;
+        d[4 * q + 3] = dd.w;
+      }
+      uint64_t prev = 0;
+      if (tid && i0 - 1 < m) {
+        dprev = S.din[i0 - 1];
+        prev = dprev ? 0ull : S.xin[i0 - 1];
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const bool in = i0 + j < m;
+        if (!in) d[j] = 0;
+        const uint64_t cur = d[j] ? 0ull : x[j];
+        w[j] = in ? tcms((uint64_t)(cur - prev)) : 0ull;
+        prev = cur;
+        dor |= d[j];
+      }
+    }
+    // the stage has been read: hand it back so the next tile loads during this one
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.empty_in[0]);
+    bool dist_zero = false;  // the tile has no FCM match (set by part 0's plan)
     for (uint32_t part = 0; part < 2; ++part, ++oit) {  // chunk 2t: V, chunk 2t+1: Dist (A-16)
       const uint64_t c = 2 * t + part;
       if (tid == 0) trace_stamp(a, c, 1);
       const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
+      uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       const bool cacheable = part == 1 && dist_zero && m == kTileWords;
       if (cacheable && S.zlen) {  // the fixed stream of an all-zero Dist chunk, made once per CTA
         const uint32_t len = S.zlen;
@@ -567,47 +618,45 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         if (lane == 0) mbar_arrive(&S.full_out[o]);
         continue;
       }
-      // FCM outputs (L170–185) and DIFFMS₆₄ (L187) into w[]
-      uint64_t nzacc = 0;
-      uint32_t dor = 0;
-      for (uint32_t i = tid; i < m; i += kDT) {
-        uint64_t cur, prev;
-        if (part == 0) {
-          const uint32_t d = S.din[i], dp = i ? S.din[i - 1] : 0u;
-          cur = d ? 0ull : S.xin[i];
-          prev = i ? (dp ? 0ull : S.xin[i - 1]) : 0ull;
-          S.dcp[i] = d;
-          dor |= d;
-        } else {
-          cur = S.dcp[i];
-          prev = i ? (uint64_t)S.dcp[i - 1] : 0ull;
+      if (part == 1) {  // DIFFMS₆₄ of the distances
+        uint64_t pd = dprev;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          w[j] = tcms((uint64_t)d[j] - pd);
+          pd = d[j];
         }
-        const uint64_t wv = tcms((uint64_t)(cur - prev));
-        S.w[i] = wv;
-        nzacc |= wv;
       }
-      // RAZE then RARE (L189–201)
+      // ---- RAZE (L189) into S.rz ----
+      const APlan P1 = a_plan<false>(w, 0ull, 8 * m, S.sc, par, tid, part == 0 && dor != 0,
+                                     reinterpret_cast<uint4*>(S.rz), (rz_used + 8 + 15) / 16);
+      par ^= 1;
+      if (part == 0) dist_zero = !P1.anyd;
       uint32_t l1;
-      const bool any = bar_d_or(nzacc != 0);
-      if (part == 0) dist_zero = !bar_d_or(dor != 0);
-      // the tile's stage has been read (V's DIFFMS words are in w, the
-      // distances in dcp): hand it back so the next tile loads during this one
-      if (part == 0 && lane == 0) mbar_arrive(&S.empty_in[0]);
-      if (any) {
-        l1 = adaptive_encode(reinterpret_cast<const uint8_t*>(S.w), 8 * m, S.rz, false, S.sc, tid);
-      } else {
+      if (P1.allzero) {
         // all-zero DIFFMS words (e.g. the Dist chunk of a tile without FCM
-        // matches): RAZE's plan is fixed — every clz is 64, so k = 64, B1..B3
-        // are zero and nothing repeats — and the stream is L | k=64 | L3 zero
-        // bytes (FORMAT.md §6.2; the same bytes adaptive_encode writes)
+        // matches): k = 64, B1..B3 are zero and nothing repeats — the stream is
+        // L | k=64 | L3 zero bytes (FORMAT.md §6.2, what a_emit would write)
         const uint32_t L = 8 * m, L3 = (((m + 7) / 8 + 7) / 8 + 7) / 8;
-        if (tid < 3 + L3) S.rz[tid] = tid == 0 ? (uint8_t)L : tid == 1 ? (uint8_t)(L >> 8) : tid == 2 ? 64 : 0;
+        if (tid < 3) S.rz[tid] = tid == 0 ? (uint8_t)L : tid == 1 ? (uint8_t)(L >> 8) : 64;
         l1 = 3 + L3;
-        bar_d();  // adaptive_plan reads its input before its first barrier
+      } else if (P1.bypass) {
+        a_emit_bypass_regs(w, m, S.rz, tid);
+        l1 = 3 + 8 * m;
+      } else {
+        a_emit(w, P1, 8 * m, nullptr, S.rz, S.sc, tid);
+        l1 = P1.total;
       }
-      // RARE is planned first: the chunk's size — and its aggregate for the
-      // look-back of later chunks — is known before an output slot is needed
-      const uint32_t l2 = adaptive_plan(S.rz, l1, true, S.sc, tid);
+      rz_used = l1;
+      bar_d();  // S.rz complete
+      // ---- RARE (L195) of the RAZE stream; planned first, so the chunk's size —
+      // and its aggregate for the look-back of later chunks — is known before an
+      // output slot is needed ----
+      uint64_t r[8];
+      load8(reinterpret_cast<const uint64_t*>(S.rz), l1 / 8, tid, r);
+      const uint64_t rp = (tid && i0 - 1 < l1 / 8) ? reinterpret_cast<const uint64_t*>(S.rz)[i0 - 1] : 0ull;
+      const APlan P2 = a_plan<true>(r, rp, l1, S.sc, par, tid, false, nullptr, 0);
+      par ^= 1;
+      const uint32_t l2 = P2.bypass ? 3 + l1 : P2.total;
       const uint32_t raw_len = 8 * m;
       const bool raw = l2 >= raw_len;  // L104, ties → raw
       const uint32_t len = raw ? raw_len : l2;
@@ -615,40 +664,36 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         lookback_publish(ctx, c, round16(len));
         trace_stamp(a, c, 2);
       }
-      mbar_wait(&S.empty_out[o], pho ^ 1);
+      mbar_wait(&S.empty_out[o], pho ^ 1);  // (the storer hands slots back zeroed)
       if (tid == 0) trace_stamp(a, c, 3);
-      uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       if (raw) {  // the V / Dist words themselves
         uint64_t* ow = reinterpret_cast<uint64_t*>(ob);
-        if (part == 0) {  // V = DIFFMS⁻¹(w): words 8·tid .. 8·tid+7, serial run + CTA scan
+        if (part == 0) {  // V = DIFFMS⁻¹(w): serial run + CTA scan
           uint64_t run = 0;
 #pragma unroll
-          for (uint32_t j = 0; j < 8; ++j) {
-            const uint32_t i = 8 * tid + j;
-            if (i < m) run += tcms_inv(S.w[i]);
-          }
+          for (uint32_t j = 0; j < 8; ++j) run += tcms_inv(w[j]);
           uint64_t all;
           uint64_t v = cta_scan_u64(run, S.scan, tid, all);
 #pragma unroll
           for (uint32_t j = 0; j < 8; ++j) {
-            const uint32_t i = 8 * tid + j;
-            if (i < m) {
-              v += tcms_inv(S.w[i]);
-              ow[i] = v;
-            }
+            v += tcms_inv(w[j]);
+            if (i0 + j < m) ow[i0 + j] = v;
           }
         } else {
-          for (uint32_t i = tid; i < m; i += kDT) ow[i] = S.dcp[i];
+#pragma unroll
+          for (uint32_t j = 0; j < 8; ++j)
+            if (i0 + j < m) ow[i0 + j] = d[j];
         }
         if (tid < 2 && (m & 1)) ow[m + tid] = 0;  // round16 pad
+      } else if (P2.bypass) {
+        a_emit_bypass_smem(S.rz, l1, ob, tid);
       } else {
-        adaptive_emit(S.rz, l1, ob, true, S.sc, tid);
-        if (tid < 16 && len + tid < round16(len)) ob[len + tid] = 0;
-        if (cacheable && round16(len) <= sizeof(S.zc)) {  // remember it (read after later barriers)
-          bar_d();
-          if (tid < round16(len)) S.zc[tid] = ob[tid];
-          if (tid == 0) S.zlen = len;
-        }
+        a_emit(r, P2, l1, S.rz + 8 * P2.n, ob, S.sc, tid);
+      }
+      if (cacheable && !raw && round16(len) <= sizeof(S.zc)) {  // remember it (read after later barriers)
+        bar_d();
+        if (tid < round16(len)) S.zc[tid] = ob[tid];
+        if (tid == 0) S.zlen = len;
       }
       if (tid == 0) {
         S.out_chunk[o] = c;
@@ -663,11 +708,16 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
   }
 }
 
-__global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kDEncThreads, 2) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (uint32_t i = threadIdx.x; i < 65; i += blockDim.x) S.sc.hist[i] = 0;  // adaptive_plan's invariant
+  // invariants: both histograms, S.rz and the output slots start zeroed
+  for (uint32_t i = threadIdx.x; i < 2 * 66; i += blockDim.x) (&S.sc.hist[0][0])[i] = 0;
+  for (uint32_t i = threadIdx.x; i < sizeof(S.rz) / 16; i += blockDim.x)
+    reinterpret_cast<uint4*>(S.rz)[i] = make_uint4(0, 0, 0, 0);
+  for (uint32_t i = threadIdx.x; i < sizeof(S.out) / 16; i += blockDim.x)
+    reinterpret_cast<uint4*>(&S.out[0][0])[i] = make_uint4(0, 0, 0, 0);
   if (threadIdx.x == 0) S.zlen = 0;
   if (threadIdx.x == 0) {
     mbar_init(&S.full_in[0], 1);
@@ -680,7 +730,7 @@ __global__ void __launch_bounds__(kDEncThreads) dpratio_encode_kernel(EncArgs a,
   }
   __syncthreads();
   if (warp == 0) d_enc_loader(S, a, ctx, lane);
-  else if (warp == 1) enc_storer<kDOut, 1>(S, a, ctx, lane, 0);
+  else if (warp == 1) enc_storer<kDOut, 1, DEncSmem, false, true>(S, a, ctx, lane, 0);
   else d_enc_compute(S, a, ctx, threadIdx.x - 64);
 }
 

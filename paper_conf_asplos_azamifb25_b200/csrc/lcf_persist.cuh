@@ -68,7 +68,9 @@ __device__ __forceinline__ void enc_loader(Sm& S, const EncArgs& a, const Launch
 // kInPlace: the compute warps encode into the chunk's own input stage (S.in),
 // and the storer hands that stage back to the loader (S.empty_in) once the TMA
 // unit has read it — no separate output ring.
-template <int NO, int NSTORERS, class Sm, bool kInPlace = false>
+// kZeroOut: the storer re-zeroes the stored bytes of an output slot before it
+// hands the slot back (the compute warps OR bit fields into a zeroed slot).
+template <int NO, int NSTORERS, class Sm, bool kInPlace = false, bool kZeroOut = false>
 __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
                                            uint32_t first) {
   for (uint32_t it = first;; it += NSTORERS) {
@@ -92,10 +94,18 @@ __device__ __forceinline__ void enc_storer(Sm& S, const EncArgs& a, const Launch
         for (uint32_t i = 0; i < a.pad_len; ++i) a.pad_start[i] = 0;
       tma_store_wait_read0();  // the slot's bytes have been read by the TMA unit
       trace_stamp(a, t, 7);
-      if constexpr (kInPlace) mbar_arrive(&S.empty_in[o]);
-      else mbar_arrive(&S.empty_out[o]);
+      if constexpr (!kZeroOut) {
+        if constexpr (kInPlace) mbar_arrive(&S.empty_in[o]);
+        else mbar_arrive(&S.empty_out[o]);
+      }
     }
     __syncwarp();
+    if constexpr (kZeroOut) {
+      uint4* z = reinterpret_cast<uint4*>(S.out[o]);
+      for (uint32_t j = lane; j < round16(len) / 16; j += 32) z[j] = make_uint4(0, 0, 0, 0);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.empty_out[o]);
+    }
   }
   if (lane == 0) tma_store_wait_all0();
 }

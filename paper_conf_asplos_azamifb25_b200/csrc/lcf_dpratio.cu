@@ -47,11 +47,6 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
 }
 
 // ============================ RAZE / RARE in shared memory ============================
-struct AdaptScratch {  // decoder
-  uint32_t cnt[64];    // set words before each B1 word
-  uint32_t b1[64];     // B1 bitmap words (n ≤ 2048 bits)
-  uint32_t flag, s2;
-};
 
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
 
@@ -359,9 +354,11 @@ __device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t 
 
 // Decode a RAZE/RARE stream of `len` bytes at src (16-byte aligned, ≥ 16 bytes
 // of readable slack) into dst (8-byte aligned, capacity cap). Returns the
-// decoded length or −1 if malformed. All kDT compute threads call it.
+// decoded length or −1 if malformed. All kDT compute threads call it. Every
+// warp rebuilds B1 from B3 → B2 → B1 itself (lane l: B1 words 2l, 2l+1 and
+// their set-word prefixes), so the only barrier is the one after dst.
 __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, uint32_t cap, bool rare,
-                               AdaptScratch& sc, uint32_t tid) {
+                               uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   if (len < 3) return -1;
   const uint32_t L = src[0] | ((uint32_t)src[1] << 8), k = src[2];
@@ -377,71 +374,63 @@ __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, u
   if (k > 64) return -1;
   const uint32_t n = L / 8, tl = L % 8, L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
   const uint32_t wl = 64 - k;
-  if (warp == 0) {
-    int bad = len < 3 + L3;
-    uint32_t b3 = 0;
-    if (!bad)
-      for (uint32_t j = 0; j < L3; ++j) b3 |= (uint32_t)src[len - L3 + j] << (8 * j);
-    const uint32_t v2 = L2 >= 32 ? 0xFFFFFFFFu : ((1u << L2) - 1u);
-    const int32_t s2 = (int32_t)len - (int32_t)L3 - __popc(b3 & v2);
-    if (s2 < 3) bad = 1;
-    const uint32_t r2 = __popc(b3 & v2 & (0xFFFFFFFFu >> (31 - lane)));
-    const uint32_t b2 = (!bad && lane < L2 && r2) ? src[s2 + r2 - 1] : 0u;  // B2 byte `lane`
-    // B1 bytes [8·lane, 8·lane+8) from the bits of B2 byte `lane`
-    const uint32_t vb = (8 * lane >= L1) ? 0u : (L1 - 8 * lane >= 8 ? 0xFFu : ((1u << (L1 - 8 * lane)) - 1u));
-    const uint32_t bits = b2 & vb;
-    uint32_t x = __popc(bits);
+  int bad = len < 3 + L3;
+  uint32_t b3 = 0;
+  if (!bad)
+    for (uint32_t j = 0; j < L3; ++j) b3 |= (uint32_t)src[len - L3 + j] << (8 * j);
+  const uint32_t v2 = L2 >= 32 ? 0xFFFFFFFFu : ((1u << L2) - 1u);
+  const int32_t s2 = (int32_t)len - (int32_t)L3 - __popc(b3 & v2);
+  if (s2 < 3) bad = 1;
+  const uint32_t r2 = __popc(b3 & v2 & (0xFFFFFFFFu >> (31 - lane)));
+  const uint32_t b2 = (!bad && lane < L2 && r2) ? src[s2 + r2 - 1] : 0u;  // B2 byte `lane`
+  // B1 bytes [8·lane, 8·lane+8) from the bits of B2 byte `lane`
+  const uint32_t vb = (8 * lane >= L1) ? 0u : (L1 - 8 * lane >= 8 ? 0xFFu : ((1u << (L1 - 8 * lane)) - 1u));
+  const uint32_t bits = b2 & vb;
+  uint32_t x = __popc(bits);
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
-      if ((int)lane >= d) x += y;
-    }
-    const int32_t s1 = s2 - (int32_t)__shfl_sync(0xFFFFFFFFu, x, 31);
-    if (s1 < 3) bad = 1;
-    bad = __any_sync(0xFFFFFFFFu, bad);
-    uint32_t r = x - __popc(bits), w0 = 0, w1 = 0;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      r += (bits >> j) & 1;
-      const uint32_t val = (!bad && r) ? src[s1 + r - 1] : 0u;
-      if (j < 4) w0 |= val << (8 * j);
-      else w1 |= val << (8 * (j - 4));
-    }
-    // B1 words cover bits 64·lane .. : mask bits ≥ n
-    const uint32_t nb0 = n > 64 * lane ? n - 64 * lane : 0;
-    if (nb0 < 32) w0 &= nb0 ? ((1u << nb0) - 1u) : 0u;
-    if (nb0 < 64) w1 &= nb0 > 32 ? ((1u << (nb0 - 32)) - 1u) : 0u;
-    sc.b1[2 * lane] = w0;
-    sc.b1[2 * lane + 1] = w1;
-    const uint32_t cw0 = __popc(w0), cw1 = __popc(w1);
-    uint32_t c = cw0 + cw1;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, c, d);
-      if ((int)lane >= d) c += y;
-    }
-    sc.cnt[2 * lane] = c - cw0 - cw1;
-    sc.cnt[2 * lane + 1] = c - cw1;
-    const uint32_t nset = __shfl_sync(0xFFFFFFFFu, c, 31);
-    const uint32_t hib = (nset * k + 7) / 8, lob = (n * wl + 7) / 8;
-    if (!bad && (int32_t)(3 + hib + lob + tl) != s1) bad = 1;
-    if (lane == 0) {
-      sc.flag = bad;
-      sc.s2 = hib;
-    }
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+    if ((int)lane >= d) x += y;
   }
-  bar_d();
-  if (sc.flag) return -1;
-  const uint32_t hib = sc.s2;
+  const int32_t s1 = s2 - (int32_t)__shfl_sync(0xFFFFFFFFu, x, 31);
+  if (s1 < 3) bad = 1;
+  bad = __any_sync(0xFFFFFFFFu, bad);
+  uint32_t r = x - __popc(bits), w0 = 0, w1 = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    r += (bits >> j) & 1;
+    const uint32_t val = (!bad && r) ? src[s1 + r - 1] : 0u;
+    if (j < 4) w0 |= val << (8 * j);
+    else w1 |= val << (8 * (j - 4));
+  }
+  // B1 words cover bits 64·lane .. : mask bits ≥ n
+  const uint32_t nb0 = n > 64 * lane ? n - 64 * lane : 0;
+  if (nb0 < 32) w0 &= nb0 ? ((1u << nb0) - 1u) : 0u;
+  if (nb0 < 64) w1 &= nb0 > 32 ? ((1u << (nb0 - 32)) - 1u) : 0u;
+  const uint32_t cw0 = __popc(w0), cw1 = __popc(w1);
+  uint32_t c = cw0 + cw1;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, c, d);
+    if ((int)lane >= d) c += y;
+  }
+  const uint32_t cnt0 = c - cw0 - cw1, cnt1 = c - cw1;  // set words before B1 words 2l, 2l+1
+  const uint32_t nset = __shfl_sync(0xFFFFFFFFu, c, 31);
+  const uint32_t hib = (nset * k + 7) / 8, lob = (n * wl + 7) / 8;
+  if (!bad && (int32_t)(3 + hib + lob + tl) != s1) bad = 1;
+  if (bad) return -1;  // (warp-uniform, and the same in every warp)
   const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
   const uint64_t lo_base = 8ull * (3 + hib);
-  // word i = 32·(b1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane
+  // word i = 32·(B1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane;
+  // q's parity is the warp's (kDW even), so the source register is warp-uniform
+  static_assert(kDW % 2 == 0, "B1 word parity = warp parity");
+  const uint32_t wsel = (warp & 1) ? w1 : w0, csel = (warp & 1) ? cnt1 : cnt0;
 #pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const uint32_t i = tid + kDT * r;
-    const uint32_t q = r * kDW + warp;
-    const uint32_t bw = sc.b1[q];
-    const uint32_t re = sc.cnt[q] + __popc(bw & ((1u << lane) - 1));  // set words before i
+  for (int r8 = 0; r8 < 8; ++r8) {
+    const uint32_t i = tid + kDT * r8;
+    const uint32_t q = r8 * kDW + warp;
+    const uint32_t bw = __shfl_sync(0xFFFFFFFFu, wsel, q >> 1);
+    const uint32_t re = __shfl_sync(0xFFFFFFFFu, csel, q >> 1) + __popc(bw & ((1u << lane) - 1));  // set words before i
     const bool set = (bw >> lane) & 1;
     if (i < n) {
       uint64_t tp;
@@ -460,8 +449,10 @@ __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, u
   return (int)L;
 }
 
-// CTA-wide exclusive scan of u64 over the kDT compute threads (slot `sh`).
-__device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t* sh, uint32_t tid, uint64_t& total) {
+// CTA-wide exclusive scan of u64 over the kDT compute threads. The warp sums go
+// to slot sh[sp] and sp flips, so consecutive scans need no trailing barrier.
+__device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t (*sh)[kDW], uint32_t& sp, uint32_t tid,
+                                                 uint64_t& total) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   uint64_t x = v;
 #pragma unroll
@@ -469,17 +460,18 @@ __device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t* sh, uint3
     const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
     if ((int)lane >= d) x += y;
   }
-  if (lane == 31) sh[warp] = x;
+  uint64_t* s = sh[sp];
+  sp ^= 1;
+  if (lane == 31) s[warp] = x;
   bar_d();
   uint64_t base = 0;
   total = 0;
 #pragma unroll
   for (uint32_t i = 0; i < kDW; ++i) {
-    const uint64_t s = sh[i];
-    if (i < warp) base += s;
-    total += s;
+    const uint64_t t = s[i];
+    if (i < warp) base += t;
+    total += t;
   }
-  bar_d();  // the slot may be reused right away
   return base + x - v;
 }
 
@@ -492,7 +484,7 @@ struct DEncSmem {
   uint64_t full_in[1], empty_in[1], full_out[kDOut], empty_out[kDOut];
   uint64_t in_chunk[1], out_chunk[kDOut];
   uint32_t out_len[kDOut], out_raw[kDOut];
-  uint64_t scan[kDW];
+  uint64_t scan[2][kDW];  // cta_scan_u64 slots (alternating)
   alignas(16) uint8_t zc[64];  // the Dist chunk of a full tile without distances: its stream, once made
   uint32_t zlen;               // (0 = not yet)
   EncScratch sc;
@@ -546,6 +538,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
   uint32_t oit = 0;       // output-slot iteration (two chunks per tile)
   uint32_t par = 0;       // histogram parity
   uint32_t rz_used = 0;   // bytes of S.rz written by the last RAZE (re-zeroed by the next plan)
+  uint32_t sp = 0;        // cta_scan_u64 slot parity
   for (uint32_t it = 0;; ++it) {
     mbar_wait(&S.full_in[0], it & 1);
     const uint64_t t = S.in_chunk[0];
@@ -673,7 +666,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
 #pragma unroll
           for (uint32_t j = 0; j < 8; ++j) run += tcms_inv(w[j]);
           uint64_t all;
-          uint64_t v = cta_scan_u64(run, S.scan, tid, all);
+          uint64_t v = cta_scan_u64(run, S.scan, sp, tid, all);
 #pragma unroll
           for (uint32_t j = 0; j < 8; ++j) {
             v += tcms_inv(w[j]);
@@ -745,8 +738,7 @@ struct DDecSmem {
   uint64_t full_in[1], empty_in[1];
   uint64_t tile[1];
   uint32_t len[1][2], flags[1];
-  uint64_t scan[kDW];
-  AdaptScratch sc;
+  uint64_t scan[2][kDW];  // cta_scan_u64 slots (alternating)
   int32_t bad;
 };
 
@@ -842,10 +834,10 @@ __device__ __forceinline__ int d_decode_step1(DDecSmem& S, const uint8_t* pay, u
     nz = bar_d_or(acc != 0);
     return kRawDone;
   }
-  return adaptive_decode(pay, len, rz, kChunkBytes + 3, true, S.sc, tid);
+  return adaptive_decode(pay, len, rz, kChunkBytes + 3, true, tid);
 }
 __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_t* rz, uint32_t m, uint64_t* arr,
-                                               bool& nz, bool want_zeros, uint32_t tid) {
+                                               bool& nz, bool want_zeros, uint32_t& sp, uint32_t tid) {
   if (l1 == kRawDone) return true;
   if (l1 < 0) return false;
   {  // the RAZE stream of an all-zero chunk: k = 64 and nothing but the B3
@@ -857,14 +849,15 @@ __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_
       bool z = true;
       for (uint32_t j = 0; j < L3; ++j) z = z && rz[3 + j] == 0;
       if (!z) return false;
-      if (want_zeros)
-        for (uint32_t i = tid; i < m; i += kDT) arr[i] = 0;  // DIFFMS⁻¹ of zeros
       nz = false;
-      bar_d();
+      if (want_zeros) {  // DIFFMS⁻¹ of zeros
+        for (uint32_t i = tid; i < m; i += kDT) arr[i] = 0;
+        bar_d();
+      }
       return true;
     }
   }
-  const int l0 = adaptive_decode(rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, S.sc, tid);
+  const int l0 = adaptive_decode(rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, tid);
   if (l0 != (int)(8 * m)) return false;
   // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8), moved as 16-byte pairs
   uint64_t v[8], run = 0;
@@ -876,7 +869,7 @@ __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_
     run += v[j] + v[j + 1];
   }
   uint64_t tot;
-  uint64_t acc = cta_scan_u64(run, S.scan, tid, tot);
+  uint64_t acc = cta_scan_u64(run, S.scan, sp, tid, tot);
   uint64_t any = 0;
 #pragma unroll
   for (int j = 0; j < 8; j += 2) {
@@ -886,7 +879,7 @@ __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_
     if (8 * tid + j < m) any |= a0;
     if (8 * tid + j + 1 < m) any |= a1;
   }
-  nz = bar_d_or(any != 0);
+  nz = want_zeros ? false : bar_d_or(any != 0);  // (V: not needed; its readers follow later barriers)
   return true;
 }
 
@@ -899,6 +892,7 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   // completion (and the tile's flag) is awaited only before S.V is written
   // again, or at exit.
   uint64_t pending = kNoChunk;
+  uint32_t sp = 0;  // cta_scan_u64 slot parity
   auto finish_pending = [&]() {
     if (tid == 0 && pending != kNoChunk) {
       tma_store_wait_all0();
@@ -920,10 +914,11 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
     if (tid == 0) trace_stamp(a, t, 2);
     bool ok = !(fl & 4), nzV = false, nzD = false;
     int l1V = -1, l1D = -1;
-    if (fl & 1) {  // a raw V chunk is copied into S.V right away
-      finish_pending();
-      bar_d();
-    }
+    // thread 0 waits for the previous tile's bulk store out of S.V; step 1's
+    // barriers order that before anything writes S.V (a raw V chunk is copied
+    // into S.V by step 1 itself, so it gets a barrier of its own)
+    finish_pending();
+    if (fl & 1) bar_d();
     if (ok) {
       l1V = d_decode_step1(S, S.in[0], S.len[0][0], fl & 1, m, S.rz[0], S.V, nzV, tid);
       l1D = d_decode_step1(S, S.in[1], S.len[0][1], (fl >> 1) & 1, m, S.rz[1], S.D, nzD, tid);
@@ -933,15 +928,15 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
     __syncwarp();
     if (lane == 0) mbar_arrive(&S.empty_in[0]);
     if (tid == 0) trace_stamp(a, t, 3);
-    finish_pending();  // (step 2 writes S.V only after its first barrier)
-    if (ok) ok = d_decode_step2(S, l1V, S.rz[0], m, S.V, nzV, true, tid);
+    if (ok) ok = d_decode_step2(S, l1V, S.rz[0], m, S.V, nzV, true, sp, tid);
     if (tid == 0) trace_stamp(a, t, 4);
-    if (ok) ok = d_decode_step2(S, l1D, S.rz[1], m, S.D, nzD, false, tid);  // (D unread if all zero)
+    if (ok) ok = d_decode_step2(S, l1D, S.rz[1], m, S.D, nzD, false, sp, tid);  // (D unread if all zero)
     if (tid == 0) trace_stamp(a, t, 5);
     // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
     const uint64_t t0 = t * kTileWords;
     bool bad = !ok;
     if (ok && nzD) {  // (no distances: x = V as it stands)
+      bar_d();  // S.V complete (V's DIFFMS⁻¹ ends without a barrier)
       for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
         const uint32_t li = b + tid;
         int32_t p = -1;

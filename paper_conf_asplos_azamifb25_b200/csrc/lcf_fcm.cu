@@ -26,7 +26,10 @@ namespace {
 
 constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
 constexpr int kDigitBits = 10, kDigits = 1 << kDigitBits;
-constexpr int kSortWarps = 16, kSortThreads = kSortWarps * 32, kWarpRecs = 1024;
+#ifndef LCF_WARP_RECS
+#define LCF_WARP_RECS 1024
+#endif
+constexpr int kSortWarps = 16, kSortThreads = kSortWarps * 32, kWarpRecs = LCF_WARP_RECS;
 constexpr uint32_t kTile = kSortWarps * kWarpRecs;
 constexpr int kRecHashShift = 44, kRecFpShift = 32;
 constexpr uint64_t kRecIdxMask = 0xFFFFFFFFull;

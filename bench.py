@@ -306,6 +306,7 @@ def run_lcf(args):
 
     e2e = run_e2e(lcf, jobs, args) if rank == 0 else None
     cpu = run_cpu_baseline(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
+    cpu_codec = run_cpu_codec(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
     if rank == 0:
         line = {
             "metric": "compress+decompress throughput (uncompressed GB/s)", "value": value, "unit": "GB/s",
@@ -314,7 +315,7 @@ def run_lcf(args):
             "vs_baseline": None, "dtype": "u32/u64 (f32/f64 bits)", "data": "synthetic",
             "config": {"workload": WORKLOAD, "l2": "flushed (256 MiB write) before every timed call",
                        "parallelism": f"chunk-range shards x{world}" if world > 1 else "single GPU"},
-            "per_codec": per_codec, "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "per_codec": per_codec, "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "cpu_codec": cpu_codec, "e2e": e2e,
             "gpu_launches": launches, "clocks": clk.summary(),
         }
         print(json.dumps(line))
@@ -388,6 +389,30 @@ def run_cpu_baseline(jobs, budget_s: float = 12.0):
     return {"value": done_bytes / spent / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
             "sample": f"first {sample_bytes >> 20} MiB of every (codec, field) of the workload, compress+decompress, "
                       f"x{reps}; {spent:.1f} s single-threaded"}
+
+
+def run_cpu_codec(jobs):
+    """The multi-threaded CPU codec (liblcf_cpu.so) on the
+    whole workload, one step, all host cores: same metric; its streams must be
+    the GPU's bytes (the paper's CPU/GPU compatibility, L354)."""
+    from paper_conf_asplos_azamifb25_b200 import lcf_cpu
+    lcf_cpu.lib()
+    nt = os.cpu_count() or 1
+    host = []
+    for j in jobs:
+        words = j["x"].cpu().numpy()
+        host.append((j, words.view(np.uint32 if words.dtype == np.int32 else np.uint64),
+                     j["s"][: j["sbytes"]].cpu().numpy()))
+    total, spent, same = 0, 0.0, True
+    for j, words, s_gpu in host:
+        t0 = time.perf_counter()
+        s = lcf_cpu.lcf_cpu_compress(j["codec"], words, n_threads=nt)
+        y = lcf_cpu.lcf_cpu_decompress(j["codec"], s, n_threads=nt)
+        spent += time.perf_counter() - t0
+        total += 2 * words.nbytes
+        same = same and s.tobytes() == s_gpu.tobytes() and np.array_equal(y, words)
+    return {"value": total / spent / 1e9, "unit": "GB/s", "cores": nt, "kind": "cpu_codec (liblcf_cpu.so)",
+            "streams_equal_gpu": bool(same), "sample": "the whole workload, one step (compress + decompress)"}
 
 
 def run_reference(args):

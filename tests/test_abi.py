@@ -69,3 +69,27 @@ def test_no_device_means_error_not_fallback(L):
     with pytest.raises(L.LcfError) as e:
         L.lcf_compress_host("SPspeed", None, x, x.nbytes, out, out.nbytes, stream=0)
     assert e.value.status == 5
+
+
+def test_cpu_library_exports_every_declared_symbol():
+    """liblcf_cpu.so (include/lcf_cpu.h): separate from liblcf.so, which must not
+    export any lcf_cpu_* symbol (the GPU library has no CPU codec path)."""
+    from paper_conf_asplos_azamifb25_b200 import build
+    build.build_cpu()
+    with open(os.path.join(ROOT, "include", "lcf_cpu.h")) as f:
+        src = re.sub(r"/\*.*?\*/", "", f.read(), flags=re.S)
+    names = sorted(set(re.findall(r"\b(lcf_cpu_[a-z_]+)\s*\(", src)))
+    assert len(names) == 3
+    lib = ctypes.CDLL(build.CPU_LIB)
+    for n in names:
+        assert hasattr(lib, n), n
+    gpu = ctypes.CDLL(build.LIB)
+    for n in names:
+        assert not hasattr(gpu, n), n
+
+
+@pytest.mark.parametrize("algo", ["SPspeed", "SPratio", "DPspeed", "DPratio"])
+def test_cpu_max_size_matches(L, algo):
+    from paper_conf_asplos_azamifb25_b200 import lcf_cpu
+    for n in [0, 8, 16384, 16384 * 3 + 8, 25920000, 301989888]:
+        assert lcf_cpu.lcf_cpu_max_compressed_size(algo, n) == L.lcf_max_compressed_size(algo, None, n)

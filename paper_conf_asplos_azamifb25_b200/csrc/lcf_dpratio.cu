@@ -357,17 +357,19 @@ __device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t 
 // decoded length or −1 if malformed. All kDT compute threads call it. Every
 // warp rebuilds B1 from B3 → B2 → B1 itself (lane l: B1 words 2l, 2l+1 and
 // their set-word prefixes), so the only barrier is the one after dst.
-__device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, uint32_t cap, bool rare,
+__device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, uint8_t* dst, uint32_t cap, bool rare,
                                uint32_t tid) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
+  const uint8_t* src = base + off;  // the stream (base: 4-byte aligned)
   if (len < 3) return -1;
   const uint32_t L = src[0] | ((uint32_t)src[1] << 8), k = src[2];
   if (L > cap) return -1;
   if (k == 0) {  // bypass: dst[j] = src[3 + j], one funnel shift per word
     if (len != 3 + L) return -1;
-    const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
+    const uint32_t* sw = reinterpret_cast<const uint32_t*>(base) + (off + 3) / 4;
+    const uint32_t fs = 8 * ((off + 3) % 4);
     uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
-    for (uint32_t w = tid; w < (L + 3) / 4; w += kDT) dw[w] = __funnelshift_r(sw[w], sw[w + 1], 24);
+    for (uint32_t w = tid; w < (L + 3) / 4; w += kDT) dw[w] = __funnelshift_r(sw[w], sw[w + 1], fs);
     bar_d();
     return (int)L;
   }
@@ -419,8 +421,9 @@ __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, u
   const uint32_t hib = (nset * k + 7) / 8, lob = (n * wl + 7) / 8;
   if (!bad && (int32_t)(3 + hib + lob + tl) != s1) bad = 1;
   if (bad) return -1;  // (warp-uniform, and the same in every warp)
-  const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
-  const uint64_t lo_base = 8ull * (3 + hib);
+  const uint32_t* sw = reinterpret_cast<const uint32_t*>(base);
+  const uint64_t f0 = 8ull * off;  // bit position of the stream in base
+  const uint64_t lo_base = f0 + 8ull * (3 + hib);
   // word i = 32·(B1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane;
   // q's parity is the warp's (kDW even), so the source register is warp-uniform
   static_assert(kDW % 2 == 0, "B1 word parity = warp parity");
@@ -436,15 +439,15 @@ __device__ int adaptive_decode(const uint8_t* src, uint32_t len, uint8_t* dst, u
       uint64_t tp;
       if (rare) {
         const uint32_t ri = re + set;  // set words up to and including i
-        tp = ri ? get_field(sw, 24 + (uint64_t)(ri - 1) * k, k) : 0;
+        tp = ri ? get_field(sw, f0 + 24 + (uint64_t)(ri - 1) * k, k) : 0;
       } else {
-        tp = set ? get_field(sw, 24 + (uint64_t)re * k, k) : 0;
+        tp = set ? get_field(sw, f0 + 24 + (uint64_t)re * k, k) : 0;
       }
       const uint64_t lw = get_field(sw, lo_base + (uint64_t)i * wl, wl);
       *reinterpret_cast<uint64_t*>(dst + 8 * i) = k == 64 ? tp : ((tp << wl) | lw);
     }
   }
-  if (tid < tl) dst[8 * n + tid] = src[lo_base / 8 + (n * wl + 7) / 8 + tid];
+  if (tid < tl) dst[8 * n + tid] = base[lo_base / 8 + (n * wl + 7) / 8 + tid];
   bar_d();
   return (int)L;
 }
@@ -728,19 +731,26 @@ __global__ void __launch_bounds__(kDEncThreads, 2) dpratio_encode_kernel(EncArgs
 }
 
 // =================================== decode ======================================
+// Four 16.5 KB buffers (3 CTAs per SM): the V payload stage sv (released right
+// after V's RARE⁻¹), the Dist payload stage sd (which then holds the Dist
+// words: raw in place, or RAZE⁻¹'s output), rz (RARE⁻¹ output of V, then of
+// Dist; the FCM decode's pointer-jumping scratch) and X (V, then the decoded
+// tile in place, stored by TMA).
 struct DDecSmem {
-  alignas(128) uint8_t in[2][kChunkBytes + 128];  // stage: V and Dist payloads of a tile
-  alignas(128) uint8_t rz[2][kChunkBytes + 128];  // RARE⁻¹ outputs (RAZE streams) of V and Dist
-  alignas(128) uint64_t V[kTileWords + 8];        // V, then the decoded tile in place
-  alignas(128) uint64_t D[kTileWords + 8];
-  int32_t pj[2][kDT];                             // pointer jumping: target (−1 done)
-  uint64_t vj[2][kDT];
-  uint64_t full_in[1], empty_in[1];
+  alignas(128) uint8_t sv[kChunkBytes + 128];
+  alignas(128) uint8_t sd[kChunkBytes + 128];
+  alignas(128) uint8_t rz[kChunkBytes + 128];
+  alignas(128) uint64_t X[kTileWords + 8];
+  uint64_t full_v[1], empty_v[1], full_d[1], empty_d[1];
   uint64_t tile[1];
-  uint32_t len[1][2], flags[1];
+  uint32_t len[2], flags[1];
   uint64_t scan[2][kDW];  // cta_scan_u64 slots (alternating)
-  int32_t bad;
 };
+struct FcmScratch {  // pointer jumping (aliases S.rz)
+  int32_t pj[2][kDT];  // target (−1 done)
+  uint64_t vj[2][kDT];
+};
+static_assert(sizeof(FcmScratch) <= kChunkBytes, "FCM scratch fits in rz");
 
 __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t lane) {
   uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
@@ -753,12 +763,12 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
     if (lane == 0) tb = atomicAdd(ctx.ticket, 1ull);
     tb = __shfl_sync(0xFFFFFFFFu, tb, 0) * kDBatch;
     if (!hdr_ok || small || tb >= T) {
-      mbar_wait(&S.empty_in[0], (it & 1) ^ 1);
+      mbar_wait(&S.empty_v[0], (it & 1) ^ 1);
       if (lane == 0) {
         if (tb == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
         if (tb == 0 && small) record_error(ctx, DERR_SMALL);
         S.tile[0] = kNoChunk;
-        mbar_arrive(&S.full_in[0]);
+        mbar_arrive(&S.full_v[0]);
         ticket_retire(ctx);
       }
       return;
@@ -793,71 +803,55 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
       const uint32_t r0 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j), r1 = __shfl_sync(0xFFFFFFFFu, raw, 2 * j + 1);
       const bool b0 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j), b1 = __shfl_sync(0xFFFFFFFFu, bad, 2 * j + 1);
       const uint64_t e0 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j), e1 = __shfl_sync(0xFFFFFFFFu, excl, 2 * j + 1);
+      const bool bb = b0 || b1;
       if (lane == 0) trace_stamp(a, tb + j, 0);
-      mbar_wait(&S.empty_in[0], (it & 1) ^ 1);
+      mbar_wait(&S.empty_v[0], (it & 1) ^ 1);
       if (lane == 0) {
         trace_stamp(a, tb + j, 1);
-        const bool bb = b0 || b1;
         if (bb) record_error(ctx, DERR_CORRUPT);
         S.tile[0] = tb + j;
-        S.len[0][0] = l0;
-        S.len[0][1] = l1;
+        S.len[0] = l0;
+        S.len[1] = l1;
         S.flags[0] = r0 | (r1 << 1) | (bb ? 4u : 0u);
-        const uint32_t tx = bb ? 0 : (uint32_t)(round16(l0) + round16(l1));
-        if (tx) {
-          mbar_arrive_expect_tx(&S.full_in[0], tx);
-          if (l0) tma_load_1d(S.in[0], a.stream + base + e0, (uint32_t)round16(l0), &S.full_in[0]);
-          if (l1) tma_load_1d(S.in[1], a.stream + base + e1, (uint32_t)round16(l1), &S.full_in[0]);
+        if (!bb && l0) {
+          mbar_arrive_expect_tx(&S.full_v[0], (uint32_t)round16(l0));
+          tma_load_1d(S.sv, a.stream + base + e0, (uint32_t)round16(l0), &S.full_v[0]);
         } else {
-          mbar_arrive(&S.full_in[0]);
+          mbar_arrive(&S.full_v[0]);
+        }
+      }
+      mbar_wait(&S.empty_d[0], (it & 1) ^ 1);
+      if (lane == 0) {
+        if (!bb && l1) {
+          mbar_arrive_expect_tx(&S.full_d[0], (uint32_t)round16(l1));
+          tma_load_1d(S.sd, a.stream + base + e1, (uint32_t)round16(l1), &S.full_d[0]);
+        } else {
+          mbar_arrive(&S.full_d[0]);
         }
       }
     }
   }
 }
 
-// One chunk of a tile in two steps, so that the tile's payload stage can be
-// released between them. Step 1 reads the payload: RARE⁻¹ into rz (returns its
-// length), or a raw chunk straight into arr (returns kRawDone; *nz = any
-// non-zero word). Step 2: RAZE⁻¹ into arr and DIFFMS⁻¹ in place (*nz = any
-// non-zero result). Both return −1 / false if malformed.
-constexpr int kRawDone = -2;
-__device__ __forceinline__ int d_decode_step1(DDecSmem& S, const uint8_t* pay, uint32_t len, bool raw, uint32_t m,
-                                              uint8_t* rz, uint64_t* arr, bool& nz, uint32_t tid) {
-  if (raw) {
-    uint64_t acc = 0;
-    for (uint32_t i = tid; i < m; i += kDT) {
-      const uint64_t w = reinterpret_cast<const uint64_t*>(pay)[i];
-      arr[i] = w;
-      acc |= w;
-    }
-    nz = bar_d_or(acc != 0);
-    return kRawDone;
-  }
-  return adaptive_decode(pay, len, rz, kChunkBytes + 3, true, tid);
+// RAZE stream of an all-zero chunk (the encoder's fixed stream): k = 64 and
+// nothing but L3 zero B3 bytes. Returns 1 if rz is exactly that, 0 if it is
+// not of that shape, −1 if it has that shape with a non-zero B3 byte (any set
+// B3 bit would claim nr(B2) bytes that are not there: malformed).
+__device__ __forceinline__ int fixed_zero_stream(const uint8_t* rz, int l1, uint32_t m) {
+  const uint32_t L = rz[0] | ((uint32_t)rz[1] << 8), n = L / 8;
+  const uint32_t L3 = (((n + 7) / 8 + 7) / 8 + 7) / 8;
+  if (!(l1 >= 3 && rz[2] == 64 && L == 8 * m && (uint32_t)l1 == 3 + L3)) return 0;
+  for (uint32_t j = 0; j < L3; ++j)
+    if (rz[3 + j]) return -1;
+  return 1;
 }
-__device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_t* rz, uint32_t m, uint64_t* arr,
-                                               bool& nz, bool want_zeros, uint32_t& sp, uint32_t tid) {
-  if (l1 == kRawDone) return true;
-  if (l1 < 0) return false;
-  {  // the RAZE stream of an all-zero chunk: k = 64 and nothing but the B3
-     // bytes, which a valid stream then has all zero (any set B3 bit would
-     // claim nr(B2) bytes that are not there) — the encoder's fixed stream
-    const uint32_t L = rz[0] | ((uint32_t)rz[1] << 8), n = L / 8;
-    const uint32_t L3 = (((n + 7) / 8 + 7) / 8 + 7) / 8;
-    if (l1 >= 3 && rz[2] == 64 && L == 8 * m && (uint32_t)l1 == 3 + L3) {
-      bool z = true;
-      for (uint32_t j = 0; j < L3; ++j) z = z && rz[3 + j] == 0;
-      if (!z) return false;
-      nz = false;
-      if (want_zeros) {  // DIFFMS⁻¹ of zeros
-        for (uint32_t i = tid; i < m; i += kDT) arr[i] = 0;
-        bar_d();
-      }
-      return true;
-    }
-  }
-  const int l0 = adaptive_decode(rz, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, tid);
+
+// RAZE⁻¹ of the stream at rz + off (length l1) into arr (m words) and
+// DIFFMS⁻¹ in place (L94: the inverse stages in reverse order). Ends without a
+// barrier after the scan; returns false if malformed.
+__device__ __forceinline__ bool raze_diffms_inv(const uint8_t* rz, uint32_t off, int l1, uint32_t m, uint64_t* arr,
+                                                uint64_t& any, DDecSmem& S, uint32_t& sp, uint32_t tid) {
+  const int l0 = adaptive_decode(rz, off, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, tid);
   if (l0 != (int)(8 * m)) return false;
   // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8), moved as 16-byte pairs
   uint64_t v[8], run = 0;
@@ -870,7 +864,7 @@ __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_
   }
   uint64_t tot;
   uint64_t acc = cta_scan_u64(run, S.scan, sp, tid, tot);
-  uint64_t any = 0;
+  any = 0;
 #pragma unroll
   for (int j = 0; j < 8; j += 2) {
     const uint64_t a0 = acc + v[j], a1 = a0 + v[j + 1];
@@ -879,7 +873,6 @@ __device__ __forceinline__ bool d_decode_step2(DDecSmem& S, int l1, const uint8_
     if (8 * tid + j < m) any |= a0;
     if (8 * tid + j + 1 < m) any |= a1;
   }
-  nz = want_zeros ? false : bar_d_or(any != 0);  // (V: not needed; its readers follow later barriers)
   return true;
 }
 
@@ -888,8 +881,8 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
   const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / 8;
   uint64_t* out = reinterpret_cast<uint64_t*>(a.out);
-  // The decoded tile leaves S.V by a TMA bulk store issued by thread 0; its
-  // completion (and the tile's flag) is awaited only before S.V is written
+  // The decoded tile leaves S.X by a TMA bulk store issued by thread 0; its
+  // completion (and the tile's flag) is awaited only before S.X is written
   // again, or at exit.
   uint64_t pending = kNoChunk;
   uint32_t sp = 0;  // cta_scan_u64 slot parity
@@ -902,55 +895,107 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
     }
     pending = kNoChunk;
   };
+  auto release = [&](uint64_t* bar) {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(bar);
+  };
+  FcmScratch& F = *reinterpret_cast<FcmScratch*>(S.rz);
   for (uint32_t it = 0;; ++it) {
-    mbar_wait(&S.full_in[0], it & 1);
+    mbar_wait(&S.full_v[0], it & 1);
     const uint64_t t = S.tile[0];
     if (t == kNoChunk) {
       finish_pending();
       return;
     }
-    const uint32_t fl = S.flags[0];
+    const uint32_t fl = S.flags[0], lenV = S.len[0], lenD = S.len[1];
     const uint32_t m = (uint32_t)umin64(kTileWords, n_words - t * kTileWords);
     if (tid == 0) trace_stamp(a, t, 2);
-    bool ok = !(fl & 4), nzV = false, nzD = false;
-    int l1V = -1, l1D = -1;
-    // thread 0 waits for the previous tile's bulk store out of S.V; step 1's
-    // barriers order that before anything writes S.V (a raw V chunk is copied
-    // into S.V by step 1 itself, so it gets a barrier of its own)
-    finish_pending();
-    if (fl & 1) bar_d();
-    if (ok) {
-      l1V = d_decode_step1(S, S.in[0], S.len[0][0], fl & 1, m, S.rz[0], S.V, nzV, tid);
-      l1D = d_decode_step1(S, S.in[1], S.len[0][1], (fl >> 1) & 1, m, S.rz[1], S.D, nzD, tid);
+    bool ok = !(fl & 4);
+    const uint64_t t0 = t * kTileWords;
+    // ---- Dist first: RARE⁻¹ → rz, RAZE⁻¹ → sd (a raw Dist chunk stays in sd) ----
+    mbar_wait(&S.full_d[0], it & 1);
+    const uint64_t* Dw = reinterpret_cast<const uint64_t*>(S.sd);
+    bool nzD = false;
+    if (ok && (fl & 2)) {
+      uint64_t acc = 0;
+      for (uint32_t i = tid; i < m; i += kDT) acc |= Dw[i];
+      nzD = bar_d_or(acc != 0);
+    } else if (ok) {
+      const int l1D = adaptive_decode(S.sd, 0, lenD, S.rz, kChunkBytes + 3, true, tid);
+      const int fz = l1D < 0 ? -1 : fixed_zero_stream(S.rz, l1D, m);
+      if (fz < 0) {
+        ok = false;
+      } else if (!fz) {
+        uint64_t any;
+        ok = raze_diffms_inv(S.rz, 0, l1D, m, reinterpret_cast<uint64_t*>(S.sd), any, S, sp, tid);
+        if (ok) nzD = bar_d_or(any != 0);
+      }
     }
-    // both payloads have been read (RARE⁻¹ outputs in rz, raw chunks in V / D):
-    // the loader may fetch the next tile while this one finishes
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&S.empty_in[0]);
+    // thread 0 waits for a previous bulk store out of X (only tiles with
+    // distances use one); the barrier orders that and every read of rz before
+    // V writes X and rz
+    finish_pending();
+    ok = !bar_d_or(!ok);
+    if (!nzD) release(&S.empty_d[0]);
     if (tid == 0) trace_stamp(a, t, 3);
-    if (ok) ok = d_decode_step2(S, l1V, S.rz[0], m, S.V, nzV, true, sp, tid);
+    // ---- V: RAZE⁻¹ → X and DIFFMS⁻¹ in X (the decoded tile leaves X by a TMA
+    // bulk store) ----
+    if (ok && (fl & 1)) {  // raw V chunk: the V words themselves
+      const uint64_t* sw = reinterpret_cast<const uint64_t*>(S.sv);
+      for (uint32_t i = tid; i < m; i += kDT) S.X[i] = sw[i];
+      bar_d();
+      release(&S.empty_v[0]);
+    } else if (ok) {
+      // RARE bypassed (k = 0, A-23): RAZE⁻¹ reads the stream in place at sv + 3;
+      // otherwise RARE⁻¹ → rz first and sv is released right away
+      const uint32_t L = S.sv[0] | ((uint32_t)S.sv[1] << 8);
+      const bool inplace = lenV >= 3 && S.sv[2] == 0 && lenV == 3 + L;
+      int l1V = (int)L;
+      if (!inplace) {
+        l1V = adaptive_decode(S.sv, 0, lenV, S.rz, kChunkBytes + 3, true, tid);
+        ok = l1V >= 0;
+        release(&S.empty_v[0]);
+      }
+      const uint8_t* zb = inplace ? S.sv : S.rz;
+      const uint32_t zoff = inplace ? 3 : 0;
+      if (ok) {
+        const int fz = fixed_zero_stream(zb + zoff, l1V, m);
+        if (fz < 0) {
+          ok = false;
+        } else if (fz) {  // DIFFMS⁻¹ of zeros
+          for (uint32_t i = tid; i < m; i += kDT) S.X[i] = 0;
+        } else {
+          uint64_t any;
+          ok = raze_diffms_inv(zb, zoff, l1V, m, S.X, any, S, sp, tid);
+        }
+      }
+      if (inplace) {
+        bar_d();  // every thread is past its reads of sv
+        release(&S.empty_v[0]);
+      }
+    } else {
+      release(&S.empty_v[0]);
+    }
     if (tid == 0) trace_stamp(a, t, 4);
-    if (ok) ok = d_decode_step2(S, l1D, S.rz[1], m, S.D, nzD, false, sp, tid);  // (D unread if all zero)
     if (tid == 0) trace_stamp(a, t, 5);
     // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
-    const uint64_t t0 = t * kTileWords;
     bool bad = !ok;
     if (ok && nzD) {  // (no distances: x = V as it stands)
-      bar_d();  // S.V complete (V's DIFFMS⁻¹ ends without a barrier)
+      bar_d();  // X complete (V's DIFFMS⁻¹ ends without a barrier)
       for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
         const uint32_t li = b + tid;
         int32_t p = -1;
         uint64_t val = 0;
         if (li < m) {
-          const uint64_t d = S.D[li], gi = t0 + li;
+          const uint64_t d = Dw[li], gi = t0 + li;
           if (d == 0) {
-            val = S.V[li];
-          } else if (d > gi || S.V[li] != 0) {
+            val = S.X[li];
+          } else if (d > gi || S.X[li] != 0) {
             bad = true;
           } else if (gi - d >= t0 + b) {
             p = (int32_t)(gi - d - t0 - b);  // inside this block: resolve below
           } else if (gi - d >= t0) {
-            val = S.V[gi - d - t0];  // earlier block of this tile: already final
+            val = S.X[gi - d - t0];  // earlier block of this tile: already final
           } else {  // earlier tile: wait for its completion flag, then read the output
             const uint64_t j = gi - d, tj = j / kTileWords;
             while (ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
@@ -959,37 +1004,38 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
         }
         // pointer jumping inside the block (≤ 8 rounds; chains point backwards)
         uint32_t par = 0;
-        S.pj[0][tid] = p;
-        S.vj[0][tid] = val;
+        F.pj[0][tid] = p;
+        F.vj[0][tid] = val;
         while (bar_d_or(p >= 0)) {
           if (p >= 0) {
-            const int32_t q = S.pj[par][p];
+            const int32_t q = F.pj[par][p];
             if (q < 0) {
-              val = S.vj[par][p];
+              val = F.vj[par][p];
               p = -1;
             } else {
               p = q;
             }
           }
-          S.pj[par ^ 1][tid] = p;
-          S.vj[par ^ 1][tid] = val;
+          F.pj[par ^ 1][tid] = p;
+          F.vj[par ^ 1][tid] = val;
           par ^= 1;
         }
-        if (li < m) S.V[li] = val;  // x, in place
+        if (li < m) S.X[li] = val;  // x, in place
         bar_d();
       }
+      release(&S.empty_d[0]);
     }
     if (tid == 0) trace_stamp(a, t, 6);
-    fence_proxy_async_smem();  // S.V (generic-proxy writes) → the bulk store
+    fence_proxy_async_smem();  // S.X (generic-proxy writes) → the bulk store
     if (bar_d_or(bad)) {
       if (tid == 0) record_error(ctx, DERR_CORRUPT);
     } else if (m % 2 == 0) {
       if (tid == 0) {
-        tma_store_1d(out + t0, S.V, 8 * m);
+        tma_store_1d(out + t0, S.X, 8 * m);
         tma_store_commit();
       }
     } else {  // ragged last tile: thread stores
-      for (uint32_t i = tid; i < m; i += kDT) __stcs(out + t0 + i, S.V[i]);
+      for (uint32_t i = tid; i < m; i += kDT) __stcs(out + t0 + i, S.X[i]);
       __threadfence();
       bar_d();
     }
@@ -997,13 +1043,15 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   }
 }
 
-__global__ void __launch_bounds__(kDDecThreads) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DDecSmem& S = *reinterpret_cast<DDecSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
-    mbar_init(&S.full_in[0], 1);
-    mbar_init(&S.empty_in[0], kDW);
+    mbar_init(&S.full_v[0], 1);
+    mbar_init(&S.empty_v[0], kDW);
+    mbar_init(&S.full_d[0], 1);
+    mbar_init(&S.empty_d[0], kDW);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();

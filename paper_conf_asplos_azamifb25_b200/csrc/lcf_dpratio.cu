@@ -136,6 +136,9 @@ struct BitWriter {
 // bit runs. A plan takes two CTA barriers; everything after the second one
 // (the k choice, B2, B3, the section sizes) is computed redundantly by every
 // warp from shared data, so no warp waits on another's serial work.
+#ifndef LCF_ENC_MINB
+#define LCF_ENC_MINB 2
+#endif
 #ifndef LCF_HISTW
 #define LCF_HISTW 0
 #endif
@@ -541,7 +544,6 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
   uint32_t oit = 0;       // output-slot iteration (two chunks per tile)
   uint32_t par = 0;       // histogram parity
   uint32_t rz_used = 0;   // bytes of S.rz written by the last RAZE (re-zeroed by the next plan)
-  uint32_t sp = 0;        // cta_scan_u64 slot parity
   for (uint32_t it = 0;; ++it) {
     mbar_wait(&S.full_in[0], it & 1);
     const uint64_t t = S.in_chunk[0];
@@ -552,9 +554,10 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
     const uint32_t m = (uint32_t)umin64(kTileWords, a.n_words_total - t * kTileWords);
     // ---- FCM outputs (L170–185) and DIFFMS₆₄ (L187) of V in registers: words 8·tid … 8·tid+7 ----
     uint64_t w[8];
-    uint32_t d[8], dprev = 0, dor = 0;
+    uint32_t dprev = 0, dor = 0;
     {
       uint64_t x[8];
+      uint32_t d[8];
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const ulonglong2 xx = reinterpret_cast<const ulonglong2*>(S.xin)[4 * tid + q];
@@ -614,12 +617,14 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         if (lane == 0) mbar_arrive(&S.full_out[o]);
         continue;
       }
+      const uint32_t* gd = a.fcm_dist + t * kTileWords;  // (the stage is gone: distances from L2)
       if (part == 1) {  // DIFFMS₆₄ of the distances
         uint64_t pd = dprev;
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          w[j] = tcms((uint64_t)d[j] - pd);
-          pd = d[j];
+          const uint64_t dj = i0 + j < m ? (uint64_t)__ldcg(gd + i0 + j) : 0ull;
+          w[j] = tcms(dj - pd);
+          pd = dj;
         }
       }
       // ---- RAZE (L189) into S.rz ----
@@ -662,23 +667,12 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       }
       mbar_wait(&S.empty_out[o], pho ^ 1);  // (the storer hands slots back zeroed)
       if (tid == 0) trace_stamp(a, c, 3);
-      if (raw) {  // the V / Dist words themselves
+      if (raw) {  // the V / Dist words themselves, rebuilt from x and the distances (L2)
         uint64_t* ow = reinterpret_cast<uint64_t*>(ob);
-        if (part == 0) {  // V = DIFFMS⁻¹(w): serial run + CTA scan
-          uint64_t run = 0;
-#pragma unroll
-          for (uint32_t j = 0; j < 8; ++j) run += tcms_inv(w[j]);
-          uint64_t all;
-          uint64_t v = cta_scan_u64(run, S.scan, sp, tid, all);
-#pragma unroll
-          for (uint32_t j = 0; j < 8; ++j) {
-            v += tcms_inv(w[j]);
-            if (i0 + j < m) ow[i0 + j] = v;
-          }
-        } else {
-#pragma unroll
-          for (uint32_t j = 0; j < 8; ++j)
-            if (i0 + j < m) ow[i0 + j] = d[j];
+        const uint64_t* gx = reinterpret_cast<const uint64_t*>(a.in) + t * kTileWords;
+        for (uint32_t i = tid; i < m; i += kDT) {
+          const uint32_t di = __ldcg(gd + i);
+          ow[i] = part ? (uint64_t)di : (di ? 0ull : __ldcg(gx + i));
         }
         if (tid < 2 && (m & 1)) ow[m + tid] = 0;  // round16 pad
       } else if (P2.bypass) {
@@ -704,7 +698,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
   }
 }
 
-__global__ void __launch_bounds__(kDEncThreads, 2) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kDEncThreads, LCF_ENC_MINB) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

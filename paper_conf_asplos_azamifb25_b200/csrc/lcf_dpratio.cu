@@ -139,14 +139,14 @@ struct BitWriter {
 #ifndef LCF_ENC_MINB
 #define LCF_ENC_MINB 2
 #endif
-#ifndef LCF_HISTW
-#define LCF_HISTW 0
-#endif
 struct EncScratch {
   uint32_t hist[2][66];  // clz histograms, alternating per plan; [65]: the tile has an FCM distance
   uint32_t b1[64];       // B1 bitmap; byte t = thread t's words
   uint32_t wtot[kDW];    // set words per warp
 };
+
+// 0x00/0xFF bytes → 4 bits (byte j → bit j)
+__device__ __forceinline__ uint32_t bits4(uint32_t m) { return ((m & 0x01010101u) * 0x01020408u) >> 24; }
 
 struct APlan {
   uint32_t n, tl, k, byte, rank0, c1m, off1, nr1, b3, hib, total;
@@ -167,39 +167,16 @@ __device__ __forceinline__ APlan a_plan(const uint64_t (&v)[8], uint64_t p, uint
   P.tl = L % 8;
   const uint32_t n = P.n, i0 = 8 * tid;
   uint32_t* H = sc.hist[par];
-#if LCF_HISTW
-  {  // counts of z ∈ [b, b+6) (b = the warp's smallest z) are summed in packed
-     // 10-bit fields over the warp, one shared atomic per bin; others directly
-    uint32_t z[8], zmin = 65;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
-      z[j] = i0 + j < n ? clz64(v[j] ^ ref) : 65u;
-      zmin = min(zmin, z[j]);
-    }
-    const uint32_t b = __reduce_min_sync(0xFFFFFFFFu, zmin);
-    uint32_t pk0 = 0, pk1 = 0;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const uint32_t dz = z[j] - b;
-      if (dz < 3) pk0 += 1u << (10 * dz);
-      else if (dz < 6) pk1 += 1u << (10 * (dz - 3));
-      else if (z[j] <= 64) atomicAdd(&H[z[j]], 1u);
-    }
-    pk0 = __reduce_add_sync(0xFFFFFFFFu, pk0);
-    pk1 = __reduce_add_sync(0xFFFFFFFFu, pk1);
-    if (lane < 6) {
-      const uint32_t cnt = ((lane < 3 ? pk0 : pk1) >> (10 * (lane % 3))) & 1023u;
-      if (cnt && b + lane <= 64) atomicAdd(&H[b + lane], cnt);
-    }
-  }
-#else
+  // z_j = clz(v_j ⊕ ref_j) as bytes (0xFF past n): B1 bit j is [z_j < k] for
+  // RAZE (top(v) ≠ 0) and RARE (top(v_j) ≠ top(v_{j−1})) alike
+  uint32_t zpk[2] = {0u, 0u};
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
     const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
-    if (i0 + j < n) atomicAdd(&H[clz64(v[j] ^ ref)], 1u);
+    const uint32_t z = i0 + j < n ? clz64(v[j] ^ ref) : 0xFFu;
+    if (z <= 64) atomicAdd(&H[z], 1u);
+    zpk[j >> 2] |= z << (8 * (j & 3));
   }
-#endif
   if (__any_sync(0xFFFFFFFFu, dflag) && lane == 0) atomicOr(&H[65], 1u);
   if (tid < 66) sc.hist[par ^ 1][tid] = 0;  // read by the previous plan before a later barrier
   for (uint32_t j = tid; j < zn; j += kDT) zp[j] = make_uint4(0, 0, 0, 0);
@@ -229,12 +206,9 @@ __device__ __forceinline__ APlan a_plan(const uint64_t (&v)[8], uint64_t p, uint
   if (P.bypass) return P;
   const uint32_t k = P.k, sh = 64 - k;  // top(v) = v >> sh (k = 64: sh = 0)
   // ---- B1 byte t = this thread's set bits; ranks of the set words ----
-  uint32_t byte = 0;
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const uint64_t ref = RARE ? (j ? v[j - 1] : p) : 0ull;
-    if (i0 + j < n && (v[j] >> sh) != (ref >> sh)) byte |= 1u << j;
-  }
+  (void)sh;
+  const uint32_t kk = k * 0x01010101u;
+  const uint32_t byte = bits4(__vcmpltu4(zpk[0], kk)) | (bits4(__vcmpltu4(zpk[1], kk)) << 4);
   P.byte = byte;
   reinterpret_cast<uint8_t*>(sc.b1)[tid] = (uint8_t)byte;
   const uint32_t c = __popc(byte);
@@ -258,13 +232,9 @@ __device__ __forceinline__ APlan a_plan(const uint64_t (&v)[8], uint64_t p, uint
   const uint32_t L1 = (n + 7) / 8, L2 = (L1 + 7) / 8, L3 = (L2 + 7) / 8;
   const uint32_t b1w0 = sc.b1[2 * lane], b1w1 = sc.b1[2 * lane + 1];
   const uint32_t prevb = __shfl_up_sync(0xFFFFFFFFu, b1w1 >> 24, 1);
-  uint32_t c1m = 0;
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const uint32_t cur = ((j < 4 ? b1w0 : b1w1) >> (8 * (j & 3))) & 0xFF;
-    const uint32_t pre = j ? (((j - 1) < 4 ? b1w0 : b1w1) >> (8 * ((j - 1) & 3))) & 0xFF : (lane ? prevb : 0u);
-    if (cur != pre && 8 * lane + j < L1) c1m |= 1u << j;
-  }
+  const uint32_t pre0 = (b1w0 << 8) | (lane ? prevb : 0u), pre1 = (b1w1 << 8) | (b1w0 >> 24);
+  const uint32_t vb = 8 * lane >= L1 ? 0u : (L1 - 8 * lane >= 8 ? 0xFFu : (1u << (L1 - 8 * lane)) - 1u);
+  const uint32_t c1m = (bits4(__vcmpne4(b1w0, pre0)) | (bits4(__vcmpne4(b1w1, pre1)) << 4)) & vb;
   uint32_t y = __popc(c1m);
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {

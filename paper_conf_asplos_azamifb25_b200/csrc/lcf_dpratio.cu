@@ -309,19 +309,25 @@ __device__ __forceinline__ void a_emit_bypass_regs(const uint64_t (&v)[8], uint3
   }
 }
 
-// RARE bypass from shared memory: dst[0..3) = u16 L ‖ u8 0, dst[3 + j] = src[j],
-// one funnel shift per output word (whole words written; the last is masked).
+// RARE bypass from shared memory: dst[0..3) = u16 L ‖ u8 0, dst[3 + j] = src[j].
+// Four output words per thread per step (one 16-byte store, funnel shifts over
+// a 16-byte load and the word before it); words past the stream are 0.
 __device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t L, uint8_t* dst, uint32_t tid) {
   const uint32_t* sw = reinterpret_cast<const uint32_t*>(src);
-  uint32_t* dw = reinterpret_cast<uint32_t*>(dst);
-  const uint32_t nw = (L + 3 + 3) / 4;
-  for (uint32_t w = tid; w < nw; w += kDT) {
-    const uint32_t lo = w ? sw[w - 1] : 0u;
-    const uint32_t hi = 4 * w < L ? sw[w] : 0u;
-    uint32_t val = w ? __funnelshift_r(lo, hi, 8) : ((L & 0xFFFFu) | (hi << 24));
-    const uint32_t keep = 3 + L - 4 * w;  // bytes of this word inside the output
-    if (keep < 4) val &= (1u << (8 * keep)) - 1u;
-    dw[w] = val;
+  const uint32_t nw = (L + 3 + 3) / 4;  // output words
+  for (uint32_t g = tid; 4 * g < nw; g += kDT) {
+    const uint32_t w = 4 * g;
+    const uint4 q = reinterpret_cast<const uint4*>(src)[g];  // src words w .. w+3 (slack-safe)
+    const uint32_t pw = w ? sw[w - 1] : 0u;
+    uint32_t o[4] = {__funnelshift_r(pw, q.x, 8), __funnelshift_r(q.x, q.y, 8), __funnelshift_r(q.y, q.z, 8),
+                     __funnelshift_r(q.z, q.w, 8)};
+    if (w == 0) o[0] = (L & 0xFFFFu) | (q.x << 24);
+#pragma unroll
+    for (uint32_t i = 0; i < 4; ++i) {
+      const uint32_t keep = w + i < nw ? 3 + L - 4 * (w + i) : 0;  // bytes of this word inside the output
+      if (keep < 4) o[i] &= keep ? (1u << (8 * keep)) - 1u : 0u;
+    }
+    reinterpret_cast<uint4*>(dst)[g] = make_uint4(o[0], o[1], o[2], o[3]);
   }
 }
 

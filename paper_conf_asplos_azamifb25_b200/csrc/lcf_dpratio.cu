@@ -573,26 +573,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       const uint32_t o = oit % kDOut, pho = (oit / kDOut) & 1;
       uint8_t* ob = reinterpret_cast<uint8_t*>(S.out[o]);
       const bool cacheable = part == 1 && dist_zero && m == kTileWords;
-      if (cacheable && S.zlen) {  // the fixed stream of an all-zero Dist chunk, made once per CTA
-        const uint32_t len = S.zlen;
-        if (tid == 0) {
-          lookback_publish(ctx, c, round16(len));
-          trace_stamp(a, c, 2);
-        }
-        mbar_wait(&S.empty_out[o], pho ^ 1);
-        if (tid < round16(len) / 4) S.out[o][tid] = reinterpret_cast<const uint32_t*>(S.zc)[tid];
-        if (tid == 0) {
-          S.out_chunk[o] = c;
-          S.out_len[o] = len;
-          S.out_raw[o] = 0;
-          trace_stamp(a, c, 3);
-        }
-        fence_proxy_async_smem();
-        bar_d();
-        if (tid == 0) trace_stamp(a, c, 4);
-        if (lane == 0) mbar_arrive(&S.full_out[o]);
-        continue;
-      }
+      if (cacheable && S.zlen) continue;  // written with the V chunk (below)
       const uint32_t* gd = a.fcm_dist + t * kTileWords;  // (the stage is gone: distances from L2)
       if (part == 1) {  // DIFFMS₆₄ of the distances
         uint64_t pd = dprev;
@@ -666,10 +647,29 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
         S.out_len[o] = len;
         S.out_raw[o] = raw;
       }
+      // the next chunk — this tile's Dist — is the all-zero chunk whose stream
+      // this CTA already holds: it goes into the next slot now, under the same
+      // barrier (uniform: dist_zero and S.zlen are read after barriers)
+      const bool zd = part == 0 && dist_zero && m == kTileWords && S.zlen != 0;
+      const uint32_t o2 = (oit + 1) % kDOut, pho2 = ((oit + 1) / kDOut) & 1;
+      if (zd) {
+        const uint32_t zl = S.zlen;
+        if (tid == 0) lookback_publish(ctx, c + 1, round16(zl));
+        mbar_wait(&S.empty_out[o2], pho2 ^ 1);
+        if (tid < round16(zl) / 4) S.out[o2][tid] = reinterpret_cast<const uint32_t*>(S.zc)[tid];
+        if (tid == 0) {
+          S.out_chunk[o2] = c + 1;
+          S.out_len[o2] = zl;
+          S.out_raw[o2] = 0;
+        }
+      }
       fence_proxy_async_smem();
       bar_d();
       if (tid == 0) trace_stamp(a, c, 4);
-      if (lane == 0) mbar_arrive(&S.full_out[o]);
+      if (lane == 0) {
+        mbar_arrive(&S.full_out[o]);
+        if (zd) mbar_arrive(&S.full_out[o2]);
+      }
     }
   }
 }

@@ -153,6 +153,29 @@ def test_dpratio_mixed_match_tiles(L, orc):
     check_parity(L, orc, "DPratio", x, "mixed_match_tiles")
 
 
+def test_dpratio_raw_tiles_with_matches(L, orc):
+    """Random-bit tiles (V and Dist chunks stored raw) that still carry FCM
+    matches: copied 16-word runs from random earlier positions, copies of
+    copies (chains across tiles), and a ragged last tile. Exercises the
+    decoder's raw-V + FCM path and cross-tile chain resolution."""
+    if "DPratio" not in algos_available(L):
+        pytest.skip("DPratio not built")
+    rng = np.random.default_rng(11)
+    T = 2048
+    x = rng.integers(0, 2**63, size=12 * T + 333, dtype=np.uint64)
+    for t in range(2, 13):
+        run = 16 if t % 2 else 6  # even tiles: two short runs only, so V stays incompressible (raw)
+        for _ in range(40 if t % 2 else 2):
+            i = t * T + int(rng.integers(0, T - run))
+            if i + run > len(x):
+                continue
+            j = int(rng.integers(0, i - run))
+            x[i:i + run] = x[j:j + run]
+    _, table, _ = fmt_ref.parse_stream(orc.compress("DPratio", x))
+    assert any(e >> 31 for e in table[::2]), "expected raw V chunks"
+    check_parity(L, orc, "DPratio", x, "raw_tiles_with_matches")
+
+
 def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
     """Full-size check: GPU stream vs oracle on a sample of chunks (compress_chunks)."""
     s = L.compress(algo, x_dev)

@@ -126,6 +126,7 @@ struct RDecSmem {
   uint32_t len[kRDecStages], flags[kRDecStages];
   uint64_t sc64[2][kRW];
   uint32_t sc32[3][kRW];
+  uint32_t xsel[16];  // __byte_perm selectors: byte j ← source byte #(set bits of m below j) if bit j of m, else 0
   int32_t s2, bad;
 };
 
@@ -473,14 +474,23 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
       bar_r();  // keep the barrier count of every compute warp in step
       continue;
     }
+    // expand: word wi of the unit takes popc(m) bytes from nz(D) at p
+    // (one unaligned 4-byte read = two words + a funnel shift) and spreads them
+    // to its set byte positions with one byte permute (S.xsel[m])
+    const uint32_t* in32 = reinterpret_cast<const uint32_t*>(in);
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
       const uint32_t u = g + kRT * k;
       if (u >= NU) continue;
-      uint32_t wv[4] = {0, 0, 0, 0}, p = koff[k];
+      uint32_t wv[4], p = koff[k];
 #pragma unroll
-      for (int b = 0; b < 16; ++b)
-        if ((ub[k] >> b) & 1) wv[b >> 2] |= (uint32_t)in[p++] << (8 * (b & 3));
+      for (int wi = 0; wi < 4; ++wi) {
+        const uint32_t m = (ub[k] >> (4 * wi)) & 0xFu;
+        const uint32_t q = p >> 2;
+        const uint32_t src = __funnelshift_r(in32[q], in32[q + 1], 8 * (p & 3));
+        wv[wi] = __byte_perm(src, 0u, S.xsel[m]);
+        p += __popc(m);
+      }
       reinterpret_cast<uint4*>(S.T)[u] = make_uint4(wv[0], wv[1], wv[2], wv[3]);
     }
     __syncwarp();
@@ -538,6 +548,15 @@ __global__ void __launch_bounds__(kRDecThreads) spratio_decode_kernel(DecArgs a,
   extern __shared__ __align__(128) uint8_t smem_raw[];
   RDecSmem& S = *reinterpret_cast<RDecSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < 16) {
+    const uint32_t m = threadIdx.x;
+    uint32_t sel = 0, c = 0;
+    for (int j = 0; j < 4; ++j) {
+      sel |= (((m >> j) & 1u) ? c : 4u) << (4 * j);
+      c += (m >> j) & 1u;
+    }
+    S.xsel[m] = sel;
+  }
   if (threadIdx.x == 0) {
     for (int i = 0; i < kRDecStages; ++i) {
       mbar_init(&S.full_in[i], 1);

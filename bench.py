@@ -145,8 +145,9 @@ def kernel_traffic():
 
 
 def kernel_bytes(j):
-    """Algorithmic bytes per launch of every kernel a job's compress and
-    decompress launch: the I/O the method itself must move."""
+    """Algorithmic bytes of every kernel a job's compress and decompress
+    launch, summed over the job's launches of that kernel (DESIGN.md §6 gives
+    the per-launch figures): the I/O the method itself must move."""
     n, sb, codec = j["nbytes"], j["sbytes"], j["codec"]
     words = n // (4 if codec.startswith("SP") else 8)
     io = n + sb
@@ -157,9 +158,10 @@ def kernel_bytes(j):
     if codec == "SPratio":
         return {"spratio_encode": io, "spratio_decode": io}
     tiles = -(-words // 16384)
-    return {"fcm_sort_hist": 8 * words,               # x (pass 1) or pass-1 records (pass 2) in
-            "fcm_sort_scan": 8 * 1024 * tiles,        # the tile × digit count matrix, read and rewritten
-            "fcm_sort_scatter": 16 * words,           # 8-byte records (or x) in, records out
+    # the sort kernels launch once per radix pass (two passes per job)
+    return {"fcm_sort_hist": 2 * 8 * words,           # x (pass 1) or pass-1 records (pass 2) in
+            "fcm_sort_scan": 2 * 8 * 1024 * tiles,    # the tile × digit count matrix, read and rewritten
+            "fcm_sort_scatter": 2 * 16 * words,       # 8-byte records (or x) in, records out
             "fcm_match": 8 * words,                   # sorted records in (x gathered, matches scattered)
             "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
             "dpratio_decode": sb + n}                 # stream in, x out

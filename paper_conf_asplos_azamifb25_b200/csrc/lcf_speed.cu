@@ -338,8 +338,15 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
   }
 }
 
+// (an explicit minimum of 1 block per SM makes ptxas allocate more registers
+// than the plain bound, which costs a CTA per SM)
+#ifdef LCF_ENC_MINB
+#define LCF_ENC_BOUNDS __launch_bounds__(kEncThreads, LCF_ENC_MINB)
+#else
+#define LCF_ENC_BOUNDS __launch_bounds__(kEncThreads)
+#endif
 template <typename U>
-__global__ void __launch_bounds__(kEncThreads) speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__global__ void LCF_ENC_BOUNDS speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   EncSmem& S = *reinterpret_cast<EncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -489,8 +496,13 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
   }
 }
 
+#ifdef LCF_DEC_MINB
+#define LCF_DEC_BOUNDS __launch_bounds__(kDecThreads, LCF_DEC_MINB)
+#else
+#define LCF_DEC_BOUNDS __launch_bounds__(kDecThreads)
+#endif
 template <typename U>
-__global__ void __launch_bounds__(kDecThreads) speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
+__global__ void LCF_DEC_BOUNDS speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DecSmem<U>& S = *reinterpret_cast<DecSmem<U>*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

@@ -35,7 +35,7 @@ constexpr int kRecHashShift = 44, kRecFpShift = 32;
 constexpr uint64_t kRecIdxMask = 0xFFFFFFFFull;
 constexpr uint32_t kNoDigit = kDigits;  // records past n
 constexpr int kMatchBlock = 256;
-constexpr int kScanWarps = 32, kScanBlocks = kDigits / 32;
+constexpr int kScanWarps = 32, kScanBlocks = kDigits / 8;  // 8 digits per CTA (sort_scan_kernel)
 
 __device__ __forceinline__ uint32_t rec_digit(uint64_t rec, int pass) {
   return pass == 0 ? (uint32_t)(rec >> kRecHashShift) & (kDigits - 1) : (uint32_t)(rec >> (kRecHashShift + kDigitBits));
@@ -141,25 +141,49 @@ __global__ void __launch_bounds__(kSortThreads) sort_hist_kernel(const uint64_t*
 }
 
 // counts[t][d] → exclusive prefix over tiles t of digit d; tot[d] = total.
+// A CTA owns kScanDig digits (one 32-byte sector of a count row); lane l
+// reads digit l mod kScanDig of tile t0 + 4k + l / kScanDig, so a warp covers
+// four consecutive rows per load and 128 CTAs share the matrix.
+constexpr int kScanDig = 8, kScanSub = 32 / kScanDig;
 __global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __restrict__ counts, uint32_t n_tiles,
                                                                    uint32_t* __restrict__ tot) {
   __shared__ uint32_t part[kScanWarps][32];
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t d = blockIdx.x * 32 + lane;
+  const uint32_t dl = lane % kScanDig, sub = lane / kScanDig;
+  const uint32_t d = blockIdx.x * kScanDig + dl;
   const uint32_t t0 = (uint32_t)((uint64_t)warp * n_tiles / kScanWarps);
   const uint32_t t1 = (uint32_t)((uint64_t)(warp + 1) * n_tiles / kScanWarps);
   uint32_t s = 0;
-  for (uint32_t t = t0; t < t1; ++t) s += counts[(uint64_t)t * kDigits + d];
+#pragma unroll 4
+  for (uint32_t t = t0 + sub; t < t1; t += kScanSub) s += counts[(uint64_t)t * kDigits + d];
+  // this digit's sum over the warp's rows: combine the kScanSub row phases
+#pragma unroll
+  for (int k = kScanDig; k < 32; k <<= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, k);
   part[warp][lane] = s;
   __syncthreads();
   uint32_t run = 0;
-  for (uint32_t w = 0; w < warp; ++w) run += part[w][lane];
-  if (warp == kScanWarps - 1) tot[d] = run + s;
-  for (uint32_t t = t0; t < t1; ++t) {
-    uint32_t* c = counts + (uint64_t)t * kDigits + d;
-    const uint32_t v = *c;
-    *c = run;
-    run += v;
+  for (uint32_t w = 0; w < warp; ++w) run += part[w][dl];
+  if (warp == kScanWarps - 1 && sub == 0) tot[d] = run + s;
+  constexpr int kB = 4;  // row groups loaded before any is rewritten
+  for (uint32_t t = t0; t < t1; t += kScanSub * kB) {
+    uint32_t v[kB];
+#pragma unroll
+    for (int b = 0; b < kB; ++b) {
+      const uint32_t tt = t + b * kScanSub + sub;
+      v[b] = tt < t1 ? counts[(uint64_t)tt * kDigits + d] : 0u;
+    }
+#pragma unroll
+    for (int b = 0; b < kB; ++b) {
+      const uint32_t tt = t + b * kScanSub + sub;
+      uint32_t incl = v[b];  // prefix over the kScanSub consecutive rows of this load
+#pragma unroll
+      for (int k = kScanDig; k < 32; k <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, k);
+        if ((int)lane >= k) incl += y;
+      }
+      if (tt < t1) counts[(uint64_t)tt * kDigits + d] = run + incl - v[b];
+      run += __shfl_sync(0xFFFFFFFFu, incl, 32 - kScanDig + dl);
+    }
   }
 }
 
@@ -195,6 +219,7 @@ struct ScatterSmem {
   uint32_t wcnt[kSW][kDigits / 2];  // packed u16 pair per word
   uint32_t run[kDigits];                   // next output position of each digit (tile-wide)
   uint32_t rstart[kDigits];                // round: first stage slot of each digit
+  uint32_t delta[kDigits];                 // round: output position − stage slot of each digit
   uint32_t rtot[kDigits / 2];              // round: packed digit totals
   uint32_t wsum[kSW];
   uint8_t tag[kSW][kDigits];        // per warp: last lane that claimed a digit
@@ -286,7 +311,10 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       }
       digit_scan(c, ex);  // (its barrier also publishes wcnt)
 #pragma unroll
-      for (int j = 0; j < 2 * kP; ++j) S.rstart[2 * kP * tid + j] = ex[j];
+      for (int j = 0; j < 2 * kP; ++j) {
+        S.rstart[2 * kP * tid + j] = ex[j];
+        S.delta[2 * kP * tid + j] = S.run[2 * kP * tid + j] - ex[j];
+      }
     }
     __syncthreads();
     // 3. ranks → stage
@@ -318,8 +346,7 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
     // 4. stage → dst, digit runs contiguous
     for (uint32_t j = tid; j < nr; j += kST) {
       const uint64_t v = S.stage[j];
-      const uint32_t d = rec_digit(v, PASS);
-      dst[S.run[d] + (j - S.rstart[d])] = v;
+      dst[S.delta[rec_digit(v, PASS)] + j] = v;
     }
     __syncthreads();
 #pragma unroll

@@ -176,6 +176,38 @@ def test_dpratio_raw_tiles_with_matches(L, orc):
     check_parity(L, orc, "DPratio", x, "raw_tiles_with_matches")
 
 
+def fcm_stress_input(n_const=300_000, seed=5):
+    """FCM inputs with long same-hash runs and matches at every candidate depth:
+      - a constant run: one hash for every position, every match at distance 1;
+      - period-50 random values: 50 hashes, each recurring every 50 positions
+        (matches at distance 50);
+      - one context (a, b, c) followed by a value cycling with period 3, 4 or 5:
+        the match is the 3rd or 4th same-hash candidate, or none (5 > 4, L174);
+      - noise between the blocks."""
+    rng = np.random.default_rng(seed)
+    parts = [np.full(n_const, 0x400921FB54442D18, dtype=np.uint64)]
+    per = rng.integers(0, 2**63, size=50, dtype=np.uint64)
+    parts.append(np.tile(per, 12_000))
+    ctx = rng.integers(0, 2**63, size=3, dtype=np.uint64)
+    for cyc in (3, 4, 5):
+        vals = rng.integers(0, 2**63, size=cyc, dtype=np.uint64)
+        blk = np.empty((20_000, 4), dtype=np.uint64)
+        blk[:, :3] = ctx
+        blk[:, 3] = vals[np.arange(20_000) % cyc]
+        parts.append(blk.reshape(-1))
+        parts.append(rng.integers(0, 2**63, size=5_000, dtype=np.uint64))
+    return np.concatenate(parts)
+
+
+def test_dpratio_fcm_long_hash_runs(L, orc):
+    """FCM distances over long same-hash runs (one hash for 300 K positions,
+    50 hashes recurring every 50 positions, matches at the 3rd/4th candidate
+    or beyond the window) — stream identical to the oracle's."""
+    if "DPratio" not in algos_available(L):
+        pytest.skip("DPratio not built")
+    check_parity(L, orc, "DPratio", fcm_stress_input(), "fcm_long_hash_runs")
+
+
 def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
     """Full-size check: GPU stream vs oracle on a sample of chunks (compress_chunks)."""
     s = L.compress(algo, x_dev)

@@ -95,7 +95,17 @@ lcf_status_t lcf_check_stream(void* stream);
 /* ---- host-buffer convenience (the end-to-end path) ----------------------
  * Same as lcf_compress / lcf_decompress but h_in and h_out are HOST buffers:
  * the library copies h_in to device scratch, runs the codec on `stream`, copies
- * the result back and synchronises. *out_bytes is always written. */
+ * the result back and synchronises. *out_bytes is always written.
+ * SPspeed, SPratio and DPspeed inputs larger than one slice (~1/8 of the input,
+ * 4..64 MiB; env LCF_HOST_SLICE_BYTES overrides) are pipelined: chunk
+ * encodings are context-free, so each slice is coded as its
+ * own sub-stream while the next slice's host→device copy and the previous
+ * slice's device→host copy run on two library-owned streams; the host stitches
+ * the same bytes lcf_compress writes (FORMAT.md). Pinned host buffers let the
+ * two copy directions overlap. compress: out_capacity must hold the stitched
+ * stream (BUFFER_TOO_SMALL otherwise; lcf_max_compressed_size always does).
+ * decompress: the header and size table are read on the host; any malformed
+ * slice reports CORRUPT_STREAM. DPratio (FCM spans the array, L170) is serial. */
 lcf_status_t lcf_compress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,
                                void* h_out, size_t out_capacity, size_t* out_bytes, void* stream);
 lcf_status_t lcf_decompress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,

@@ -3,10 +3,12 @@
 #include <lcf.h>
 
 #include <atomic>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
 #include <utility>
+#include <vector>
 
 #include "lcf_kernels.cuh"
 
@@ -31,6 +33,12 @@ struct Workspace {
   uint32_t epoch = 0, checked_epoch = 0;
   void* scratch[4] = {nullptr, nullptr, nullptr, nullptr};  // grown on demand
   size_t scratch_cap[4] = {0, 0, 0, 0};
+  // pipelined host path: copy streams, per-slice events, pinned staging
+  std::mutex host_mu;
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  std::vector<cudaEvent_t> ev;
+  uint8_t* hstage = nullptr;
+  size_t hstage_cap = 0;
 };
 
 std::mutex g_mu;
@@ -359,6 +367,182 @@ lcf_status_t lcf_check_stream(void* stream_) {
   return st;
 }
 
+// ---- pipelined host path (chunk-local codecs) -------------------------------
+// The input is cut into slices of whole chunks. Chunk encodings are
+// context-free (L104), so slice i compressed on its own is an LCF1 sub-stream
+// whose table entries and padded payloads are exactly those of chunks
+// [c0, c1) of the whole stream; the host stitches header ‖ table slices ‖
+// payload slices (FORMAT.md) — the same bytes lcf_compress writes. The H2D of
+// slice i+1, the codec on slice i and the D2H of slice i−1 run on three
+// streams, so the two PCIe directions overlap each other and the kernels.
+// Decompression mirrors it: per slice, a sub-header and table slice built on
+// the host go up with the slice's payload bytes; the decoded words come back
+// while later slices decode. DPratio is not chunk-local (FCM, L170) and keeps
+// the serial path.
+static uint64_t host_slice_chunks(uint64_t C) {
+  uint64_t want = 0;
+  if (const char* e = std::getenv("LCF_HOST_SLICE_BYTES")) want = std::strtoull(e, nullptr, 10) / kChunkBytes;
+  if (want == 0) {  // ~8 slices, 4..64 MiB each
+    want = (C + 7) / 8;
+    const uint64_t lo = (4ull << 20) / kChunkBytes, hi = (64ull << 20) / kChunkBytes;
+    want = want < lo ? lo : want > hi ? hi : want;
+  }
+  return want;
+}
+
+static lcf_status_t host_pipe_init(Workspace* ws, size_t n_events, size_t stage_bytes) {
+  if (!ws->h2d && (!cuda_ok(cudaStreamCreateWithFlags(&ws->h2d, cudaStreamNonBlocking)) ||
+                   !cuda_ok(cudaStreamCreateWithFlags(&ws->d2h, cudaStreamNonBlocking))))
+    return LCF_ERROR_CUDA;
+  while (ws->ev.size() < n_events) {
+    cudaEvent_t e;
+    if (!cuda_ok(cudaEventCreateWithFlags(&e, cudaEventDisableTiming))) return LCF_ERROR_CUDA;
+    ws->ev.push_back(e);
+  }
+  if (ws->hstage_cap < stage_bytes) {
+    if (ws->hstage) cudaFreeHost(ws->hstage);
+    ws->hstage = nullptr;
+    ws->hstage_cap = 0;
+    if (!cuda_ok(cudaMallocHost(&ws->hstage, stage_bytes))) return LCF_ERROR_OUT_OF_MEMORY;
+    ws->hstage_cap = stage_bytes;
+  }
+  return LCF_SUCCESS;
+}
+
+static void put_header(uint8_t* h, int algo, uint64_t n_bytes, uint64_t n_chunks, uint64_t payload) {
+  const uint32_t w0 = kMagic, w1 = kVersion | ((uint32_t)algo << 8) | (word_bytes_of(algo) << 16);
+  std::memcpy(h, &w0, 4);
+  std::memcpy(h + 4, &w1, 4);
+  std::memcpy(h + 8, &n_bytes, 8);
+  std::memcpy(h + 16, &n_chunks, 8);
+  std::memcpy(h + 24, &payload, 8);
+}
+
+static lcf_status_t compress_host_pipelined(lcf_algo_t algo, lcf_dtype_t dtype, const uint8_t* h_in, size_t in_bytes,
+                                     uint8_t* h_out, size_t out_capacity, size_t* out_bytes, Workspace* ws,
+                                     uint64_t C, uint64_t sc) {
+  const uint64_t k = (C + sc - 1) / sc;
+  const uint64_t base = round16(kHeaderBytes + 4 * C);
+  if (out_capacity < base) return LCF_ERROR_BUFFER_TOO_SMALL;
+  const size_t sub_cap = lcf_max_compressed_size(algo, dtype, sc * kChunkBytes);
+  lcf_status_t st;
+  if ((st = host_pipe_init(ws, 2 * k, 32 * k))) return st;
+  {
+    std::lock_guard<std::mutex> g(ws->mu);
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[0]), ws->scratch_cap[0], round16(in_bytes) + 16,
+                   ws->stream, false)) ||
+        (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[1]), ws->scratch_cap[1], k * sub_cap, ws->stream, false)))
+      return st;
+  }
+  uint8_t* d_in = static_cast<uint8_t*>(ws->scratch[0]);
+  uint8_t* d_sub = static_cast<uint8_t*>(ws->scratch[1]);
+  cudaEvent_t* evH = ws->ev.data();
+  cudaEvent_t* evC = ws->ev.data() + k;
+  uint64_t off = base;  // next payload byte of the stitched stream
+  auto finish = [&](uint64_t i) -> lcf_status_t {
+    const uint64_t c0 = i * sc, kc = (c0 + sc < C ? sc : C - c0);
+    const uint64_t sbase = round16(kHeaderBytes + 4 * kc);
+    if (!cuda_ok(cudaEventSynchronize(evC[i]))) return LCF_ERROR_CUDA;
+    uint64_t pay;
+    std::memcpy(&pay, ws->hstage + 32 * i + 24, 8);
+    if (off + pay > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+    const uint8_t* sub = d_sub + i * sub_cap;
+    if (!cuda_ok(cudaStreamWaitEvent(ws->d2h, evC[i], 0)) ||
+        !cuda_ok(cudaMemcpyAsync(h_out + kHeaderBytes + 4 * c0, sub + kHeaderBytes, 4 * kc, cudaMemcpyDeviceToHost,
+                                 ws->d2h)) ||
+        (pay && !cuda_ok(cudaMemcpyAsync(h_out + off, sub + sbase, pay, cudaMemcpyDeviceToHost, ws->d2h))))
+      return LCF_ERROR_CUDA;
+    off += pay;
+    return LCF_SUCCESS;
+  };
+  for (uint64_t i = 0; i < k; ++i) {
+    const uint64_t b0 = i * sc * kChunkBytes;
+    const uint64_t bytes = (b0 + sc * kChunkBytes < in_bytes ? sc * kChunkBytes : in_bytes - b0);
+    if (!cuda_ok(cudaMemcpyAsync(d_in + b0, h_in + b0, bytes, cudaMemcpyHostToDevice, ws->h2d)) ||
+        !cuda_ok(cudaEventRecord(evH[i], ws->h2d)) || !cuda_ok(cudaStreamWaitEvent(ws->stream, evH[i], 0)))
+      return LCF_ERROR_CUDA;
+    uint8_t* sub = d_sub + i * sub_cap;
+    if ((st = lcf_compress(algo, dtype, d_in + b0, bytes, sub, sub_cap, nullptr, ws->stream))) return st;
+    if (!cuda_ok(cudaMemcpyAsync(ws->hstage + 32 * i, sub, 32, cudaMemcpyDeviceToHost, ws->stream)) ||
+        !cuda_ok(cudaEventRecord(evC[i], ws->stream)))
+      return LCF_ERROR_CUDA;
+    if (i >= 1 && (st = finish(i - 1))) return st;
+  }
+  if ((st = finish(k - 1))) return st;
+  put_header(h_out, algo, in_bytes, C, off - base);
+  std::memset(h_out + kHeaderBytes + 4 * C, 0, base - kHeaderBytes - 4 * C);
+  if (!cuda_ok(cudaStreamSynchronize(ws->d2h))) return LCF_ERROR_CUDA;
+  *out_bytes = off;
+  return LCF_SUCCESS;
+}
+
+static lcf_status_t decompress_host_pipelined(lcf_algo_t algo, lcf_dtype_t dtype, const uint8_t* h_in, size_t in_bytes,
+                                       uint8_t* h_out, size_t out_capacity, size_t* out_bytes, Workspace* ws,
+                                       uint64_t n_bytes, uint64_t C, uint64_t payload, uint64_t sc) {
+  const uint64_t k = (C + sc - 1) / sc;
+  const uint64_t base = round16(kHeaderBytes + 4 * C);
+  const uint32_t* table = reinterpret_cast<const uint32_t*>(h_in + kHeaderBytes);
+  const uint64_t sub_hdr = round16(kHeaderBytes + 4 * sc);  // staging bytes per slice (sub-header + table + pad)
+  lcf_status_t st;
+  if ((st = host_pipe_init(ws, 2 * k, k * sub_hdr))) return st;
+  {
+    std::lock_guard<std::mutex> g(ws->mu);
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[0]), ws->scratch_cap[0],
+                   k * sub_hdr + round16(in_bytes) + 16 * k, ws->stream, false)) ||
+        (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[1]), ws->scratch_cap[1], round16(n_bytes) + 16,
+                   ws->stream, false)))
+      return st;
+  }
+  uint8_t* d_sub = static_cast<uint8_t*>(ws->scratch[0]);
+  uint8_t* d_out = static_cast<uint8_t*>(ws->scratch[1]);
+  cudaEvent_t* evH = ws->ev.data();
+  cudaEvent_t* evC = ws->ev.data() + k;
+  uint64_t off = 0, dpos = 0;  // payload offset in the stream; next free byte of d_sub
+  for (uint64_t i = 0; i < k; ++i) {
+    const uint64_t c0 = i * sc, kc = (c0 + sc < C ? sc : C - c0);
+    uint64_t pay = 0;
+    for (uint64_t c = c0; c < c0 + kc; ++c) pay += round16(table[c] & ~kRawFlag);
+    if (off + pay > payload) return LCF_ERROR_CORRUPT_STREAM;
+    const uint64_t b0 = c0 * kChunkBytes;
+    const uint64_t bytes = (b0 + kc * kChunkBytes < n_bytes ? kc * kChunkBytes : n_bytes - b0);
+    const uint64_t sbase = round16(kHeaderBytes + 4 * kc);
+    uint8_t* stg = ws->hstage + i * sub_hdr;
+    put_header(stg, algo, bytes, kc, pay);
+    std::memcpy(stg + kHeaderBytes, table + c0, 4 * kc);
+    std::memset(stg + kHeaderBytes + 4 * kc, 0, sbase - kHeaderBytes - 4 * kc);
+    uint8_t* sub = d_sub + dpos;
+    dpos += sbase + round16(pay);
+    if (!cuda_ok(cudaMemcpyAsync(sub, stg, sbase, cudaMemcpyHostToDevice, ws->h2d)) ||
+        (pay && !cuda_ok(cudaMemcpyAsync(sub + sbase, h_in + base + off, pay, cudaMemcpyHostToDevice, ws->h2d))) ||
+        !cuda_ok(cudaEventRecord(evH[i], ws->h2d)) || !cuda_ok(cudaStreamWaitEvent(ws->stream, evH[i], 0)))
+      return LCF_ERROR_CUDA;
+    if ((st = lcf_decompress(algo, dtype, sub, sbase + pay, d_out + b0, bytes, nullptr, ws->stream))) return st;
+    if (!cuda_ok(cudaEventRecord(evC[i], ws->stream)) || !cuda_ok(cudaStreamWaitEvent(ws->d2h, evC[i], 0)) ||
+        !cuda_ok(cudaMemcpyAsync(h_out + b0, d_out + b0, bytes, cudaMemcpyDeviceToHost, ws->d2h)))
+      return LCF_ERROR_CUDA;
+    off += pay;
+  }
+  if (off != payload) return LCF_ERROR_CORRUPT_STREAM;
+  if (!cuda_ok(cudaStreamSynchronize(ws->d2h))) return LCF_ERROR_CUDA;
+  if ((st = lcf_check_stream(ws->stream))) return st;  // any slice the device found malformed
+  (void)out_capacity;
+  *out_bytes = n_bytes;
+  return LCF_SUCCESS;
+}
+
+// A failed pipelined call still has copies and kernels in flight on the
+// caller's buffers: drain all three streams before reporting, and consume the
+// device error word (slices already enqueued may have flagged too — this call
+// reports one status, like every synchronising call).
+static lcf_status_t host_pipe_done(Workspace* ws, lcf_status_t st) {
+  if (st) {
+    cudaStreamSynchronize(ws->h2d);
+    cudaStreamSynchronize(ws->d2h);
+    lcf_check_stream(ws->stream);
+  }
+  return st;
+}
+
 static lcf_status_t host_roundtrip(bool compress, lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in,
                                    size_t in_bytes, void* h_out, size_t out_capacity, size_t* out_bytes,
                                    cudaStream_t stream) {
@@ -367,6 +551,26 @@ static lcf_status_t host_roundtrip(bool compress, lcf_algo_t algo, lcf_dtype_t d
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
+  if (algo != LCF_DPRATIO && dtype_matches(algo, dtype)) {  // pipelined slices (chunk-local codecs)
+    std::lock_guard<std::mutex> hg(ws->host_mu);
+    if (compress) {
+      const uint64_t C = lcf_num_chunks(algo, in_bytes);
+      const uint64_t sc = host_slice_chunks(C);
+      if (in_bytes % word_bytes_of(algo) == 0 && C > sc)
+        return host_pipe_done(ws, compress_host_pipelined(algo, dtype, static_cast<const uint8_t*>(h_in), in_bytes,
+                                                          static_cast<uint8_t*>(h_out), out_capacity, out_bytes,
+                                                          ws, C, sc));
+    } else if (in_bytes >= kHeaderBytes) {
+      uint64_t nb, C, pay;
+      if (lcf_status_t s = check_header(static_cast<const uint8_t*>(h_in), in_bytes, algo, &nb, &C, &pay)) return s;
+      if (nb > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+      const uint64_t sc = host_slice_chunks(C);
+      if (C > sc)
+        return host_pipe_done(ws, decompress_host_pipelined(algo, dtype, static_cast<const uint8_t*>(h_in),
+                                                            in_bytes, static_cast<uint8_t*>(h_out), out_capacity,
+                                                            out_bytes, ws, nb, C, pay, sc));
+    }
+  }
   size_t dcap;
   if (compress) {
     dcap = lcf_max_compressed_size(algo, dtype, in_bytes);

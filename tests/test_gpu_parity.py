@@ -327,6 +327,41 @@ def test_host_buffer_api(L, orc):
     assert m == words.nbytes and np.array_equal(back, words)
 
 
+@pytest.mark.parametrize("algo", ["SPspeed", "SPratio", "DPspeed"])
+def test_host_pipelined_slices(L, orc, algo, monkeypatch):
+    """The sliced host path (3-chunk slices: 14 slices and a ragged tail) writes
+    the oracle's stream, decodes it and the oracle's, and accepts/rejects
+    corrupted streams exactly as the oracle does."""
+    monkeypatch.setenv("LCF_HOST_SLICE_BYTES", str(3 * 16384))
+    dt = np.float32 if algo.startswith("SP") else np.float64
+    words = datagen.smooth_1d(40 * 16384 // np.dtype(dt).itemsize + 77, dt, seed=21).view(wdt(algo)).copy()
+    words[5000:9000] = words[100]  # a constant stretch (small MPLG widths / zero RZE bytes)
+    cap = L.lcf_max_compressed_size(algo, None, words.nbytes)
+    hout = np.zeros(cap, np.uint8)
+    n = L.lcf_compress_host(algo, None, words, words.nbytes, hout, cap)
+    ref = orc.compress(algo, words)
+    assert hout[:n].tobytes() == ref
+    back = np.zeros_like(words)
+    assert L.lcf_decompress_host(algo, None, hout, n, back, back.nbytes) == words.nbytes
+    assert np.array_equal(back, words)
+    with pytest.raises(L.LcfError) as e:  # the stitched stream must fit
+        L.lcf_compress_host(algo, None, words, words.nbytes, hout, n - 1)
+    assert e.value.status == 3
+    rng = np.random.default_rng(4)
+    for trial in range(40):
+        t = np.frombuffer(ref, np.uint8).copy()
+        pos = int(rng.integers(32, len(ref))) if trial % 4 else int(rng.integers(32, 32 + 4 * 41))
+        t[pos] ^= np.uint8(1 << int(rng.integers(0, 8)))
+        try:
+            L.lcf_decompress_host(algo, None, t, len(t), back, back.nbytes)
+            ok_gpu = True
+        except L.LcfError:
+            ok_gpu = False
+        assert ok_gpu == (orc.decompress_status(algo, t.tobytes()) == 0), (trial, pos)
+        if ok_gpu:
+            assert np.array_equal(back, orc.decompress(algo, t.tobytes()))
+
+
 def test_dtype_and_argument_errors(L):
     x = torch.zeros(100, dtype=torch.int32, device="cuda")
     o = torch.empty(10000, dtype=torch.uint8, device="cuda")

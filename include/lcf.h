@@ -105,7 +105,9 @@ lcf_status_t lcf_check_stream(void* stream);
  * two copy directions overlap. compress: out_capacity must hold the stitched
  * stream (BUFFER_TOO_SMALL otherwise; lcf_max_compressed_size always does).
  * decompress: the header and size table are read on the host; any malformed
- * slice reports CORRUPT_STREAM. DPratio (FCM spans the array, L170) is serial. */
+ * slice reports CORRUPT_STREAM. DPratio decompression streams by tile ranges
+ * (distances into earlier slices read their final output); DPratio
+ * compression is serial (FCM's sort needs the whole array, L172). */
 lcf_status_t lcf_compress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,
                                void* h_out, size_t out_capacity, size_t* out_bytes, void* stream);
 lcf_status_t lcf_decompress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,

@@ -530,6 +530,76 @@ static lcf_status_t decompress_host_pipelined(lcf_algo_t algo, lcf_dtype_t dtype
   return LCF_SUCCESS;
 }
 
+// DPratio decompression in tile ranges: the header and size table go up first,
+// then slice i's payload bytes; the tile-range decode of slice i (DecArgs
+// first_tile/end_tile/base_off) resolves FCM distances into earlier slices
+// from the output they already wrote (same stream, so final), and its tiles
+// come back while later slices go up and decode. Compression stays serial:
+// FCM's sort needs the whole array before anything is encoded (L172).
+static lcf_status_t decompress_host_dpratio_pipelined(const uint8_t* h_in, size_t in_bytes, uint8_t* h_out,
+                                                      size_t* out_bytes, Workspace* ws, uint64_t n_bytes,
+                                                      uint64_t C, uint64_t payload, uint64_t st_tiles) {
+  const uint64_t T = C / 2, k = (T + st_tiles - 1) / st_tiles;
+  const uint64_t base = round16(kHeaderBytes + 4 * C);
+  const uint32_t* table = reinterpret_cast<const uint32_t*>(h_in + kHeaderBytes);
+  lcf_status_t st;
+  if ((st = host_pipe_init(ws, 2 * k, 16))) return st;
+  {
+    std::lock_guard<std::mutex> g(ws->mu);
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[0]), ws->scratch_cap[0], round16(in_bytes) + 16,
+                   ws->stream, false)) ||
+        (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[1]), ws->scratch_cap[1], round16(n_bytes) + 16,
+                   ws->stream, false)) ||
+        (st = grow(ws->status, ws->status_cap, C, ws->stream, true)) ||
+        (st = grow(ws->tile_flag, ws->tile_cap, T + 1, ws->stream, true)))
+      return st;
+  }
+  uint8_t* d_in = static_cast<uint8_t*>(ws->scratch[0]);
+  uint8_t* d_out = static_cast<uint8_t*>(ws->scratch[1]);
+  cudaEvent_t* evH = ws->ev.data();
+  cudaEvent_t* evC = ws->ev.data() + k;
+  if (!cuda_ok(cudaMemcpyAsync(d_in, h_in, base, cudaMemcpyHostToDevice, ws->h2d))) return LCF_ERROR_CUDA;
+  uint64_t off = 0;
+  for (uint64_t i = 0; i < k; ++i) {
+    const uint64_t t0 = i * st_tiles, t1 = (t0 + st_tiles < T ? t0 + st_tiles : T);
+    uint64_t pay = 0;
+    for (uint64_t c = 2 * t0; c < 2 * t1; ++c) pay += round16(table[c] & ~kRawFlag);
+    if (off + pay > payload) return LCF_ERROR_CORRUPT_STREAM;
+    if ((pay && !cuda_ok(cudaMemcpyAsync(d_in + base + off, h_in + base + off, pay, cudaMemcpyHostToDevice,
+                                         ws->h2d))) ||
+        !cuda_ok(cudaEventRecord(evH[i], ws->h2d)) || !cuda_ok(cudaStreamWaitEvent(ws->stream, evH[i], 0)))
+      return LCF_ERROR_CUDA;
+    {
+      std::lock_guard<std::mutex> g(ws->mu);
+      DecArgs a{};
+      a.stream = d_in;
+      a.stream_bytes = in_bytes;
+      a.out = d_out;
+      a.out_capacity = n_bytes;
+      a.algo = LCF_DPRATIO;
+      a.word_bytes = 8;
+      a.tile_flag = ws->tile_flag;
+      a.first_tile = t0;
+      a.end_tile = t1;
+      a.base_off = off;
+      LaunchCtx ctx = make_ctx(ws);
+      launch_dpratio_decode(a, ctx, t1 - t0, ws->stream);
+      ++g_launches;
+      if ((st = last_launch_status())) return st;
+    }
+    const uint64_t b0 = t0 * 2048 * 8, b1 = (t1 * 2048 * 8 < n_bytes ? t1 * 2048 * 8 : n_bytes);
+    if (!cuda_ok(cudaEventRecord(evC[i], ws->stream)) || !cuda_ok(cudaStreamWaitEvent(ws->d2h, evC[i], 0)) ||
+        !cuda_ok(cudaMemcpyAsync(h_out + b0, d_out + b0, b1 - b0, cudaMemcpyDeviceToHost, ws->d2h)))
+      return LCF_ERROR_CUDA;
+    off += pay;
+  }
+  if (off != payload) return LCF_ERROR_CORRUPT_STREAM;
+  if (!cuda_ok(cudaStreamSynchronize(ws->d2h))) return LCF_ERROR_CUDA;
+  if ((st = lcf_check_stream(ws->stream))) return st;
+  *out_bytes = n_bytes;
+  return LCF_SUCCESS;
+}
+
 // A failed pipelined call still has copies and kernels in flight on the
 // caller's buffers: drain all three streams before reporting, and consume the
 // device error word (slices already enqueued may have flagged too — this call
@@ -551,6 +621,17 @@ static lcf_status_t host_roundtrip(bool compress, lcf_algo_t algo, lcf_dtype_t d
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
+  if (algo == LCF_DPRATIO && dtype_matches(algo, dtype) && !compress && in_bytes >= kHeaderBytes) {
+    std::lock_guard<std::mutex> hg(ws->host_mu);
+    uint64_t nb, C, pay;
+    if (lcf_status_t s = check_header(static_cast<const uint8_t*>(h_in), in_bytes, algo, &nb, &C, &pay)) return s;
+    if (nb > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+    const uint64_t st_tiles = host_slice_chunks(C / 2);  // a tile decodes to one 16 KiB chunk of words
+    if (C / 2 > st_tiles)
+      return host_pipe_done(ws, decompress_host_dpratio_pipelined(static_cast<const uint8_t*>(h_in), in_bytes,
+                                                                  static_cast<uint8_t*>(h_out), out_bytes, ws, nb,
+                                                                  C, pay, st_tiles));
+  }
   if (algo != LCF_DPRATIO && dtype_matches(algo, dtype)) {  // pipelined slices (chunk-local codecs)
     std::lock_guard<std::mutex> hg(ws->host_mu);
     if (compress) {

@@ -726,17 +726,17 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
   uint64_t n_words = 0, n_chunks = 0, base = 0, payload = 0;
   const bool hdr_ok = read_header(a, ctx, n_words, n_chunks, base, payload);
   const bool small = hdr_ok && n_words * 8 > a.out_capacity;
-  const uint64_t T = n_chunks / 2;
+  const uint64_t T = a.end_tile && a.end_tile < n_chunks / 2 ? a.end_tile : n_chunks / 2;
   uint32_t it = 0;
   for (;;) {
     uint64_t tb = 0;
     if (lane == 0) tb = atomicAdd(ctx.ticket, 1ull);
-    tb = __shfl_sync(0xFFFFFFFFu, tb, 0) * kDBatch;
+    tb = a.first_tile + __shfl_sync(0xFFFFFFFFu, tb, 0) * kDBatch;
     if (!hdr_ok || small || tb >= T) {
       mbar_wait(&S.empty_v[0], (it & 1) ^ 1);
       if (lane == 0) {
-        if (tb == 0 && !hdr_ok) record_error(ctx, DERR_CORRUPT);
-        if (tb == 0 && small) record_error(ctx, DERR_SMALL);
+        if (tb == a.first_tile && !hdr_ok) record_error(ctx, DERR_CORRUPT);
+        if (tb == a.first_tile && small) record_error(ctx, DERR_SMALL);
         S.tile[0] = kNoChunk;
         mbar_arrive(&S.full_v[0]);
         ticket_retire(ctx);
@@ -763,9 +763,11 @@ __device__ __forceinline__ void d_dec_loader(DDecSmem& S, const DecArgs& a, cons
       if ((int)lane >= d) x += y;
     }
     x -= agg;
-    const uint64_t base_b = lookback_warp(ctx, 2 * tb, __shfl_sync(0xFFFFFFFFu, agg, 0));
-    const uint64_t excl = base_b + x;
-    if (lane > 0 && lane < 2 * nb) st_relaxed_u64(ctx.status + c, make_status(kFlagInc, ctx.epoch, excl + agg));
+    // prefixes relative to the launch's first chunk; a.base_off makes them absolute
+    const uint64_t base_b = lookback_warp(ctx, 2 * tb, __shfl_sync(0xFFFFFFFFu, agg, 0), 2 * a.first_tile);
+    const uint64_t rel = base_b + x;
+    if (lane > 0 && lane < 2 * nb) st_relaxed_u64(ctx.status + c, make_status(kFlagInc, ctx.epoch, rel + agg));
+    const uint64_t excl = rel + a.base_off;
     const uint64_t end = excl + round16(len);
     if (lane < 2 * nb && !bad && (end > payload || (c == n_chunks - 1 && end != payload))) bad = true;
     for (uint32_t j = 0; j < nb; ++j, ++it) {
@@ -967,8 +969,8 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
           } else if (gi - d >= t0) {
             val = S.X[gi - d - t0];  // earlier block of this tile: already final
           } else {  // earlier tile: wait for its completion flag, then read the output
-            const uint64_t j = gi - d, tj = j / kTileWords;
-            while (ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
+            const uint64_t j = gi - d, tj = j / kTileWords;  // (tiles before first_tile: final already)
+            while (tj >= a.first_tile && ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
             val = ld_cg_u64(out + j);
           }
         }

@@ -86,9 +86,12 @@ __device__ __forceinline__ void lookback_publish(const LaunchCtx& ctx, uint64_t 
 #ifndef LCF_LB_SLEEP
 #define LCF_LB_SLEEP 64
 #endif
-__device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t c, uint64_t agg) {
+// c_min: the launch's first chunk (a tile-range decode, lcf_api.cu): chunks
+// below it belong to earlier launches and count as a zero inclusive prefix.
+__device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t c, uint64_t agg,
+                                                  uint64_t c_min = 0) {
   const unsigned lane = threadIdx.x & 31;
-  if (c == 0) return 0;
+  if (c == c_min) return 0;
   uint64_t excl = 0;
   int64_t pos = (int64_t)c - 1;
   while (true) {
@@ -98,7 +101,7 @@ __device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t
     unsigned need, bad;
     int first_incl;
     while (true) {
-      if (idx >= 0) {
+      if (idx >= (int64_t)c_min) {
         s = ld_relaxed_u64(ctx.status + idx);
         const uint32_t ep = (uint32_t)(s >> 40) & 0x3FFFFFu;
         valid = (s >> 62) != 0 && ep == ctx.epoch;
@@ -114,7 +117,7 @@ __device__ __forceinline__ uint64_t lookback_warp(const LaunchCtx& ctx, uint64_t
       if (!bad) break;
       __nanosleep(LCF_LB_SLEEP);
     }
-    uint64_t v = ((int)lane <= first_incl && idx >= 0) ? (s & ((1ull << 40) - 1)) : 0;
+    uint64_t v = ((int)lane <= first_incl && idx >= (int64_t)c_min) ? (s & ((1ull << 40) - 1)) : 0;
 #pragma unroll
     for (int d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, d);
     excl += v;

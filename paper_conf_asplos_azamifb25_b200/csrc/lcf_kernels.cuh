@@ -63,6 +63,11 @@ struct DecArgs {
   uint32_t algo, word_bytes;
   uint32_t* tile_flag;    // DPratio: per-tile completion (epoch) flags
   unsigned long long* trace;  // lcf__trace_decompress only: 8 globaltimer stamps per chunk / tile
+  // DPratio tile-range decode (pipelined host path): tiles [first_tile,
+  // end_tile) only (end_tile 0: all); base_off = payload offset of chunk
+  // 2·first_tile; earlier tiles are already final in `out` (an earlier launch
+  // on the same stream) and only their payload bytes may be absent.
+  uint64_t first_tile, end_tile, base_off;
 };
 
 struct DecChunk {

@@ -327,10 +327,11 @@ def test_host_buffer_api(L, orc):
     assert m == words.nbytes and np.array_equal(back, words)
 
 
-@pytest.mark.parametrize("algo", ["SPspeed", "SPratio", "DPspeed"])
+@pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_host_pipelined_slices(L, orc, algo, monkeypatch):
-    """The sliced host path (3-chunk slices: 14 slices and a ragged tail) writes
-    the oracle's stream, decodes it and the oracle's, and accepts/rejects
+    """The sliced host path (3-chunk slices: 14 slices and a ragged tail; for
+    DPratio 3-tile decode slices whose FCM distances reach into earlier slices)
+    writes the oracle's stream, decodes it and the oracle's, and accepts/rejects
     corrupted streams exactly as the oracle does."""
     monkeypatch.setenv("LCF_HOST_SLICE_BYTES", str(3 * 16384))
     dt = np.float32 if algo.startswith("SP") else np.float64

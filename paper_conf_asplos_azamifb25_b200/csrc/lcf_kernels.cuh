@@ -50,9 +50,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// Stamps are compiled in only with -DLCF_TRACE=1 (scripts/build_variants.sh):
+// the per-stamp test of a.trace cost ~2 % of the speed encoder's instructions.
+#ifndef LCF_TRACE
+#define LCF_TRACE 0
+#endif
 template <class Args>
 __device__ __forceinline__ void trace_stamp(const Args& a, uint64_t chunk, int k) {
-  if (a.trace) a.trace[chunk * 8 + k] = gtimer();
+  if (LCF_TRACE && a.trace) a.trace[chunk * 8 + k] = gtimer();
 }
 
 struct DecArgs {

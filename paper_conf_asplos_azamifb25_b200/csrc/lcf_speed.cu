@@ -443,12 +443,14 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
 #pragma unroll
       for (int j = 0; j < 4; ++j) U4[j] = __funnelshift_r(T[j], T[j + 1], r);
       split_string(U4, w, d[q]);
+      if (hq >> 7) {  // the TCMS retry (L114, rare): a second inverse; hq is warp-uniform
+#pragma unroll
+        for (int j = 0; j < K; ++j) d[q][j] = tcms_inv(d[q][j]);
+      }
       U tot = 0;
 #pragma unroll
       for (int j = 0; j < K; ++j) {
-        U u = d[q][j];
-        if (hq >> 7) u = tcms_inv(u);
-        d[q][j] = tcms_inv(u);
+        d[q][j] = tcms_inv(d[q][j]);
         tot += d[q][j];
       }
       lane_tot[q] = tot;

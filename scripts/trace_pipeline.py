@@ -1,6 +1,8 @@
 """Per-chunk pipeline trace of a speed-codec compress (globaltimer stamps from
 lcf__trace_compress): where does a chunk's latency go, and how busy is the
-pipeline over time?"""
+pipeline over time? The stamps exist only in a library built with
+-DLCF_TRACE=1 (e.g. `scripts/build_variants.sh` with that define, then
+LCF_LIB_PATH=build/variants/<name>.so)."""
 import argparse
 import ctypes
 import os

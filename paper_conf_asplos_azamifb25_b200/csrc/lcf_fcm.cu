@@ -396,10 +396,17 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
     } else {
       r[0] = r[1] = r[2] = r[3] = 0;
     }
+    // the high word of a record is h(20) | fp(12): equal hash ⇔ (a ^ b) >> 12 == 0,
+    // equal hash and fingerprint ⇔ a == b
+    uint32_t hw[4 + kMatchItems];
+#pragma unroll
+    for (int t = 0; t < 4 + kMatchItems; ++t) hw[t] = (uint32_t)(r[t] >> 32);
 #pragma unroll
     for (int j = 0; j < kMatchItems; ++j) {
       const uint64_t k = k0 + j;
       if (k >= n) break;
+      const uint32_t hk = hw[4 + j];
+      if (k == 0 || ((hw[3 + j] ^ hk) >> 12)) continue;  // the predecessor has another hash: no candidate
       const uint64_t rk = r[4 + j];
       const uint32_t i = (uint32_t)(rk & kRecIdxMask);
       uint32_t d = 0;
@@ -408,10 +415,10 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
 #pragma unroll
       for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
         if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
-        const uint64_t rb = r[4 + j - back];
-        if ((rb >> kRecHashShift) != (rk >> kRecHashShift)) break;  // left the hash's run
-        if ((rb >> kRecFpShift) == (rk >> kRecFpShift)) {           // same hash and fingerprint
-          const uint32_t jj = (uint32_t)(rb & kRecIdxMask);
+        const uint32_t hb = hw[4 + j - back];
+        if ((hb ^ hk) >> 12) break;  // left the hash's run
+        if (hb == hk) {              // same hash and fingerprint
+          const uint32_t jj = (uint32_t)(r[4 + j - back] & kRecIdxMask);
           if (!have) {
             xi = x[i];
             have = true;

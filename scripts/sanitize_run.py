@@ -32,3 +32,23 @@ s = lcf.compress("DPratio", x)
 assert torch.equal(lcf.decompress("DPratio", s), x)
 print("DPratio slab ok")
 torch.cuda.synchronize()
+# the sliced host-buffer path (3-chunk slices; DPratio: tile-range decodes)
+os.environ["LCF_HOST_SLICE_BYTES"] = str(3 * 16384)
+for algo in ("SPspeed", "SPratio", "DPspeed", "DPratio"):
+    W = 32 if algo.startswith("SP") else 64
+    dt = np.float32 if W == 32 else np.float64
+    words = datagen.smooth_1d(12 * 16384 // (W // 8) + 77, dt, seed=5).view(np.uint32 if W == 32 else np.uint64).copy()
+    words[3000:5000] = words[7]
+    cap = lcf.lcf_max_compressed_size(algo, None, words.nbytes)
+    hout = np.zeros(cap, np.uint8)
+    n = lcf.lcf_compress_host(algo, None, words, words.nbytes, hout, cap)
+    back = np.zeros_like(words)
+    lcf.lcf_decompress_host(algo, None, hout, n, back, back.nbytes)
+    assert np.array_equal(back, words), algo
+    hout[40] ^= 0x5A
+    try:
+        lcf.lcf_decompress_host(algo, None, hout, n, back, back.nbytes)
+    except lcf.LcfError:
+        pass
+    print(algo, "host slices ok")
+torch.cuda.synchronize()

@@ -313,6 +313,12 @@ def run_lcf(args):
         ms_step = float(tt.item())
         value = world * tot_bytes / ms_step / 1e6
 
+    transfer = None
+    if world > 1:
+        try:
+            transfer = run_transfer(jobs, rank, dev)
+        except Exception as e:  # a measurement extra: never fail the bench line for it
+            print(f"[bench] transfer measurement failed: {e!r}", file=sys.stderr)
     e2e = run_e2e(lcf, jobs, args) if rank == 0 else None
     cpu = run_cpu_baseline(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
     cpu_codec = run_cpu_codec(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
@@ -327,9 +333,56 @@ def run_lcf(args):
             "per_codec": per_codec, "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "cpu_codec": cpu_codec, "e2e": e2e,
             "gpu_launches": launches, "clocks": clk.summary(),
         }
+        if transfer is not None:
+            line["transfer"] = transfer
         print(json.dumps(line))
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def run_transfer(jobs, rank, dev, reps: int = 3):
+    """NEXT-3 (transfer.py): rank 0 → rank 1 over NCCL, the raw words
+    (dist.send) against the compressed sub-streams (send_compressed /
+    recv_compressed), per chunk-local job. GB/s = uncompressed bytes / time,
+    timed on the device (events on each rank's current stream), max over the
+    pair, median of `reps`."""
+    import statistics
+    import torch.distributed as dist
+    from paper_conf_asplos_azamifb25_b200 import transfer as tr
+    out = []
+    for j in jobs:
+        if j["codec"] == "DPratio":
+            continue
+        x = j["x"]
+        buf = torch.empty_like(x)
+        res = {}
+        for mode in ("raw", "compressed"):
+            ts = []
+            for _ in range(reps):
+                dist.barrier()
+                torch.cuda.synchronize()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                if rank == 0:
+                    if mode == "raw":
+                        dist.send(x, 1)
+                    else:
+                        tr.send_compressed(x, 1, j["codec"])
+                elif rank == 1:
+                    if mode == "raw":
+                        dist.recv(buf, 0)
+                    else:
+                        tr.recv_compressed(0, j["codec"], out=buf)
+                e1.record()
+                torch.cuda.synchronize()
+                t = torch.tensor([e0.elapsed_time(e1) if rank < 2 else 0.0], device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ts.append(float(t.item()))
+            res[mode] = j["nbytes"] / statistics.median(ts) / 1e6
+        out.append({"codec": j["codec"], "field": j["field"], "bytes": j["nbytes"], "raw_gbs": res["raw"],
+                    "compressed_gbs": res["compressed"], "ratio": j["nbytes"] / j["sbytes"]})
+    return {"pair": "rank 0 -> rank 1 (NCCL)", "timing": "device events, max over the pair, median of 3",
+            "jobs": out}
 
 
 def run_e2e(lcf, jobs, args):

@@ -363,6 +363,31 @@ def test_host_pipelined_slices(L, orc, algo, monkeypatch):
             assert np.array_equal(back, orc.decompress(algo, t.tobytes()))
 
 
+@pytest.mark.parametrize("algo", GPU_ALGOS)
+def test_transfer_gpu_slices(L, orc, algo):
+    """NEXT-3 slice coder on the B200: the sub-streams send_compressed puts on
+    the wire equal the CPU codec's, and decoding them slice by slice (the
+    receiver's path, loopback without a second GPU) restores the array."""
+    from paper_conf_asplos_azamifb25_b200 import transfer
+    dt = np.float32 if algo.startswith("SP") else np.float64
+    words = datagen.smooth_1d(20 * 16384 // np.dtype(dt).itemsize + 77, dt, seed=33).view(wdt(algo)).copy()
+    words[2000:6000] = words[9]
+    x = to_dev(words)
+    subs = transfer.substreams(x, algo, slice_bytes=3 * 16384)
+    ref = transfer.substreams(torch.from_numpy(words.view(np.int32 if dt == np.float32 else np.int64)), algo,
+                              codec=transfer.CpuCodec(), slice_bytes=3 * 16384)
+    assert [s.cpu().numpy().tobytes() for s in subs] == [r.numpy().tobytes() for r in ref]
+    out = torch.empty_like(x)
+    codec = transfer.GpuCodec()
+    wb = words.itemsize
+    bounds = list(transfer._slices(words.nbytes, wb, 3 * 16384 if algo != "DPratio" else transfer._whole(words.nbytes)))
+    assert len(bounds) == len(subs)
+    for (w0, w1), s in zip(bounds, subs):
+        codec.decompress_into(transfer._algo_id(algo), s, out[w0:w1])
+    codec.finish()
+    assert torch.equal(out, x)
+
+
 def test_dtype_and_argument_errors(L):
     x = torch.zeros(100, dtype=torch.int32, device="cuda")
     o = torch.empty(10000, dtype=torch.uint8, device="cuda")

@@ -240,6 +240,23 @@ def test_full_size_sampled_parity(L, orc, algo, config, field):
     torch.cuda.empty_cache()
 
 
+def test_full_size_dpratio_stream(L, orc):
+    """The bench's DPratio workload at full size (Miranda density, 256×384×384
+    f64, 37.7 M words: 2304 FCM sort tiles, 18,432 encode tiles): the whole GPU
+    stream equals the oracle's byte for byte (the oracle needs ~1 min), and it
+    decodes back."""
+    if "DPratio" not in algos_available(L):
+        pytest.skip("DPratio not built")
+    x = datagen.field("miranda_256x384x384_f64", "density", device="cuda").reshape(-1).view(torch.int64)
+    s = L.compress("DPratio", x)
+    ref = orc.compress("DPratio", x.cpu().numpy().view(np.uint64))
+    assert s.numel() == len(ref)
+    assert np.array_equal(s.cpu().numpy(), np.frombuffer(ref, np.uint8))
+    assert torch.equal(L.decompress("DPratio", s), x)
+    del x, s
+    torch.cuda.empty_cache()
+
+
 @pytest.mark.parametrize("algo", SPEED_ALGOS)
 def test_async_path_and_corruption(L, orc, algo):
     words = datagen.smooth_1d(3 * 4096 + 77, np.float32 if algo == "SPspeed" else np.float64, seed=3)

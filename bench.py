@@ -314,7 +314,7 @@ def run_lcf(args):
         value = world * tot_bytes / ms_step / 1e6
 
     transfer = None
-    if world > 1:
+    if world > 1 and args.transfer:
         try:
             transfer = run_transfer(jobs, rank, dev)
         except Exception as e:  # a measurement extra: never fail the bench line for it
@@ -530,6 +530,8 @@ def main():
     ap.add_argument("--impl", default="lcf", choices=["lcf", "reference"])
     ap.add_argument("--codecs", default=",".join(ALL_CODECS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--transfer", action="store_true",
+                    help="N >= 2: also time rank 0 -> rank 1 raw vs compressed NCCL transfer (transfer.py)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

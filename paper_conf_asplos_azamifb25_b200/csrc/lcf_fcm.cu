@@ -365,7 +365,10 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
 // stops at the first other hash. The 12 records a thread needs come from six
 // 16-byte loads (no shared memory, no barriers). The distance array is
 // pre-zeroed; only matches are scattered.
-constexpr int kMatchItems = 8;
+#ifndef LCF_MATCH_ITEMS
+#define LCF_MATCH_ITEMS 8
+#endif
+constexpr int kMatchItems = LCF_MATCH_ITEMS;
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint64_t* __restrict__ rec,
                                                                 uint32_t* __restrict__ dist) {

@@ -200,7 +200,8 @@ __global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __
 #define LCF_SCAT_WARPS 16
 #endif
 #ifndef LCF_SCAT_BATCH
-#define LCF_SCAT_BATCH 16  // 8192-record rounds, 1 CTA/SM: 2×639→2×618 us (8: 2 CTAs/SM; 32: spills)
+#define LCF_SCAT_BATCH 16  // 8192-record rounds, 1 CTA/SM: 2×639→2×618 us (8: 2 CTAs/SM; 32: spills;
+                           // 32 warps × 8: 2×624 us)
 #endif
 #ifndef LCF_SCAT_MINB
 #define LCF_SCAT_MINB 1
@@ -210,8 +211,10 @@ __global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __
 #endif
 constexpr int kSW = LCF_SCAT_WARPS, kST = kSW * 32, kSB = LCF_SCAT_BATCH;
 constexpr int kRound = kST * kSB;  // records per round
-constexpr int kP = kDigits / 2 / kST;  // digit pairs per thread
-static_assert(kP * 2 * kST == kDigits, "digit pairs divide over the threads");
+// digit pairs per owning thread; with 1024 threads only the first 512 own a pair
+constexpr int kP = kDigits / 2 / kST > 0 ? kDigits / 2 / kST : 1;
+constexpr int kOwners = kDigits / 2 / kP;
+static_assert(kP * 2 * kOwners == kDigits && kOwners <= kST, "digit pairs divide over the threads");
 constexpr int kRounds = kTile / kRound;
 static_assert(kRounds * kRound == kTile, "tile = whole rounds");
 struct ScatterSmem {
@@ -237,6 +240,7 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
   // Thread tid owns the kP digit pairs [kP·tid, kP·tid + kP), i.e. digits
   // [2kP·tid, 2kP·tid + 2kP). Block exclusive scan of per-digit values c[]
   // (in this thread's digit order) → ex[] (contains a __syncthreads).
+  const bool owner = tid < (uint32_t)kOwners;
   auto digit_scan = [&](const uint32_t (&c)[2 * kP], uint32_t (&ex)[2 * kP]) {
     uint32_t own = 0;
 #pragma unroll
@@ -260,11 +264,12 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
   {  // digit bases (exclusive scan of tot) + this tile's offsets
     uint32_t c[2 * kP], ex[2 * kP];
 #pragma unroll
-    for (int j = 0; j < 2 * kP; ++j) c[j] = tot[2 * kP * tid + j];
+    for (int j = 0; j < 2 * kP; ++j) c[j] = owner ? tot[2 * kP * tid + j] : 0u;
     digit_scan(c, ex);
     const uint32_t* o = offs + (uint64_t)blockIdx.x * kDigits;
+    if (owner)
 #pragma unroll
-    for (int j = 0; j < 2 * kP; ++j) S.run[2 * kP * tid + j] = ex[j] + o[2 * kP * tid + j];
+      for (int j = 0; j < 2 * kP; ++j) S.run[2 * kP * tid + j] = ex[j] + o[2 * kP * tid + j];
   }
   const uint64_t tile0 = (uint64_t)blockIdx.x * kTile;
   // the next round's loads are issued before this round's copy-out (step 4)
@@ -299,22 +304,25 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       for (int q = 0; q < kP; ++q) {
         const uint32_t pq = kP * tid + q;
         uint32_t tw = 0;
+        if (owner) {
 #pragma unroll
-        for (int w = 0; w < kSW; ++w) {
-          const uint32_t v = S.wcnt[w][pq];
-          S.wcnt[w][pq] = tw;
-          tw += v;
+          for (int w = 0; w < kSW; ++w) {
+            const uint32_t v = S.wcnt[w][pq];
+            S.wcnt[w][pq] = tw;
+            tw += v;
+          }
+          S.rtot[pq] = tw;
         }
-        S.rtot[pq] = tw;
         c[2 * q] = tw & 0xFFFFu;
         c[2 * q + 1] = tw >> 16;
       }
       digit_scan(c, ex);  // (its barrier also publishes wcnt)
+      if (owner)
 #pragma unroll
-      for (int j = 0; j < 2 * kP; ++j) {
-        S.rstart[2 * kP * tid + j] = ex[j];
-        S.delta[2 * kP * tid + j] = S.run[2 * kP * tid + j] - ex[j];
-      }
+        for (int j = 0; j < 2 * kP; ++j) {
+          S.rstart[2 * kP * tid + j] = ex[j];
+          S.delta[2 * kP * tid + j] = S.run[2 * kP * tid + j] - ex[j];
+        }
     }
     __syncthreads();
     // 3. ranks → stage
@@ -349,12 +357,13 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       dst[S.delta[rec_digit(v, PASS)] + j] = v;
     }
     __syncthreads();
+    if (owner)
 #pragma unroll
-    for (int q = 0; q < kP; ++q) {
-      const uint32_t pq = kP * tid + q, t2 = S.rtot[pq];
-      S.run[2 * pq] += t2 & 0xFFFFu;
-      S.run[2 * pq + 1] += t2 >> 16;
-    }
+      for (int q = 0; q < kP; ++q) {
+        const uint32_t pq = kP * tid + q, t2 = S.rtot[pq];
+        S.run[2 * pq] += t2 & 0xFFFFu;
+        S.run[2 * pq + 1] += t2 >> 16;
+      }
     // (the next round's first barrier orders these updates before step 4)
   }
 }

@@ -72,7 +72,10 @@ __device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
 // them from lanes l−1, l−2, l−3 (one 32-bit rotation shuffle each); lanes
 // 0..2 use the rotated values of the previous group. Pass 1 reads the
 // records of pass 0.
-constexpr int kBatch = 8;
+#ifndef LCF_HIST_BATCH
+#define LCF_HIST_BATCH 8  // 4: 2×70.0 us, 8: 2×71.2, 16: 2×85.6, 32: 2×82.9 (Miranda)
+#endif
+constexpr int kBatch = LCF_HIST_BATCH;  // records per lane per load batch (histogram kernel)
 template <int PASS, int B = kBatch>
 struct RecReader {
   const uint64_t* src;

@@ -137,6 +137,33 @@ uint64_t lcf_num_chunks(lcf_algo_t algo, size_t in_bytes);
 lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,
                               uint64_t total_payload_bytes, void* d_stream, void* stream);
 
+/* ---- sharded DPratio -----------------------------------
+ * FCM compares a word with the ≤ 4 nearest preceding words
+ * of the same hash anywhere before it (L174), so a shard of the array needs,
+ * per hash, the last ≤ 4 words before its first word. For shards of whole
+ * 2048-word tiles, in array order:
+ *  1. lcf_dpratio_shard_summary: the shard's summary — per hash, its last ≤ 4
+ *     words (global index, value); lcf_dpratio_summary_bytes() bytes, device;
+ *  2. the summaries are exchanged (e.g. an NCCL all-gather);
+ *  3. lcf_dpratio_merge_summaries: shard g's carry from the summaries of shards
+ *     0 … g−1, contiguous in shard order (count = g; count 0: an empty carry);
+ *  4. lcf_dpratio_compress_shard: the shard's 2 chunks per tile with that carry
+ *     (NULL for shard 0), written like lcf_compress_shard: size-table slice,
+ *     payload piece from offset 0, device u64 payload byte count.
+ * The pieces assemble with lcf_write_header into exactly the 1-GPU stream.
+ * d_x points at the shard's first word (global index first_word, a multiple
+ * of 2048); the min(3, first_word) words before it must be readable (the hash
+ * context of the shard's first words, L172). shard_bytes is a multiple of
+ * 16384 unless the shard ends the array. Errors as lcf_compress_shard. */
+size_t lcf_dpratio_summary_bytes(void);
+lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,
+                                       void* d_summary, void* stream);
+lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream);
+lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, size_t total_in_bytes,
+                                        uint64_t first_word, const void* d_carry, void* d_table_slice,
+                                        void* d_payload, size_t payload_capacity, uint64_t* d_payload_bytes,
+                                        void* stream);
+
 /* Number of kernel launches the library enqueued since the process started
  * (bench/test accounting). */
 uint64_t lcf_launch_count(void);

@@ -724,6 +724,77 @@ lcf_status_t lcf_compress_shard(lcf_algo_t algo, lcf_dtype_t dtype, const void* 
   return enqueue_encode(ws, a);
 }
 
+size_t lcf_dpratio_summary_bytes(void) { return fcm_carry_bytes(); }
+
+// Validation shared by the sharded DPratio calls: whole tiles, in range.
+static lcf_status_t dp_shard_args(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word) {
+  if (total_in_bytes % 8 || shard_bytes % 8 || first_word % 2048) return LCF_ERROR_INVALID_ARGUMENT;
+  if (total_in_bytes / 8 >= (1ull << 31)) return LCF_ERROR_INVALID_ARGUMENT;  // 32-bit FCM indices
+  if (first_word * 8 + shard_bytes > total_in_bytes) return LCF_ERROR_INVALID_ARGUMENT;
+  if (first_word * 8 + shard_bytes != total_in_bytes && shard_bytes % kChunkBytes) return LCF_ERROR_INVALID_ARGUMENT;
+  if (shard_bytes && (!d_x || (reinterpret_cast<uintptr_t>(d_x) & 15))) return LCF_ERROR_INVALID_ARGUMENT;
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,
+                                       void* d_summary, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (lcf_status_t s = dp_shard_args(d_x, shard_bytes, total_in_bytes, first_word)) return s;
+  if (!d_summary) return LCF_ERROR_INVALID_ARGUMENT;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  const uint64_t n = shard_bytes / 8;
+  if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[2]), ws->scratch_cap[2], dpratio_fcm_workspace(n), stream,
+                 false)))
+    return st;
+  uint32_t* dist = nullptr;
+  g_launches += launch_fcm_shard(static_cast<const uint64_t*>(d_x), n, (uint32_t)(first_word < 3 ? first_word : 3),
+                                 first_word, nullptr, d_summary, false, ws->scratch[2], ws->scratch_cap[2], stream,
+                                 &dist);
+  return last_launch_status();
+}
+
+lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!d_carry || (count && !d_summaries) || count > 0xFFFFFFFFull) return LCF_ERROR_INVALID_ARGUMENT;
+  g_launches += launch_fcm_carry_merge(d_summaries, (uint32_t)count, d_carry, stream);
+  return last_launch_status();
+}
+
+lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, size_t total_in_bytes,
+                                        uint64_t first_word, const void* d_carry, void* d_table_slice,
+                                        void* d_payload, size_t payload_capacity, uint64_t* d_payload_bytes,
+                                        void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (lcf_status_t s = dp_shard_args(d_x, shard_bytes, total_in_bytes, first_word)) return s;
+  if (!d_payload_bytes) return LCF_ERROR_INVALID_ARGUMENT;
+  const uint64_t n = shard_bytes / 8, tiles = (n + 2047) / 2048;
+  if (tiles && (!d_table_slice || !d_payload || !aligned16(d_payload))) return LCF_ERROR_INVALID_ARGUMENT;
+  if (payload_capacity < payload_bound(LCF_DPRATIO, shard_bytes)) return LCF_ERROR_BUFFER_TOO_SMALL;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  if (tiles == 0) return cuda_ok(cudaMemsetAsync(d_payload_bytes, 0, 8, stream)) ? LCF_SUCCESS : LCF_ERROR_CUDA;
+  EncArgs a = enc_args(LCF_DPRATIO, d_x, shard_bytes);  // the shard's words; tiles of the launch from 0
+  a.first_chunk = 2 * (first_word / 2048);
+  a.n_chunks = 2 * tiles;
+  a.stream_chunks = lcf_num_chunks(LCF_DPRATIO, total_in_bytes);
+  a.table = static_cast<uint32_t*>(d_table_slice);
+  a.payload = static_cast<uint8_t*>(d_payload);
+  a.count_out = d_payload_bytes;
+  if ((st = grow(ws->status, ws->status_cap, a.n_chunks, stream, true)) ||
+      (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[2]), ws->scratch_cap[2], dpratio_fcm_workspace(n), stream,
+                 false)))
+    return st;
+  LaunchCtx ctx = make_ctx(ws);
+  g_launches += launch_dpratio_encode(a, ctx, ws->scratch[2], ws->scratch_cap[2], stream,
+                                      (uint32_t)(first_word < 3 ? first_word : 3), first_word, d_carry);
+  return last_launch_status();
+}
+
 lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,
                               uint64_t total_payload_bytes, void* d_stream, void* stream_) {
   if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;

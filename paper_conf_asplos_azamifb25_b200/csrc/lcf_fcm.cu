@@ -82,11 +82,13 @@ struct RecReader {
   uint64_t n, i0;
   uint32_t r1p, r2p, r3p;  // previous group's rotated product words (pass 0)
   uint64_t v[B];
-  __device__ __forceinline__ RecReader(const uint64_t* s, uint64_t n_, uint64_t start, uint32_t lane)
+  // halo: words src[−halo … −1] precede the array (a shard's context, ≤ 3)
+  __device__ __forceinline__ RecReader(const uint64_t* s, uint64_t n_, uint64_t start, uint32_t lane,
+                                       uint32_t halo = 0)
       : src(s), n(n_), i0(start) {
     if (PASS == 0) {  // the group before `start`: only its lanes 29..31 matter
       const int64_t j = (int64_t)start - 32 + (int64_t)lane;
-      const uint64_t y = (lane >= 29 && j >= 0 && (uint64_t)j < n) ? src[j] : 0;
+      const uint64_t y = (lane >= 29 && j >= -(int64_t)halo && (j < 0 || (uint64_t)j < n)) ? src[j] : 0;
       rotate(y, lane, r1p, r2p, r3p);
     }
   }
@@ -121,13 +123,13 @@ struct RecReader {
 
 template <int PASS>
 __global__ void __launch_bounds__(kSortThreads) sort_hist_kernel(const uint64_t* __restrict__ src, uint64_t n,
-                                                                 uint32_t* __restrict__ counts) {
+                                                                 uint32_t* __restrict__ counts, uint32_t halo) {
   __shared__ uint32_t hist[kDigits];
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   for (uint32_t d = threadIdx.x; d < kDigits; d += kSortThreads) hist[d] = 0;
   __syncthreads();
   const uint64_t start = (uint64_t)blockIdx.x * kTile + warp * kWarpRecs;
-  RecReader<PASS> rd(src, n, start, lane);
+  RecReader<PASS> rd(src, n, start, lane, halo);
   for (int s = 0; s < kWarpRecs / (32 * kBatch); ++s, rd.advance()) {
     if (rd.i0 >= n) break;  // warp-uniform
     rd.load(lane);
@@ -235,7 +237,7 @@ template <int PASS>
 __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const uint64_t* __restrict__ src, uint64_t n,
                                                                     const uint32_t* __restrict__ offs,
                                                                     const uint32_t* __restrict__ tot,
-                                                                    uint64_t* __restrict__ dst) {
+                                                                    uint64_t* __restrict__ dst, uint32_t halo) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
   const uint32_t tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -276,14 +278,14 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
   }
   const uint64_t tile0 = (uint64_t)blockIdx.x * kTile;
   // the next round's loads are issued before this round's copy-out (step 4)
-  RecReader<PASS, kSB> rd(src, n, tile0 + warp * 32 * kSB, lane);
+  RecReader<PASS, kSB> rd(src, n, tile0 + warp * 32 * kSB, lane, halo);
   rd.load(lane);
   for (int r = 0; r < kRounds; ++r) {
     const uint64_t r0 = tile0 + (uint64_t)r * kRound;
     if (r0 >= n) break;  // block-uniform
     const uint32_t nr = (uint32_t)umin64(kRound, n - r0);
     if (!LCF_SCAT_PREFETCH && r > 0) {
-      rd = RecReader<PASS, kSB>(src, n, r0 + warp * 32 * kSB, lane);
+      rd = RecReader<PASS, kSB>(src, n, r0 + warp * 32 * kSB, lane, halo);
       rd.load(lane);
     }
     // 1. this warp's records of the round and its digit counts
@@ -350,7 +352,7 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       __syncwarp();
     }
     if (LCF_SCAT_PREFETCH && r + 1 < kRounds) {
-      rd = RecReader<PASS, kSB>(src, n, r0 + kRound + warp * 32 * kSB, lane);
+      rd = RecReader<PASS, kSB>(src, n, r0 + kRound + warp * 32 * kSB, lane, halo);
       rd.load(lane);
     }
     __syncthreads();
@@ -381,9 +383,23 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
 #define LCF_MATCH_ITEMS 8
 #endif
 constexpr int kMatchItems = LCF_MATCH_ITEMS;
+// Sharded DPratio (NEXT-1): per hash, the last ≤ 4 records (nearest first) of
+// the words before this shard — global index and word — merged from the
+// lower shards' summaries. Candidates of a record are its local same-hash
+// predecessors first (nearer), then these (L174, A-14).
+struct FcmCarry {
+  const uint8_t* cnt;    // [2^20]
+  const uint32_t* idx;   // [2^20][4]
+  const uint64_t* val;   // [2^20][4]
+};
+constexpr uint64_t kHashes = 1ull << 20;
+__host__ __device__ constexpr size_t carry_bytes() { return kHashes * (1 + 4 * 4 + 4 * 8); }
+
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint64_t* __restrict__ rec,
-                                                                uint32_t* __restrict__ dist) {
+                                                                uint32_t* __restrict__ dist, FcmCarry carry,
+                                                                uint64_t gbase) {
+  const bool carry_on = carry.cnt != nullptr;
   const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
   for (uint64_t g = blockIdx.x * (uint64_t)kMatchBlock + threadIdx.x; g < groups;
        g += (uint64_t)gridDim.x * kMatchBlock) {
@@ -421,10 +437,11 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
       const uint64_t k = k0 + j;
       if (k >= n) break;
       const uint32_t hk = hw[4 + j];
-      if (k == 0 || ((hw[3 + j] ^ hk) >> 12)) continue;  // the predecessor has another hash: no candidate
+      const bool start = k == 0 || ((hw[3 + j] ^ hk) >> 12);  // first of its hash run here
+      if (start && !carry_on) continue;  // no candidate at all
       const uint64_t rk = r[4 + j];
       const uint32_t i = (uint32_t)(rk & kRecIdxMask);
-      uint32_t d = 0;
+      uint32_t d = 0, used = 0;
       uint64_t xi = 0;
       bool have = false;
 #pragma unroll
@@ -432,6 +449,7 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
         if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
         const uint32_t hb = hw[4 + j - back];
         if ((hb ^ hk) >> 12) break;  // left the hash's run
+        ++used;
         if (hb == hk) {              // same hash and fingerprint
           const uint32_t jj = (uint32_t)(r[4 + j - back] & kRecIdxMask);
           if (!have) {
@@ -444,9 +462,67 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
           }
         }
       }
+      if (carry_on && d == 0 && used < 4) {  // the remaining candidates precede the shard
+        const uint32_t h = hk >> 12, cc = carry.cnt[h];
+#pragma unroll
+        for (uint32_t q = 0; q < 4; ++q) {
+          if (q >= cc || q + used >= 4) break;
+          if (!have) {
+            xi = x[i];
+            have = true;
+          }
+          if (carry.val[4 * h + q] == xi) {
+            d = (uint32_t)(gbase + i - carry.idx[4 * h + q]);
+            break;
+          }
+        }
+      }
       if (d) dist[i] = d;
     }
   }
+}
+
+// Summary of a shard (sorted records rec[0, n)): per hash, the last ≤ 4
+// records of its run (nearest first) as global index and word.
+__global__ void __launch_bounds__(256) fcm_summary_kernel(const uint64_t* __restrict__ x, uint64_t n,
+                                                         const uint64_t* __restrict__ rec, uint64_t gbase,
+                                                         uint8_t* __restrict__ cnt, uint32_t* __restrict__ idx,
+                                                         uint64_t* __restrict__ val) {
+  for (uint64_t k = blockIdx.x * 256ull + threadIdx.x; k < n; k += (uint64_t)gridDim.x * 256) {
+    const uint64_t hk = rec[k] >> kRecHashShift;
+    if (k + 1 < n && (rec[k + 1] >> kRecHashShift) == hk) continue;  // not the end of the run
+    uint32_t c = 0;
+    for (uint32_t q = 0; q < 4 && q <= k; ++q) {
+      const uint64_t r = rec[k - q];
+      if ((r >> kRecHashShift) != hk) break;
+      const uint32_t i = (uint32_t)(r & kRecIdxMask);
+      idx[4 * hk + q] = (uint32_t)(gbase + i);
+      val[4 * hk + q] = x[i];
+      ++c;
+    }
+    cnt[hk] = (uint8_t)c;
+  }
+}
+
+// Carry of shard g: per hash, walk the summaries of shards g−1, g−2, … 0 and
+// keep the first four entries (most recent first).
+__global__ void __launch_bounds__(256) fcm_carry_merge_kernel(const uint8_t* __restrict__ sums, uint32_t count,
+                                                             uint8_t* __restrict__ out) {
+  const uint64_t h = blockIdx.x * 256ull + threadIdx.x;
+  if (h >= kHashes) return;
+  auto cnt_of = [&](const uint8_t* b) { return b; };
+  auto idx_of = [&](const uint8_t* b) { return reinterpret_cast<const uint32_t*>(b + kHashes); };
+  auto val_of = [&](const uint8_t* b) { return reinterpret_cast<const uint64_t*>(b + kHashes * 17); };
+  uint32_t m = 0;
+  for (int32_t r = (int32_t)count - 1; r >= 0 && m < 4; --r) {
+    const uint8_t* b = sums + (uint64_t)r * carry_bytes();
+    const uint32_t c = cnt_of(b)[h];
+    for (uint32_t q = 0; q < c && m < 4; ++q, ++m) {
+      reinterpret_cast<uint32_t*>(out + kHashes)[4 * h + m] = idx_of(b)[4 * h + q];
+      reinterpret_cast<uint64_t*>(out + kHashes * 17)[4 * h + m] = val_of(b)[4 * h + q];
+    }
+  }
+  out[h] = (uint8_t)m;
 }
 
 uint64_t n_tiles_of(uint64_t n) { return (n + kTile - 1) / kTile; }
@@ -457,7 +533,14 @@ size_t fcm_dist_workspace(uint64_t n) {
   return 2 * round16(8 * n) + round16(4 * n_tiles_of(n) * kDigits) + 4 * kDigits + 256;
 }
 
-int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
+size_t fcm_carry_bytes() { return carry_bytes(); }
+
+// The FCM distances of x[0, n) (sharded: a shard whose words x[−halo, 0)
+// precede it and whose first word has global index gbase; carry = the merged
+// summaries of the earlier shards, or null). summary (optional) receives this
+// shard's own summary; with match false only the summary is made.
+int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
   (void)ws_bytes;
   uint8_t* p = static_cast<uint8_t*>(ws);
   uint64_t* rec_a = reinterpret_cast<uint64_t*>(p);
@@ -467,16 +550,20 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   uint32_t* tot = reinterpret_cast<uint32_t*>(p + 2 * round16(8 * n) + round16(4 * T * kDigits));
   uint32_t* dist = reinterpret_cast<uint32_t*>(rec_a);  // pass-1 records are dead after pass 2
   *dist_out = dist;
-  if (n == 0) return 0;
+  if (n == 0) {
+    if (summary) cudaMemsetAsync(summary, 0, kHashes, st);  // no entries
+    return 0;
+  }
   static const bool init = [] {
     cudaFuncSetAttribute(sort_scatter_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScatterSmem));
     cudaFuncSetAttribute(sort_scatter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScatterSmem));
     return true;
   }();
   (void)init;
+  int launches = 6;
   {
     KTrace kt("fcm_sort_hist", st);
-    sort_hist_kernel<0><<<(unsigned)T, kSortThreads, 0, st>>>(x, n, counts);
+    sort_hist_kernel<0><<<(unsigned)T, kSortThreads, 0, st>>>(x, n, counts, halo);
   }
   {
     KTrace kt("fcm_sort_scan", st);
@@ -484,11 +571,11 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   }
   {
     KTrace kt("fcm_sort_scatter", st);
-    sort_scatter_kernel<0><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(x, n, counts, tot, rec_a);
+    sort_scatter_kernel<0><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(x, n, counts, tot, rec_a, halo);
   }
   {
     KTrace kt("fcm_sort_hist", st);
-    sort_hist_kernel<1><<<(unsigned)T, kSortThreads, 0, st>>>(rec_a, n, counts);
+    sort_hist_kernel<1><<<(unsigned)T, kSortThreads, 0, st>>>(rec_a, n, counts, 0);
   }
   {
     KTrace kt("fcm_sort_scan", st);
@@ -496,16 +583,41 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   }
   {
     KTrace kt("fcm_sort_scatter", st);
-    sort_scatter_kernel<1><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b);
+    sort_scatter_kernel<1><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b, 0);
   }
+  if (summary) {
+    uint8_t* sb = static_cast<uint8_t*>(summary);
+    cudaMemsetAsync(sb, 0, kHashes, st);
+    KTrace kt("fcm_summary", st);
+    fcm_summary_kernel<<<(unsigned)umin64((n + 255) / 256, 148 * 16), 256, 0, st>>>(
+        x, n, rec_b, gbase, sb, reinterpret_cast<uint32_t*>(sb + kHashes), reinterpret_cast<uint64_t*>(sb + 17 * kHashes));
+    ++launches;
+  }
+  if (!match) return launches;
   cudaMemsetAsync(dist, 0, 4 * n, st);
+  FcmCarry c{nullptr, nullptr, nullptr};
+  if (carry) {
+    const uint8_t* cb = static_cast<const uint8_t*>(carry);
+    c = FcmCarry{cb, reinterpret_cast<const uint32_t*>(cb + kHashes), reinterpret_cast<const uint64_t*>(cb + 17 * kHashes)};
+  }
   {
     KTrace kt("fcm_match", st);
     const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
     const int mblocks = (int)umin64((groups + kMatchBlock - 1) / kMatchBlock, 148 * 16);
-    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist);
+    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
   }
-  return 7;
+  return launches + 1;
+}
+
+int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
+  return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out);
+}
+
+int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st) {
+  KTrace kt("fcm_carry_merge", st);
+  fcm_carry_merge_kernel<<<(unsigned)(kHashes / 256), 256, 0, st>>>(static_cast<const uint8_t*>(summaries), count,
+                                                                    static_cast<uint8_t*>(carry));
+  return 1;
 }
 
 }  // namespace lcf

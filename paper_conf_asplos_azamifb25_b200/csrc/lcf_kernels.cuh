@@ -156,8 +156,17 @@ void launch_write_header(const EncArgs& a, cudaStream_t st);
 // (returns the number of kernels; *dist points into ws, n u32 values).
 size_t fcm_dist_workspace(uint64_t n_words);
 int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist);
+// Sharded DPratio (NEXT-1, lcf_fcm.cu): the same over a shard with `halo`
+// context words before x, global first index gbase, the merged summaries of
+// earlier shards (carry, nullable); `summary` (nullable) receives this
+// shard's summary (fcm_carry_bytes() bytes); match = false: summary only.
+size_t fcm_carry_bytes();
+int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist);
+int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st);
 size_t dpratio_fcm_workspace(uint64_t n_words);
-int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st);
+int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st,
+                          uint32_t halo = 0, uint64_t gbase = 0, const void* carry = nullptr);
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);
 
 }  // namespace lcf

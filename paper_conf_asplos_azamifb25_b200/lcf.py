@@ -54,6 +54,14 @@ def lib() -> ctypes.CDLL:
         L.lcf_compress_shard.restype = i32
         L.lcf_write_header.argtypes = [i32, i32, sz, u64, vp, vp]
         L.lcf_write_header.restype = i32
+        L.lcf_dpratio_summary_bytes.argtypes = []
+        L.lcf_dpratio_summary_bytes.restype = sz
+        L.lcf_dpratio_shard_summary.argtypes = [vp, sz, sz, u64, vp, vp]
+        L.lcf_dpratio_shard_summary.restype = i32
+        L.lcf_dpratio_merge_summaries.argtypes = [vp, sz, vp, vp]
+        L.lcf_dpratio_merge_summaries.restype = i32
+        L.lcf_dpratio_compress_shard.argtypes = [vp, sz, sz, u64, vp, vp, vp, sz, vp, vp]
+        L.lcf_dpratio_compress_shard.restype = i32
         L.lcf_launch_count.argtypes = []
         L.lcf_launch_count.restype = u64
         L.lcf_profile_enable.argtypes = [i32]
@@ -174,6 +182,27 @@ def lcf_compress_shard(algo, dtype, d_in_shard, shard_bytes, total_in_bytes, fir
     _check(lib().lcf_compress_shard(a, _dtype(dtype, a), _ptr(d_in_shard), shard_bytes, total_in_bytes,
                                     first_chunk, _ptr(d_table_slice), _ptr(d_payload), payload_capacity,
                                     _ptr(d_payload_bytes), _stream(stream)), "lcf_compress_shard")
+
+
+def lcf_dpratio_summary_bytes() -> int:
+    return int(lib().lcf_dpratio_summary_bytes())
+
+
+def lcf_dpratio_shard_summary(d_x, shard_bytes, total_in_bytes, first_word, d_summary, stream=None) -> None:
+    _check(lib().lcf_dpratio_shard_summary(_ptr(d_x), shard_bytes, total_in_bytes, first_word, _ptr(d_summary),
+                                           _stream(stream)), "lcf_dpratio_shard_summary")
+
+
+def lcf_dpratio_merge_summaries(d_summaries, count, d_carry, stream=None) -> None:
+    _check(lib().lcf_dpratio_merge_summaries(_ptr(d_summaries), count, _ptr(d_carry), _stream(stream)),
+           "lcf_dpratio_merge_summaries")
+
+
+def lcf_dpratio_compress_shard(d_x, shard_bytes, total_in_bytes, first_word, d_carry, d_table_slice, d_payload,
+                               payload_capacity, d_payload_bytes, stream=None) -> None:
+    _check(lib().lcf_dpratio_compress_shard(_ptr(d_x), shard_bytes, total_in_bytes, first_word, _ptr(d_carry),
+                                            _ptr(d_table_slice), _ptr(d_payload), payload_capacity,
+                                            _ptr(d_payload_bytes), _stream(stream)), "lcf_dpratio_compress_shard")
 
 
 def lcf_write_header(algo, dtype, total_in_bytes, total_payload_bytes, d_stream, stream=None) -> None:

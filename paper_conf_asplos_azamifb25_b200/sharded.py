@@ -12,8 +12,8 @@ concatenation header ‖ table slices ‖ pad ‖ payload pieces is byte-identic
 the 1-GPU stream. Decompression needs no exchange: every rank decodes its local
 stream.
 
-DPratio is not sharded by chunk range: FCM is a whole-array pass (L104). It
-runs whole fields per rank instead.
+DPratio shards by whole tiles with one more exchange (the FCM summaries, see
+below); its pieces assemble into the 1-GPU stream the same way.
 """
 from __future__ import annotations
 
@@ -134,3 +134,91 @@ def lcf_local_compress(algo: str, shard):
 def lcf_local_decompress(algo: str, local_stream, out=None):
     from . import lcf
     return lcf.decompress(algo, local_stream, out=out)
+
+
+# ---- sharded DPratio -------------------------------------
+# FCM (L170–185) compares a word with the ≤ 4 nearest preceding same-hash words
+# anywhere before it. Ranks own whole 2048-word tiles; each computes a summary
+# of its shard (per hash, its last ≤ 4 words), the summaries are all-gathered,
+# and rank g merges those of ranks 0 … g−1 into its carry (lcf.h). With the
+# carry, the shard's chunks are exactly the 1-GPU stream's chunks 2·t, 2·t+1 of
+# its tiles t, and the pieces assemble like the chunk-local codecs'.
+
+TILE_WORDS = 2048
+
+
+def dp_shard_words(n_words: int, world: int, rank: int):
+    """(first_word, n_words) of `rank`'s contiguous range of whole tiles."""
+    T = -(-n_words // TILE_WORDS)
+    t0, t1 = T * rank // world, T * (rank + 1) // world
+    first = t0 * TILE_WORDS
+    return first, max(0, min(n_words, t1 * TILE_WORDS) - first)
+
+
+def dp_compress_piece(x_shard, n_total_words: int, first_word: int, carry, rank: int):
+    """One shard's table slice, payload piece and device payload byte count
+    (lcf_dpratio_compress_shard). x_shard: int64 CUDA tensor view of the
+    shard's words inside a buffer that also holds the 3 words before it."""
+    import torch
+    from . import lcf
+    nb = x_shard.numel() * 8
+    tiles = -(-x_shard.numel() // TILE_WORDS)
+    cap = max(16, 2 * tiles * CHUNK)
+    table = torch.empty(max(1, 2 * tiles), dtype=torch.int32, device=x_shard.device)
+    payload = torch.empty(cap, dtype=torch.uint8, device=x_shard.device)
+    count = torch.zeros(1, dtype=torch.int64, device=x_shard.device)
+    lcf.lcf_dpratio_compress_shard(x_shard, nb, 8 * n_total_words, first_word, carry, table, payload, cap, count)
+    return table[:2 * tiles], payload, count
+
+
+def dp_simulate_shards(x, world: int) -> bytes:
+    """All ranks' steps on one device, in rank order (the exchange becomes a
+    stacked tensor): the assembled stream, for identity tests."""
+    import torch
+    from . import lcf
+    n = x.numel()
+    sb = lcf.lcf_dpratio_summary_bytes()
+    sums = torch.empty(world * sb, dtype=torch.uint8, device=x.device)
+    ranges = [dp_shard_words(n, world, g) for g in range(world)]
+    for g, (f, k) in enumerate(ranges):
+        lcf.lcf_dpratio_shard_summary(x[f:f + k] if k else x, 8 * k, 8 * n, f, sums[g * sb:(g + 1) * sb])
+    carry = torch.empty(sb, dtype=torch.uint8, device=x.device)
+    tables, pays = [], []
+    for g, (f, k) in enumerate(ranges):
+        if g:
+            lcf.lcf_dpratio_merge_summaries(sums, g, carry)
+        t, p, c = dp_compress_piece(x[f:f + k] if k else x[:0], n, f, carry if g else None, g)
+        torch.cuda.synchronize()
+        tables.append(t.cpu().numpy().tobytes())
+        pays.append(p[:int(c.item())].cpu().numpy().tobytes())
+    C = 2 * -(-n // TILE_WORDS)
+    tab = b"".join(tables)
+    assert len(tab) == 4 * C
+    base = round16(HEADER + 4 * C)
+    payload = b"".join(pays)
+    hdr = (0x3146434C).to_bytes(4, "little") + bytes([1, 3, 8, 0]) + (8 * n).to_bytes(8, "little") + \
+        C.to_bytes(8, "little") + len(payload).to_bytes(8, "little")
+    return hdr + tab + bytes(base - HEADER - 4 * C) + payload
+
+
+def dp_compress_sharded(x_shard, n_total_words: int, first_word: int, group=None):
+    """The distributed version (one process per GPU, NCCL): the summary
+    all-gather, this rank's carry, its piece and the payload-count exchange.
+    Returns (table slice, payload piece, payload offset, total payload)."""
+    import torch
+    import torch.distributed as dist
+    from . import lcf
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    sb = lcf.lcf_dpratio_summary_bytes()
+    mine = torch.empty(sb, dtype=torch.uint8, device=x_shard.device)
+    lcf.lcf_dpratio_shard_summary(x_shard, x_shard.numel() * 8, 8 * n_total_words, first_word, mine)
+    sums = torch.empty(world * sb, dtype=torch.uint8, device=x_shard.device)
+    dist.all_gather_into_tensor(sums, mine, group=group)
+    carry = None
+    if rank:
+        carry = torch.empty(sb, dtype=torch.uint8, device=x_shard.device)
+        lcf.lcf_dpratio_merge_summaries(sums, rank, carry)
+    table, payload, count = dp_compress_piece(x_shard, n_total_words, first_word, carry, rank)
+    counts = exchange_counts(count, group=group)
+    off = sum(counts[:rank])
+    return table, payload[:counts[rank]], off, sum(counts)

@@ -94,5 +94,43 @@ def test_nccl_single_rank_exchange(L):
         piece = sharded.compress_sharded("SPspeed", x, total, sharded.lcf_local_compress)
         stream = sharded.assemble("SPspeed", total, [piece])
         assert stream == L.compress("SPspeed", x).cpu().numpy().tobytes()
+        # the distributed DPratio entry point (summary all-gather, count exchange) on one rank
+        xd = _words("DPratio", 5 * 2048 + 17)
+        table, payload, off, tot = sharded.dp_compress_sharded(xd, xd.numel(), 0)
+        full = L.compress("DPratio", xd).cpu().numpy()
+        C = 2 * 6
+        base = (32 + 4 * C + 15) // 16 * 16
+        assert off == 0 and tot == len(full) - base
+        assert table.cpu().numpy().tobytes() == full[32:32 + 4 * C].tobytes()
+        assert payload.cpu().numpy().tobytes() == full[base:].tobytes()
     finally:
         dist.destroy_process_group()
+
+
+def _dp_inputs():
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from test_gpu_parity import fcm_stress_input
+    rng = np.random.default_rng(12)
+    mixed = rng.integers(0, 2**63, size=40 * 2048 + 999, dtype=np.uint64)
+    for _ in range(300):  # copies from anywhere earlier: matches that cross shard boundaries
+        n = int(rng.integers(1, 40))
+        i = int(rng.integers(n + 1, len(mixed) - n))
+        j = int(rng.integers(0, i - n))
+        mixed[i:i + n] = mixed[j:j + n]
+    slab = datagen.field("miranda_256x384x384_f64", "density", shape=(2, 384, 384)).numpy().reshape(-1).view(np.uint64)
+    return {"fcm_stress": fcm_stress_input(), "copies": mixed, "miranda_slab": slab.copy()}
+
+
+@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab"])
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_dpratio_shards_assemble_to_global(L, orc, name, world):
+    """Sharded DPratio (NEXT-1): shard summaries → per-shard carries → shard
+    pieces assemble into exactly the 1-GPU stream (and the oracle's)."""
+    words = _dp_inputs()[name]
+    x = torch.from_numpy(words.view(np.int64)).cuda()
+    full = L.compress("DPratio", x).cpu().numpy().tobytes()
+    got = sharded.dp_simulate_shards(x, world)
+    assert got == full
+    if name != "fcm_stress":
+        assert got == orc.compress("DPratio", words)

@@ -395,11 +395,14 @@ struct FcmCarry {
 constexpr uint64_t kHashes = 1ull << 20;
 __host__ __device__ constexpr size_t carry_bytes() { return kHashes * (1 + 4 * 4 + 4 * 8); }
 
+// CARRY: a shard after the first (compiled separately: the carry test costs
+// the unsharded match a third of its time)
+template <bool CARRY>
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint64_t* __restrict__ rec,
                                                                 uint32_t* __restrict__ dist, FcmCarry carry,
                                                                 uint64_t gbase) {
-  const bool carry_on = carry.cnt != nullptr;
+  constexpr bool carry_on = CARRY;
   const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
   for (uint64_t g = blockIdx.x * (uint64_t)kMatchBlock + threadIdx.x; g < groups;
        g += (uint64_t)gridDim.x * kMatchBlock) {
@@ -449,7 +452,7 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
         if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
         const uint32_t hb = hw[4 + j - back];
         if ((hb ^ hk) >> 12) break;  // left the hash's run
-        ++used;
+        if (CARRY) ++used;
         if (hb == hk) {              // same hash and fingerprint
           const uint32_t jj = (uint32_t)(r[4 + j - back] & kRecIdxMask);
           if (!have) {
@@ -462,7 +465,7 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
           }
         }
       }
-      if (carry_on && d == 0 && used < 4) {  // the remaining candidates precede the shard
+      if (CARRY && d == 0 && used < 4) {  // the remaining candidates precede the shard
         const uint32_t h = hk >> 12, cc = carry.cnt[h];
 #pragma unroll
         for (uint32_t q = 0; q < 4; ++q) {
@@ -604,7 +607,8 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
     KTrace kt("fcm_match", st);
     const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
     const int mblocks = (int)umin64((groups + kMatchBlock - 1) / kMatchBlock, 148 * 16);
-    fcm_match_kernel<<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
+    if (carry) fcm_match_kernel<true><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
+    else fcm_match_kernel<false><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
   }
   return launches + 1;
 }

@@ -154,7 +154,10 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  * d_x points at the shard's first word (global index first_word, a multiple
  * of 2048); the min(3, first_word) words before it must be readable (the hash
  * context of the shard's first words, L172). shard_bytes is a multiple of
- * 16384 unless the shard ends the array. Errors as lcf_compress_shard. */
+ * 16384 unless the shard ends the array. Errors as lcf_compress_shard.
+ * lcf_dpratio_compress_shard right after lcf_dpratio_shard_summary of the same
+ * shard (same d_x, size, first_word) on the same stream reuses the summary's
+ * sort of the shard; its words must not change in between. */
 size_t lcf_dpratio_summary_bytes(void);
 lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,
                                        void* d_summary, void* stream);

@@ -39,6 +39,11 @@ struct Workspace {
   std::vector<cudaEvent_t> ev;
   uint8_t* hstage = nullptr;
   size_t hstage_cap = 0;
+  // sharded DPratio: scratch[2] holds the sorted FCM records of this shard
+  // (set by lcf_dpratio_shard_summary, consumed by the next compress_shard)
+  const void* sorted_x = nullptr;
+  const void* sorted_ws = nullptr;
+  uint64_t sorted_n = 0, sorted_first = 0;
 };
 
 std::mutex g_mu;
@@ -167,6 +172,7 @@ EncArgs enc_args(int algo, const void* in, uint64_t in_bytes) {
 lcf_status_t enqueue_encode(Workspace* ws, EncArgs& a) {
   if (lcf_status_t s = grow(ws->status, ws->status_cap, a.n_chunks, ws->stream, true)) return s;
   if (a.algo == LCF_DPRATIO) {
+    ws->sorted_x = nullptr;  // scratch[2] is rewritten
     const size_t need = dpratio_fcm_workspace(a.n_words_total);
     if (lcf_status_t s = grow(reinterpret_cast<uint8_t*&>(ws->scratch[2]), ws->scratch_cap[2], need, ws->stream, false))
       return s;
@@ -753,7 +759,12 @@ lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size
   g_launches += launch_fcm_shard(static_cast<const uint64_t*>(d_x), n, (uint32_t)(first_word < 3 ? first_word : 3),
                                  first_word, nullptr, d_summary, false, ws->scratch[2], ws->scratch_cap[2], stream,
                                  &dist);
-  return last_launch_status();
+  if ((st = last_launch_status())) return st;
+  ws->sorted_x = d_x;
+  ws->sorted_ws = ws->scratch[2];
+  ws->sorted_n = n;
+  ws->sorted_first = first_word;
+  return LCF_SUCCESS;
 }
 
 lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream_) {
@@ -789,9 +800,13 @@ lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, siz
       (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[2]), ws->scratch_cap[2], dpratio_fcm_workspace(n), stream,
                  false)))
     return st;
+  // the summary call on this stream already sorted this shard: skip the sort
+  const bool sorted = ws->sorted_x == d_x && ws->sorted_ws == ws->scratch[2] && ws->sorted_n == n &&
+                      ws->sorted_first == first_word;
+  ws->sorted_x = nullptr;
   LaunchCtx ctx = make_ctx(ws);
   g_launches += launch_dpratio_encode(a, ctx, ws->scratch[2], ws->scratch_cap[2], stream,
-                                      (uint32_t)(first_word < 3 ? first_word : 3), first_word, d_carry);
+                                      (uint32_t)(first_word < 3 ? first_word : 3), first_word, d_carry, sorted);
   return last_launch_status();
 }
 

@@ -1037,13 +1037,13 @@ __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs
 size_t dpratio_fcm_workspace(uint64_t n) { return fcm_dist_workspace(n); }
 
 int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st,
-                          uint32_t halo, uint64_t gbase, const void* carry) {
+                          uint32_t halo, uint64_t gbase, const void* carry, bool sorted) {
   const uint64_t n = a0.n_words_total;
   int launches = 0;
   if (n) {
     uint32_t* dist = nullptr;  // FCM distances (L170–185), lcf_fcm.cu; a shard's with its carry
     launches += launch_fcm_shard(reinterpret_cast<const uint64_t*>(a0.in), n, halo, gbase, carry, nullptr, true, ws,
-                                 ws_bytes, st, &dist);
+                                 ws_bytes, st, &dist, sorted);
     EncArgs a = a0;
     a.fcm_dist = dist;
     const size_t smem = sizeof(DEncSmem);

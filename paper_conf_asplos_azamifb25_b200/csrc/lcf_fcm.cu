@@ -543,7 +543,7 @@ size_t fcm_carry_bytes() { return carry_bytes(); }
 // summaries of the earlier shards, or null). summary (optional) receives this
 // shard's own summary; with match false only the summary is made.
 int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
-                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out, bool sorted) {
   (void)ws_bytes;
   uint8_t* p = static_cast<uint8_t*>(ws);
   uint64_t* rec_a = reinterpret_cast<uint64_t*>(p);
@@ -563,7 +563,8 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
     return true;
   }();
   (void)init;
-  int launches = 6;
+  int launches = sorted ? 0 : 6;
+  if (!sorted) {  // (sorted: rec_b still holds this shard's sorted records from the summary call)
   {
     KTrace kt("fcm_sort_hist", st);
     sort_hist_kernel<0><<<(unsigned)T, kSortThreads, 0, st>>>(x, n, counts, halo);
@@ -587,6 +588,7 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
   {
     KTrace kt("fcm_sort_scatter", st);
     sort_scatter_kernel<1><<<(unsigned)T, kST, sizeof(ScatterSmem), st>>>(rec_a, n, counts, tot, rec_b, 0);
+  }
   }
   if (summary) {
     uint8_t* sb = static_cast<uint8_t*>(summary);
@@ -614,7 +616,7 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
 }
 
 int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
-  return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out);
+  return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out, false);
 }
 
 int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st) {

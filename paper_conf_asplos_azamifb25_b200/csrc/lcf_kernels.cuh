@@ -162,11 +162,11 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
 // shard's summary (fcm_carry_bytes() bytes); match = false: summary only.
 size_t fcm_carry_bytes();
 int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
-                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist);
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist, bool sorted = false);
 int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st);
 size_t dpratio_fcm_workspace(uint64_t n_words);
 int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st,
-                          uint32_t halo = 0, uint64_t gbase = 0, const void* carry = nullptr);
+                          uint32_t halo = 0, uint64_t gbase = 0, const void* carry = nullptr, bool sorted = false);
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);
 
 }  // namespace lcf

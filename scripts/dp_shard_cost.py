@@ -39,6 +39,13 @@ for world in [int(w) for w in sys.argv[1:]] or [8]:
     t_sum = timed(lambda: lcf.lcf_dpratio_shard_summary(x[f:f + k], 8 * k, 8 * n, f, sums[g * sb:(g + 1) * sb]))
     t_merge = timed(lambda: lcf.lcf_dpratio_merge_summaries(sums, g, carry))
     t_comp = timed(lambda: sharded.dp_compress_piece(x[f:f + k], n, f, carry, g))
+
+    def rank_seq():  # what the rank runs: summary, merge, compress (the sort is reused)
+        lcf.lcf_dpratio_shard_summary(x[f:f + k], 8 * k, 8 * n, f, sums[g * sb:(g + 1) * sb])
+        lcf.lcf_dpratio_merge_summaries(sums, g, carry)
+        sharded.dp_compress_piece(x[f:f + k], n, f, carry, g)
+    t_rank = timed(rank_seq)
     t_full = timed(lambda: lcf.compress("DPratio", x)) if world == int(sys.argv[1] if len(sys.argv) > 1 else 8) else 0
     print(f"world {world}: shard {8 * k / 1e6:.1f} MB: summary {t_sum:.0f} us, merge {t_merge:.0f} us, "
-          f"compress {t_comp:.0f} us (1-GPU whole field {t_full:.0f} us)")
+          f"compress {t_comp:.0f} us; the rank's sequence (sort reused) {t_rank:.0f} us "
+          f"(1-GPU whole field {t_full:.0f} us)")

@@ -354,7 +354,13 @@ def run_transfer(jobs, rank, dev, reps: int = 3):
         if j["codec"] == "DPratio":
             continue
         x = j["x"]
-        buf = torch.empty_like(x)
+        # the receiver sizes its buffer from the sender's (shards of one stream differ in length)
+        nel = torch.tensor([x.numel()], dtype=torch.int64, device=dev)
+        if rank == 0:
+            dist.send(nel, 1)
+        elif rank == 1:
+            dist.recv(nel, 0)
+        buf = torch.empty(int(nel.item()), dtype=x.dtype, device=dev)
         res = {}
         for mode in ("raw", "compressed"):
             ts = []
@@ -372,7 +378,7 @@ def run_transfer(jobs, rank, dev, reps: int = 3):
                     if mode == "raw":
                         dist.recv(buf, 0)
                     else:
-                        tr.recv_compressed(0, j["codec"], out=buf)
+                        tr.recv_compressed(0, j["codec"], device=dev)
                 e1.record()
                 torch.cuda.synchronize()
                 t = torch.tensor([e0.elapsed_time(e1) if rank < 2 else 0.0], device=dev)

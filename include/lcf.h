@@ -157,7 +157,18 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  * 16384 unless the shard ends the array. Errors as lcf_compress_shard.
  * lcf_dpratio_compress_shard right after lcf_dpratio_shard_summary of the same
  * shard (same d_x, size, first_word) on the same stream reuses the summary's
- * sort of the shard; its words must not change in between. */
+ * sort of the shard; its words must not change in between.
+ *
+ * Decompression of a shard: d_in is the shard's own LCF1 sub-stream (header
+ * for its words, its size-table slice, its payload piece), whose word 0 is
+ * global word first_word. Distances that stay in the shard are resolved (L197);
+ * a word whose chain leaves the shard is left pending: d_out holds the global
+ * index of the word it copies, and its bit in d_pending is set (u32 bitmap of
+ * ceil(out_capacity / 8 / 32) words, cleared by the call). Asynchronous;
+ * malformed input is reported by lcf_check_stream. lcf_dpratio_resolve_pending
+ * then replaces every pending word by d_prefix[target], d_prefix holding the
+ * final words of global indices [0, first_word) (device). Shards are resolved
+ * in array order. */
 size_t lcf_dpratio_summary_bytes(void);
 lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,
                                        void* d_summary, void* stream);
@@ -166,6 +177,10 @@ lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, siz
                                         uint64_t first_word, const void* d_carry, void* d_table_slice,
                                         void* d_payload, size_t payload_capacity, uint64_t* d_payload_bytes,
                                         void* stream);
+lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uint64_t first_word, void* d_out,
+                                          size_t out_capacity, uint32_t* d_pending, void* stream);
+lcf_status_t lcf_dpratio_resolve_pending(void* d_out, size_t shard_bytes, const uint32_t* d_pending,
+                                         const void* d_prefix, void* stream);
 
 /* Number of kernel launches the library enqueued since the process started
  * (bench/test accounting). */

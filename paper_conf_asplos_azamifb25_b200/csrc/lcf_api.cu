@@ -810,6 +810,50 @@ lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, siz
   return last_launch_status();
 }
 
+lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uint64_t first_word, void* d_out,
+                                          size_t out_capacity, uint32_t* d_pending, void* stream_) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  if (!d_in || !aligned16(d_in) || !d_pending || (out_capacity && (!d_out || !aligned16(d_out))))
+    return LCF_ERROR_INVALID_ARGUMENT;
+  if (first_word % 2048) return LCF_ERROR_INVALID_ARGUMENT;
+  if (in_bytes < kHeaderBytes) return LCF_ERROR_CORRUPT_STREAM;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  const uint64_t by_table = (in_bytes - kHeaderBytes) / 4;
+  const uint64_t by_out = 2 * ((out_capacity + kChunkBytes - 1) / kChunkBytes);
+  uint64_t grid = by_table < by_out ? by_table : by_out;
+  if (grid == 0) grid = 1;
+  if ((st = grow(ws->status, ws->status_cap, grid, stream, true)) ||
+      (st = grow(ws->tile_flag, ws->tile_cap, grid / 2 + 1, stream, true)))
+    return st;
+  if (!cuda_ok(cudaMemsetAsync(d_pending, 0, 4 * ((out_capacity / 8 + 31) / 32), stream))) return LCF_ERROR_CUDA;
+  DecArgs a{};
+  a.stream = static_cast<const uint8_t*>(d_in);
+  a.stream_bytes = in_bytes;
+  a.out = static_cast<uint8_t*>(d_out);
+  a.out_capacity = out_capacity;
+  a.algo = LCF_DPRATIO;
+  a.word_bytes = 8;
+  a.tile_flag = ws->tile_flag;
+  a.gbase = first_word;
+  a.pend = d_pending;
+  LaunchCtx ctx = make_ctx(ws);
+  launch_dpratio_decode(a, ctx, grid / 2 + 1, stream);
+  ++g_launches;
+  return last_launch_status();
+}
+
+lcf_status_t lcf_dpratio_resolve_pending(void* d_out, size_t shard_bytes, const uint32_t* d_pending,
+                                         const void* d_prefix, void* stream_) {
+  if (shard_bytes % 8 || (shard_bytes && (!d_out || !d_pending || !d_prefix))) return LCF_ERROR_INVALID_ARGUMENT;
+  launch_dp_resolve_pending(static_cast<uint64_t*>(d_out), shard_bytes / 8, d_pending,
+                            static_cast<const uint64_t*>(d_prefix), (cudaStream_t)stream_);
+  ++g_launches;
+  return last_launch_status();
+}
+
 lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,
                               uint64_t total_payload_bytes, void* d_stream, void* stream_) {
   if (!valid_algo(algo)) return LCF_ERROR_INVALID_ARGUMENT;

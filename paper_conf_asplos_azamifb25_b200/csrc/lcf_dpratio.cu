@@ -711,6 +711,7 @@ struct DDecSmem {
   alignas(128) uint8_t sd[kChunkBytes + 128];
   alignas(128) uint8_t rz[kChunkBytes + 128];
   alignas(128) uint64_t X[kTileWords + 8];
+  uint32_t pmask[kTileWords / 32];  // shard decode: pending words of the tile
   uint64_t full_v[1], empty_v[1], full_d[1], empty_d[1];
   uint64_t tile[1];
   uint32_t len[2], flags[1];
@@ -719,6 +720,7 @@ struct DDecSmem {
 struct FcmScratch {  // pointer jumping (aliases S.rz)
   int32_t pj[2][kDT];  // target (−1 done)
   uint64_t vj[2][kDT];
+  uint8_t fj[2][kDT];  // shard decode: value is a pending global target
 };
 static_assert(sizeof(FcmScratch) <= kChunkBytes, "FCM scratch fits in rz");
 
@@ -848,6 +850,7 @@ __device__ __forceinline__ bool raze_diffms_inv(const uint8_t* rz, uint32_t off,
   return true;
 }
 
+template <bool SHARD>
 __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t tid) {
   const uint32_t lane = tid & 31;
   const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
@@ -953,36 +956,48 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
     // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
     bool bad = !ok;
     if (ok && nzD) {  // (no distances: x = V as it stands)
+      if (SHARD)
+        for (uint32_t w = tid; w < kTileWords / 32; w += kDT) S.pmask[w] = 0;
       bar_d();  // X complete (V's DIFFMS⁻¹ ends without a barrier)
+      const uint64_t gb = SHARD ? a.gbase : 0;  // global index of this stream's word 0
       for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
         const uint32_t li = b + tid;
         int32_t p = -1;
         uint64_t val = 0;
+        uint8_t f = 0;  // (shard decode) val is a pending global target
         if (li < m) {
-          const uint64_t d = Dw[li], gi = t0 + li;
+          const uint64_t d = Dw[li], gi = gb + t0 + li;
           if (d == 0) {
             val = S.X[li];
           } else if (d > gi || S.X[li] != 0) {
             bad = true;
-          } else if (gi - d >= t0 + b) {
-            p = (int32_t)(gi - d - t0 - b);  // inside this block: resolve below
-          } else if (gi - d >= t0) {
-            val = S.X[gi - d - t0];  // earlier block of this tile: already final
-          } else {  // earlier tile: wait for its completion flag, then read the output
-            const uint64_t j = gi - d, tj = j / kTileWords;  // (tiles before first_tile: final already)
+          } else if (gi - d >= gb + t0 + b) {
+            p = (int32_t)(gi - d - gb - t0 - b);  // inside this block: resolve below
+          } else if (gi - d >= gb + t0) {
+            const uint32_t lj = (uint32_t)(gi - d - gb - t0);
+            val = S.X[lj];  // earlier block of this tile: already final (or pending)
+            if (SHARD) f = (S.pmask[lj / 32] >> (lj % 32)) & 1;
+          } else if (!SHARD || gi - d >= gb) {  // earlier tile: wait for its flag, then read the output
+            const uint64_t j = gi - d - gb, tj = j / kTileWords;  // (tiles before first_tile: final already)
             while (tj >= a.first_tile && ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
             val = ld_cg_u64(out + j);
+            if (SHARD) f = (__ldcg(a.pend + j / 32) >> (j % 32)) & 1;
+          } else {  // before the shard: pending on the global word gi − d
+            val = gi - d;
+            f = 1;
           }
         }
         // pointer jumping inside the block (≤ 8 rounds; chains point backwards)
         uint32_t par = 0;
         F.pj[0][tid] = p;
         F.vj[0][tid] = val;
+        if (SHARD) F.fj[0][tid] = f;
         while (bar_d_or(p >= 0)) {
           if (p >= 0) {
             const int32_t q = F.pj[par][p];
             if (q < 0) {
               val = F.vj[par][p];
+              if (SHARD) f = F.fj[par][p];
               p = -1;
             } else {
               p = q;
@@ -990,11 +1005,15 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
           }
           F.pj[par ^ 1][tid] = p;
           F.vj[par ^ 1][tid] = val;
+          if (SHARD) F.fj[par ^ 1][tid] = f;
           par ^= 1;
         }
         if (li < m) S.X[li] = val;  // x, in place
+        if (SHARD && li < m && f) atomicOr(&S.pmask[li / 32], 1u << (li % 32));
         bar_d();
       }
+      if (SHARD)  // the tile's pending bits, before its completion flag (released after a barrier)
+        for (uint32_t w = tid; w < (m + 31) / 32; w += kDT) a.pend[t0 / 32 + w] = S.pmask[w];
       release(&S.empty_d[0]);
     }
     if (tid == 0) trace_stamp(a, t, 6);
@@ -1015,6 +1034,7 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   }
 }
 
+template <bool SHARD>
 __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DDecSmem& S = *reinterpret_cast<DDecSmem*>(smem_raw);
@@ -1028,7 +1048,7 @@ __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs
   }
   __syncthreads();
   if (warp == 0) d_dec_loader(S, a, ctx, lane);
-  else d_dec_compute(S, a, ctx, threadIdx.x - 32);
+  else d_dec_compute<SHARD>(S, a, ctx, threadIdx.x - 32);
 }
 
 }  // namespace
@@ -1060,16 +1080,36 @@ int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, siz
   return launches;
 }
 
+namespace {
+// Pending words of a decoded shard take the final word of their global target
+// (prefix: the words before the shard, final).
+__global__ void __launch_bounds__(256) dp_resolve_pending_kernel(uint64_t* __restrict__ out, uint64_t n,
+                                                                const uint32_t* __restrict__ pend,
+                                                                const uint64_t* __restrict__ prefix) {
+  for (uint64_t i = blockIdx.x * 256ull + threadIdx.x; i < n; i += (uint64_t)gridDim.x * 256)
+    if ((pend[i / 32] >> (i % 32)) & 1) out[i] = prefix[out[i]];
+}
+}  // namespace
+
+void launch_dp_resolve_pending(uint64_t* out, uint64_t n, const uint32_t* pend, const uint64_t* prefix,
+                               cudaStream_t st) {
+  if (!n) return;
+  KTrace kt("dpratio_resolve_pending", st);
+  dp_resolve_pending_kernel<<<(unsigned)umin64((n + 255) / 256, 148 * 16), 256, 0, st>>>(out, n, pend, prefix);
+}
+
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st) {
   const size_t smem = sizeof(DDecSmem);
   static const bool init = [&] {
-    cudaFuncSetAttribute(dpratio_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(dpratio_decode_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(dpratio_decode_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     return true;
   }();
   (void)init;
-  const int grid = persistent_grid(dpratio_decode_kernel, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
+  const int grid = persistent_grid(dpratio_decode_kernel<false>, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
   KTrace kt("dpratio_decode", st);
-  dpratio_decode_kernel<<<grid, kDDecThreads, smem, st>>>(a, ctx);
+  if (a.pend) dpratio_decode_kernel<true><<<grid, kDDecThreads, smem, st>>>(a, ctx);
+  else dpratio_decode_kernel<false><<<grid, kDDecThreads, smem, st>>>(a, ctx);
 }
 
 }  // namespace lcf

@@ -73,6 +73,11 @@ struct DecArgs {
   // 2·first_tile; earlier tiles are already final in `out` (an earlier launch
   // on the same stream) and only their payload bytes may be absent.
   uint64_t first_tile, end_tile, base_off;
+  // DPratio shard decode (NEXT-1): word 0 of this stream is global word gbase;
+  // a distance reaching before it is left pending: the output holds the global
+  // target index and `pend` (1 bit per word, zeroed) marks the word.
+  uint64_t gbase;
+  uint32_t* pend;
 };
 
 struct DecChunk {
@@ -168,5 +173,6 @@ size_t dpratio_fcm_workspace(uint64_t n_words);
 int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st,
                           uint32_t halo = 0, uint64_t gbase = 0, const void* carry = nullptr, bool sorted = false);
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);
+void launch_dp_resolve_pending(uint64_t* out, uint64_t n, const uint32_t* pend, const uint64_t* prefix, cudaStream_t st);
 
 }  // namespace lcf

@@ -62,6 +62,10 @@ def lib() -> ctypes.CDLL:
         L.lcf_dpratio_merge_summaries.restype = i32
         L.lcf_dpratio_compress_shard.argtypes = [vp, sz, sz, u64, vp, vp, vp, sz, vp, vp]
         L.lcf_dpratio_compress_shard.restype = i32
+        L.lcf_dpratio_decompress_shard.argtypes = [vp, sz, u64, vp, sz, vp, vp]
+        L.lcf_dpratio_decompress_shard.restype = i32
+        L.lcf_dpratio_resolve_pending.argtypes = [vp, sz, vp, vp, vp]
+        L.lcf_dpratio_resolve_pending.restype = i32
         L.lcf_launch_count.argtypes = []
         L.lcf_launch_count.restype = u64
         L.lcf_profile_enable.argtypes = [i32]
@@ -203,6 +207,16 @@ def lcf_dpratio_compress_shard(d_x, shard_bytes, total_in_bytes, first_word, d_c
     _check(lib().lcf_dpratio_compress_shard(_ptr(d_x), shard_bytes, total_in_bytes, first_word, _ptr(d_carry),
                                             _ptr(d_table_slice), _ptr(d_payload), payload_capacity,
                                             _ptr(d_payload_bytes), _stream(stream)), "lcf_dpratio_compress_shard")
+
+
+def lcf_dpratio_decompress_shard(d_in, in_bytes, first_word, d_out, out_capacity, d_pending, stream=None) -> None:
+    _check(lib().lcf_dpratio_decompress_shard(_ptr(d_in), in_bytes, first_word, _ptr(d_out), out_capacity,
+                                              _ptr(d_pending), _stream(stream)), "lcf_dpratio_decompress_shard")
+
+
+def lcf_dpratio_resolve_pending(d_out, shard_bytes, d_pending, d_prefix, stream=None) -> None:
+    _check(lib().lcf_dpratio_resolve_pending(_ptr(d_out), shard_bytes, _ptr(d_pending), _ptr(d_prefix),
+                                             _stream(stream)), "lcf_dpratio_resolve_pending")
 
 
 def lcf_write_header(algo, dtype, total_in_bytes, total_payload_bytes, d_stream, stream=None) -> None:

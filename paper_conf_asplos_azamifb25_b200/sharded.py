@@ -222,3 +222,119 @@ def dp_compress_sharded(x_shard, n_total_words: int, first_word: int, group=None
     counts = exchange_counts(count, group=group)
     off = sum(counts[:rank])
     return table, payload[:counts[rank]], off, sum(counts)
+
+
+def dp_shard_substream(stream: bytes, world: int, rank: int) -> bytes:
+    """Rank `rank`'s own LCF1 sub-stream of a DPratio stream: a header for its
+    words, its size-table slice and its payload piece (what it holds after a
+    sharded compression)."""
+    import numpy as np
+    h = np.frombuffer(stream[:32], np.uint64)
+    n = int(h[1]) // 8
+    C = int(h[2])
+    table = np.frombuffer(stream[HEADER:HEADER + 4 * C], np.uint32)
+    padded = (((table & 0x7FFFFFFF).astype(np.uint64) + 15) // 16) * 16
+    offs = np.concatenate([[0], np.cumsum(padded)]).astype(np.uint64)
+    base = round16(HEADER + 4 * C)
+    f, k = dp_shard_words(n, world, rank)
+    c0, c1 = 2 * (f // TILE_WORDS), 2 * (-(-(f + k) // TILE_WORDS))
+    pay = stream[base + int(offs[c0]):base + int(offs[c1])]
+    hdr = (0x3146434C).to_bytes(4, "little") + bytes([1, 3, 8, 0]) + (8 * k).to_bytes(8, "little") + \
+        (c1 - c0).to_bytes(8, "little") + len(pay).to_bytes(8, "little")
+    sub_base = round16(HEADER + 4 * (c1 - c0))
+    return hdr + table[c0:c1].tobytes() + bytes(sub_base - HEADER - 4 * (c1 - c0)) + pay
+
+
+def dp_simulate_decode_shards(stream: bytes, world: int):
+    """Sharded DPratio decompression on one device: every shard decodes its
+    sub-stream independently (cross-shard words left pending), then the shards
+    resolve their pending words in array order. Returns the int64 words."""
+    import numpy as np
+    import torch
+    from . import lcf
+    n = int(np.frombuffer(stream[8:16], np.uint64)[0]) // 8
+    out = torch.empty(max(n, 1), dtype=torch.int64, device="cuda")
+    pend, subs = [], []
+    for g in range(world):
+        f, k = dp_shard_words(n, world, g)
+        sub = torch.from_numpy(np.frombuffer(dp_shard_substream(stream, world, g), np.uint8).copy()).cuda()
+        p = torch.empty(max(1, (k + 31) // 32), dtype=torch.int32, device="cuda")
+        if k:
+            lcf.lcf_dpratio_decompress_shard(sub, sub.numel(), f, out[f:f + k], 8 * k, p)
+        subs.append(sub)
+        pend.append(p)
+    lcf.lcf_check_stream()
+    for g in range(world):  # in array order: everything before shard g is final
+        f, k = dp_shard_words(n, world, g)
+        if k:
+            lcf.lcf_dpratio_resolve_pending(out[f:f + k], 8 * k, pend[g], out)
+    torch.cuda.synchronize()
+    return out[:n]
+
+
+def _owner(j, n: int, world: int):
+    """Rank owning global word index j (tensor) under dp_shard_words."""
+    import torch
+    firsts = torch.tensor([dp_shard_words(n, world, r)[0] for r in range(world)], dtype=torch.int64,
+                          device=j.device)
+    return torch.searchsorted(firsts, j, right=True) - 1
+
+
+def dp_resolve_pending_distributed(out_local, pend, first_word: int, n_total: int, group=None):
+    """Resolve a decoded shard's pending words (lcf_dpratio_decompress_shard)
+    across ranks: in rank order r = 1 … G−1, rank r asks every lower rank for
+    the final words at its pending targets; a lower rank is final by then
+    (its own step came first). Point-to-point messages only: the request and
+    answer volume is the number of pending words. Works on any backend (NCCL
+    with CUDA tensors, gloo with CPU tensors)."""
+    import torch
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    dev = out_local.device
+    k = out_local.numel()
+    bits = pend.view(torch.int32)
+    pos = torch.arange(k, device=dev)
+    mask = ((bits[pos // 32] >> (pos % 32)) & 1).bool() if k else torch.zeros(0, dtype=torch.bool, device=dev)
+    idx = pos[mask]
+    tgt = out_local[idx].clone()
+    own = _owner(tgt, n_total, world) if idx.numel() else tgt
+    for r in range(1, world):
+        if rank == r:
+            for q in range(r):
+                sel = own == q
+                req = tgt[sel].contiguous()
+                cnt = torch.tensor([req.numel()], dtype=torch.int64, device=dev)
+                dist.send(cnt, q, group=group)
+                if req.numel():
+                    dist.send(req, q, group=group)
+                    vals = torch.empty_like(req)
+                    dist.recv(vals, q, group=group)
+                    out_local[idx[sel]] = vals
+        elif rank < r:
+            cnt = torch.empty(1, dtype=torch.int64, device=dev)
+            dist.recv(cnt, r, group=group)
+            c = int(cnt.item())
+            if c:
+                req = torch.empty(c, dtype=torch.int64, device=dev)
+                dist.recv(req, r, group=group)
+                dist.send(out_local[req - first_word].contiguous(), r, group=group)
+    return out_local
+
+
+def dp_decompress_sharded(sub_stream, first_word: int, n_total: int, group=None):
+    """The distributed sharded DPratio decompression of this rank's sub-stream
+    (dp_shard_substream layout, CUDA uint8 tensor): decode with cross-shard
+    chains pending, then resolve them against the lower ranks. Returns the
+    rank's int64 words."""
+    import torch
+    import torch.distributed as dist
+    from . import lcf
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    f, k = dp_shard_words(n_total, world, rank)
+    assert f == first_word
+    out = torch.empty(max(k, 1), dtype=torch.int64, device=sub_stream.device)
+    pend = torch.zeros(max(1, (k + 31) // 32), dtype=torch.int32, device=sub_stream.device)
+    if k:
+        lcf.lcf_dpratio_decompress_shard(sub_stream, sub_stream.numel(), f, out, 8 * k, pend)
+        lcf.lcf_check_stream()
+    return dp_resolve_pending_distributed(out[:k], pend, f, n_total, group=group)

@@ -103,6 +103,9 @@ def test_nccl_single_rank_exchange(L):
         assert off == 0 and tot == len(full) - base
         assert table.cpu().numpy().tobytes() == full[32:32 + 4 * C].tobytes()
         assert payload.cpu().numpy().tobytes() == full[base:].tobytes()
+        # and the distributed decompression entry point on the same rank
+        sub = torch.from_numpy(np.frombuffer(sharded.dp_shard_substream(full.tobytes(), 1, 0), np.uint8).copy()).cuda()
+        assert torch.equal(sharded.dp_decompress_sharded(sub, 0, xd.numel()), xd)
     finally:
         dist.destroy_process_group()
 
@@ -134,3 +137,16 @@ def test_dpratio_shards_assemble_to_global(L, orc, name, world):
     assert got == full
     if name != "fcm_stress":
         assert got == orc.compress("DPratio", words)
+
+
+@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab"])
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_dpratio_shard_decode(L, name, world):
+    """Sharded DPratio decompression (NEXT-1): each shard decodes its own
+    sub-stream with chains into earlier shards left pending, then the shards
+    resolve them in array order — the original words come back."""
+    words = _dp_inputs()[name]
+    x = torch.from_numpy(words.view(np.int64)).cuda()
+    stream = L.compress("DPratio", x).cpu().numpy().tobytes()
+    y = sharded.dp_simulate_decode_shards(stream, world)
+    assert torch.equal(y, x)

@@ -52,3 +52,13 @@ for algo in ("SPspeed", "SPratio", "DPspeed", "DPratio"):
         pass
     print(algo, "host slices ok")
 torch.cuda.synchronize()
+# sharded DPratio (NEXT-1): shard summaries / carries / pieces, and shard decodes with pending words
+from paper_conf_asplos_azamifb25_b200 import sharded  # noqa: E402
+w = datagen.field("miranda_256x384x384_f64", "density", shape=(1, 128, 384)).numpy().reshape(-1).view(np.uint64).copy()
+w[5000:9000] = w[17]
+xd = torch.from_numpy(w.view(np.int64)).cuda()
+full = lcf.compress("DPratio", xd).cpu().numpy().tobytes()
+assert sharded.dp_simulate_shards(xd, 3) == full
+assert torch.equal(sharded.dp_simulate_decode_shards(full, 3), xd)
+print("DPratio shards ok")
+torch.cuda.synchronize()

@@ -150,3 +150,29 @@ def test_dpratio_shard_decode(L, name, world):
     stream = L.compress("DPratio", x).cpu().numpy().tobytes()
     y = sharded.dp_simulate_decode_shards(stream, world)
     assert torch.equal(y, x)
+
+
+def test_dpratio_shards_small_and_errors(L):
+    """More ranks than tiles (empty shards), a ragged last tile, and argument
+    checks of the sharded DPratio calls."""
+    x = _words("DPratio", 2 * 2048 + 77)  # 3 tiles
+    x[1000:1500] = x[3]
+    full = L.compress("DPratio", x).cpu().numpy().tobytes()
+    for world in (3, 5, 8):
+        assert sharded.dp_simulate_shards(x, world) == full
+        assert torch.equal(sharded.dp_simulate_decode_shards(full, world), x)
+    sb = L.lcf_dpratio_summary_bytes()
+    summ = torch.empty(sb, dtype=torch.uint8, device="cuda")
+    n = x.numel()
+    with pytest.raises(L.LcfError) as e:  # not tile-aligned
+        L.lcf_dpratio_shard_summary(x[5:], 8 * (n - 5), 8 * n, 5, summ)
+    assert e.value.status == 1
+    with pytest.raises(L.LcfError) as e:  # a middle shard must be whole tiles
+        L.lcf_dpratio_shard_summary(x, 8 * 100, 8 * n, 0, summ)
+    assert e.value.status == 1
+    with pytest.raises(L.LcfError) as e:  # payload capacity too small
+        t = torch.empty(2, dtype=torch.int32, device="cuda")
+        p = torch.empty(64, dtype=torch.uint8, device="cuda")
+        c = torch.empty(1, dtype=torch.int64, device="cuda")
+        L.lcf_dpratio_compress_shard(x[:2048], 8 * 2048, 8 * n, 0, None, t, p, 64, c)
+    assert e.value.status == 3

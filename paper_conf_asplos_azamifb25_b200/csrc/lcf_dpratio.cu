@@ -31,6 +31,7 @@ constexpr uint32_t kDT = kDW * 32;     // compute threads
 #define LCF_DP_OUT 2
 #endif
 constexpr int kDOut = LCF_DP_OUT, kDBatch = 4;  // output slots (encode), tiles per ticket (decode)
+static_assert(kDOut >= 2, "a tile emits its V and Dist chunks into two slots (1 deadlocks; 3 measured equal)");
 constexpr int kDEncThreads = (2 + kDW) * 32, kDDecThreads = (1 + kDW) * 32;
 constexpr uint32_t kBarD = 1;
 constexpr uint32_t kTileWords = 2048;

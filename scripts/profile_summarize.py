@@ -51,7 +51,10 @@ with open(f"profiles/{tag}_launch_shares.csv", "w") as f:
 # 2. full-set captures: traffic per launch
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
-        "sm__inst_executed.sum.pct_of_peak_sustained_elapsed", "launch__registers_per_thread", "launch__grid_size"]
+        "sm__inst_executed.sum.pct_of_peak_sustained_elapsed", "launch__registers_per_thread", "launch__grid_size",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_st.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_st.sum",
+        "sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active"]
 UNIT = {"Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "byte": 1, "us": 1e-6, "ms": 1e-3, "ns": 1e-9, "s": 1.0,
         "usecond": 1e-6, "msecond": 1e-3, "nsecond": 1e-9}
 traffic = {}
@@ -85,12 +88,21 @@ for fn in sorted(os.listdir(src)):
         e["issue_pct"] = vals.get("sm__inst_executed.sum.pct_of_peak_sustained_elapsed")
         e["registers"] = vals.get("launch__registers_per_thread")
         e["grid"] = vals.get("launch__grid_size")
+        # LSU global sectors per request (TMA bulk copies bypass the LSU: 0 requests → None)
+        for op in ("ld", "st"):
+            req = vals.get(f"l1tex__t_requests_pipe_lsu_mem_global_op_{op}.sum", 0)
+            sec = vals.get(f"l1tex__t_sectors_pipe_lsu_mem_global_op_{op}.sum", 0)
+            e[f"{op}_sectors_per_request"] = sec / req if req else None
+        e["alu_pipe_pct"] = vals.get("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active")
 for k, e in traffic.items():
     e["dram_bytes_per_launch"] = e["dram_bytes"] / e["launches"]
     e["seconds_per_launch"] = e["seconds"] / e["launches"]
     lines.append(f"{k:55s} launches={e['launches']} dram/launch={e['dram_bytes_per_launch'] / 1e6:9.2f} MB "
                  f"t/launch={e['seconds_per_launch'] * 1e6:9.1f} us dram%={e['dram_pct']:.1f} "
-                 f"warps_active%={e['warps_active_pct']:.1f} issue%={e['issue_pct']:.1f} regs={e['registers']:.0f}")
+                 f"warps_active%={e['warps_active_pct']:.1f} issue%={e['issue_pct']:.1f} regs={e['registers']:.0f} "
+                 f"alu%={(e.get('alu_pipe_pct') or 0):.1f} "
+                 f"ld_sec/req={'-' if e.get('ld_sectors_per_request') is None else format(e['ld_sectors_per_request'], '.1f')} "
+                 f"st_sec/req={'-' if e.get('st_sectors_per_request') is None else format(e['st_sectors_per_request'], '.1f')}")
 json.dump(traffic, open(f"profiles/{tag}_kernel_traffic.json", "w"), indent=1)
 with open(f"profiles/{tag}_ncu_summary.txt", "w") as f:
     f.write("# ncu --set full, one capture per kernel family on the bench workload (cold cache, serialised)\n")

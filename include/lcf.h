@@ -107,7 +107,8 @@ lcf_status_t lcf_check_stream(void* stream);
  * decompress: the header and size table are read on the host; any malformed
  * slice reports CORRUPT_STREAM. DPratio decompression streams by tile ranges
  * (distances into earlier slices read their final output); DPratio
- * compression is serial (FCM's sort needs the whole array, L172). */
+ * compression by tile slices carrying the FCM state of the earlier slices (the
+ * sharded-DPratio calls below): the same bytes as lcf_compress. */
 lcf_status_t lcf_compress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,
                                void* h_out, size_t out_capacity, size_t* out_bytes, void* stream);
 lcf_status_t lcf_decompress_host(lcf_algo_t algo, lcf_dtype_t dtype, const void* h_in, size_t in_bytes,

@@ -606,6 +606,84 @@ static lcf_status_t decompress_host_dpratio_pipelined(const uint8_t* h_in, size_
   return LCF_SUCCESS;
 }
 
+// DPratio compression in tile slices (the sharded-DPratio machinery, §7 of
+// DESIGN.md, with slices for shards): slice i is summarised (its FCM sort),
+// encoded with the carry of slices < i (the sort is reused), and the carry for
+// slice i+1 = merge(carry_i, summary_i). The pieces stitch into exactly the
+// lcf_compress stream, and the H2D of slice i+1, the codec on slice i and the
+// D2H of slice i−1 overlap on the three streams.
+static lcf_status_t compress_host_dpratio_pipelined(const uint8_t* h_in, size_t in_bytes, uint8_t* h_out,
+                                                    size_t out_capacity, size_t* out_bytes, Workspace* ws,
+                                                    uint64_t st_tiles) {
+  const uint64_t n = in_bytes / 8, T = (n + 2047) / 2048, k = (T + st_tiles - 1) / st_tiles;
+  const uint64_t C = 2 * T, base = round16(kHeaderBytes + 4 * C);
+  if (out_capacity < base) return LCF_ERROR_BUFFER_TOO_SMALL;
+  const size_t sb = lcf_dpratio_summary_bytes();
+  const uint64_t slice_words = st_tiles * 2048;
+  const size_t piece_cap = round16(4 * 2 * st_tiles) + payload_bound(LCF_DPRATIO, 8 * slice_words) + 16;
+  lcf_status_t st;
+  if ((st = host_pipe_init(ws, 2 * k, 8 * k))) return st;
+  {
+    std::lock_guard<std::mutex> g(ws->mu);
+    if ((st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[0]), ws->scratch_cap[0], round16(in_bytes) + 16,
+                   ws->stream, false)) ||
+        (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[1]), ws->scratch_cap[1], k * piece_cap, ws->stream,
+                   false)) ||
+        (st = grow(reinterpret_cast<uint8_t*&>(ws->scratch[3]), ws->scratch_cap[3], 4 * sb, ws->stream, false)))
+      return st;
+  }
+  uint8_t* d_in = static_cast<uint8_t*>(ws->scratch[0]);
+  uint8_t* d_pieces = static_cast<uint8_t*>(ws->scratch[1]);
+  uint8_t* P[2] = {static_cast<uint8_t*>(ws->scratch[3]), static_cast<uint8_t*>(ws->scratch[3]) + 2 * sb};
+  // (P[j] = carry ‖ summary, contiguous for the 2-summary merge)
+  cudaEvent_t* evH = ws->ev.data();
+  cudaEvent_t* evC = ws->ev.data() + k;
+  uint64_t* cnt_h = reinterpret_cast<uint64_t*>(ws->hstage);
+  if (!cuda_ok(cudaMemsetAsync(P[0], 0, 1u << 20, ws->stream))) return LCF_ERROR_CUDA;  // empty carry of slice 0
+  uint64_t off = base;
+  auto finish = [&](uint64_t i) -> lcf_status_t {
+    const uint64_t t0 = i * st_tiles, nt = (t0 + st_tiles < T ? st_tiles : T - t0);
+    if (!cuda_ok(cudaEventSynchronize(evC[i]))) return LCF_ERROR_CUDA;
+    const uint64_t pay = cnt_h[i];
+    if (off + pay > out_capacity) return LCF_ERROR_BUFFER_TOO_SMALL;
+    const uint8_t* piece = d_pieces + i * piece_cap;
+    if (!cuda_ok(cudaStreamWaitEvent(ws->d2h, evC[i], 0)) ||
+        !cuda_ok(cudaMemcpyAsync(h_out + kHeaderBytes + 4 * 2 * t0, piece, 4 * 2 * nt, cudaMemcpyDeviceToHost,
+                                 ws->d2h)) ||
+        (pay && !cuda_ok(cudaMemcpyAsync(h_out + off, piece + round16(4 * 2 * st_tiles), pay,
+                                         cudaMemcpyDeviceToHost, ws->d2h))))
+      return LCF_ERROR_CUDA;
+    off += pay;
+    return LCF_SUCCESS;
+  };
+  for (uint64_t i = 0; i < k; ++i) {
+    const uint64_t w0 = i * slice_words, w1 = (w0 + slice_words < n ? w0 + slice_words : n);
+    const uint64_t b0 = 8 * w0, bytes = 8 * (w1 - w0);
+    if (!cuda_ok(cudaMemcpyAsync(d_in + b0, h_in + b0, bytes, cudaMemcpyHostToDevice, ws->h2d)) ||
+        !cuda_ok(cudaEventRecord(evH[i], ws->h2d)) || !cuda_ok(cudaStreamWaitEvent(ws->stream, evH[i], 0)))
+      return LCF_ERROR_CUDA;
+    uint8_t* cur = P[i & 1];  // carry_i ‖ summary_i
+    uint8_t* piece = d_pieces + i * piece_cap;
+    uint64_t* d_cnt = reinterpret_cast<uint64_t*>(piece + piece_cap - 16);
+    if ((st = lcf_dpratio_shard_summary(d_in + b0, bytes, in_bytes, w0, cur + sb, ws->stream)) ||
+        (st = lcf_dpratio_compress_shard(d_in + b0, bytes, in_bytes, w0, i ? cur : nullptr, piece,
+                                         piece + round16(4 * 2 * st_tiles), piece_cap - 16 - round16(4 * 2 * st_tiles),
+                                         d_cnt, ws->stream)))
+      return st;
+    if (i + 1 < k && (st = lcf_dpratio_merge_summaries(cur, 2, P[(i + 1) & 1], ws->stream))) return st;
+    if (!cuda_ok(cudaMemcpyAsync(cnt_h + i, d_cnt, 8, cudaMemcpyDeviceToHost, ws->stream)) ||
+        !cuda_ok(cudaEventRecord(evC[i], ws->stream)))
+      return LCF_ERROR_CUDA;
+    if (i >= 1 && (st = finish(i - 1))) return st;
+  }
+  if ((st = finish(k - 1))) return st;
+  put_header(h_out, LCF_DPRATIO, in_bytes, C, off - base);
+  std::memset(h_out + kHeaderBytes + 4 * C, 0, base - kHeaderBytes - 4 * C);
+  if (!cuda_ok(cudaStreamSynchronize(ws->d2h))) return LCF_ERROR_CUDA;
+  *out_bytes = off;
+  return LCF_SUCCESS;
+}
+
 // A failed pipelined call still has copies and kernels in flight on the
 // caller's buffers: drain all three streams before reporting, and consume the
 // device error word (slices already enqueued may have flagged too — this call
@@ -627,6 +705,16 @@ static lcf_status_t host_roundtrip(bool compress, lcf_algo_t algo, lcf_dtype_t d
   lcf_status_t st = LCF_SUCCESS;
   Workspace* ws = get_ws(stream, &st);
   if (!ws) return st;
+  if (algo == LCF_DPRATIO && dtype_matches(algo, dtype) && compress && in_bytes % 8 == 0 &&
+      in_bytes / 8 < (1ull << 31)) {
+    std::lock_guard<std::mutex> hg(ws->host_mu);
+    const uint64_t T = (in_bytes / 8 + 2047) / 2048;
+    const uint64_t st_tiles = host_slice_chunks(T);
+    if (T > st_tiles)
+      return host_pipe_done(ws, compress_host_dpratio_pipelined(static_cast<const uint8_t*>(h_in), in_bytes,
+                                                                static_cast<uint8_t*>(h_out), out_capacity, out_bytes,
+                                                                ws, st_tiles));
+  }
   if (algo == LCF_DPRATIO && dtype_matches(algo, dtype) && !compress && in_bytes >= kHeaderBytes) {
     std::lock_guard<std::mutex> hg(ws->host_mu);
     uint64_t nb, C, pay;

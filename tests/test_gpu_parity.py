@@ -253,6 +253,11 @@ def test_full_size_dpratio_stream(L, orc):
     assert s.numel() == len(ref)
     assert np.array_equal(s.cpu().numpy(), np.frombuffer(ref, np.uint8))
     assert torch.equal(L.decompress("DPratio", s), x)
+    # the host-buffer path compresses in tile slices with carried FCM state: the same bytes
+    hx = x.cpu().numpy().view(np.uint64)
+    hout = np.zeros(L.lcf_max_compressed_size("DPratio", None, hx.nbytes), np.uint8)
+    nh = L.lcf_compress_host("DPratio", None, hx, hx.nbytes, hout, hout.nbytes)
+    assert nh == len(ref) and hout[:nh].tobytes() == ref
     del x, s
     torch.cuda.empty_cache()
 

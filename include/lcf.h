@@ -61,6 +61,10 @@ size_t lcf_max_compressed_size(lcf_algo_t algo, lcf_dtype_t dtype, size_t in_byt
  * SP codecs need LCF_FLOAT32 and DP codecs LCF_FLOAT64 → else DTYPE_MISMATCH
  * (L41); out_capacity ≥ lcf_max_compressed_size(...) → else BUFFER_TOO_SMALL.
  * d_in must be 16-byte aligned. in_bytes = 0 yields the 32-byte header.
+ * DPratio only: fewer than 2^31 words (16 GiB) per call → else INVALID_ARGUMENT
+ * (its FCM sort records carry a 32-bit word index; the oracle has no such
+ * limit; larger arrays go through the sharded calls below, whose shards each
+ * stay under it).
  * Stages per 16 KiB chunk: SPspeed DIFFMS→MPLG (L108–118), SPratio
  * DIFFMS→BIT→RZE (L138–158), DPspeed DIFFMS→MPLG, DPratio FCM→DIFFMS→RAZE→RARE
  * (L168–201); raw fallback per chunk (L104); placement by a single-pass
@@ -145,16 +149,24 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  * 2048-word tiles, in array order:
  *  1. lcf_dpratio_shard_summary: the shard's summary — per hash, its last ≤ 4
  *     words (global index, value); lcf_dpratio_summary_bytes() bytes, device;
- *  2. the summaries are exchanged (e.g. an NCCL all-gather);
- *  3. lcf_dpratio_merge_summaries: shard g's carry from the summaries of shards
- *     0 … g−1, contiguous in shard order (count = g; count 0: an empty carry);
+ *  2. every shard's summary is made readable by the others (CUDA IPC over
+ *     NVLink: lcf_ipc_export / lcf_ipc_import below; on one device, plain
+ *     pointers), after a barrier;
+ *  3. lcf_dpratio_merge_summary_ptrs: shard g's carry from the summaries of
+ *     shards 0 … g−1 (d_summaries: host array of g device pointers in shard
+ *     order; count 0: an empty carry). Per hash it reads shard g−1's entries
+ *     first and goes further back only while fewer than 4 are found, so it
+ *     reads about one summary's worth, not g. lcf_dpratio_merge_summaries is
+ *     the same over g summaries stored contiguously;
  *  4. lcf_dpratio_compress_shard: the shard's 2 chunks per tile with that carry
  *     (NULL for shard 0), written like lcf_compress_shard: size-table slice,
  *     payload piece from offset 0, device u64 payload byte count.
  * The pieces assemble with lcf_write_header into exactly the 1-GPU stream.
  * d_x points at the shard's first word (global index first_word, a multiple
- * of 2048); the min(3, first_word) words before it must be readable (the hash
- * context of the shard's first words, L172). shard_bytes is a multiple of
+ * of 2048); the min(3, first_word) words before it must be readable and hold
+ * the array's words first_word − 3 … first_word − 1 (the hash context of the
+ * shard's first words, L172): a caller holding only its shard places the
+ * previous shard's last 3 words before it. shard_bytes is a multiple of
  * 16384 unless the shard ends the array. Errors as lcf_compress_shard.
  * lcf_dpratio_compress_shard right after lcf_dpratio_shard_summary of the same
  * shard (same d_x, size, first_word) on the same stream reuses the summary's
@@ -162,26 +174,59 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  *
  * Decompression of a shard: d_in is the shard's own LCF1 sub-stream (header
  * for its words, its size-table slice, its payload piece), whose word 0 is
- * global word first_word. Distances that stay in the shard are resolved (L197);
- * a word whose chain leaves the shard is left pending: d_out holds the global
- * index of the word it copies, and its bit in d_pending is set (u32 bitmap of
- * ceil(out_capacity / 8 / 32) words, cleared by the call). Asynchronous;
- * malformed input is reported by lcf_check_stream. lcf_dpratio_resolve_pending
- * then replaces every pending word by d_prefix[target], d_prefix holding the
- * final words of global indices [0, first_word) (device). Shards are resolved
- * in array order. */
+ * global word first_word. lcf_dpratio_decompress_shard decodes every tile and
+ * follows FCM chains inside a tile (L197); a word whose distance leaves its
+ * tile is read if that tile is already complete, else it is left PENDING:
+ * d_out holds the global index of the word it copies and its bit in
+ * d_pending is set (u32 bitmap of ceil(out_capacity / 8 / 32) words, fully
+ * written by the call). Asynchronous; malformed input is reported by
+ * lcf_check_stream. The pending words are then resolved over all shards, each
+ * described by an lcf_dp_view (its words and bitmap — local pointers or
+ * CUDA-IPC-mapped peer pointers; views sorted by first_word, contiguous from
+ * word 0, ≤ 64 of them; `self` is the caller's shard, whose first_word is a
+ * multiple of 32):
+ *  a. every shard's lcf_dpratio_decompress_shard has completed (barrier);
+ *  b. lcf_dpratio_find_roots(self): each pending word of shard `self` follows
+ *     its chain through the views to the first word that is not pending (its
+ *     root) and stores the root's global index (L197's union-find "find",
+ *     with path compression; only ancestor indices are ever stored, so shards
+ *     may run this concurrently);
+ *  c. every shard's find_roots has completed (barrier);
+ *  d. lcf_dpratio_gather_roots(self): each pending word of `self` takes its
+ *     root's value and the bitmap is cleared.
+ * After d on every shard (barrier), the words are final. A chain that points
+ * forwards, or outside the views, is reported as CORRUPT_STREAM. */
+typedef struct {
+  uint64_t first_word;  /* global index of the view's word 0 */
+  uint64_t n_words;     /* words in the view */
+  void* d_words;        /* its decoded words (u64), device */
+  uint32_t* d_pending;  /* its pending bitmap, device */
+} lcf_dp_view;
 size_t lcf_dpratio_summary_bytes(void);
 lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,
                                        void* d_summary, void* stream);
 lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream);
+lcf_status_t lcf_dpratio_merge_summary_ptrs(const void* const* d_summaries, size_t count, void* d_carry,
+                                            void* stream);
 lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, size_t total_in_bytes,
                                         uint64_t first_word, const void* d_carry, void* d_table_slice,
                                         void* d_payload, size_t payload_capacity, uint64_t* d_payload_bytes,
                                         void* stream);
 lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uint64_t first_word, void* d_out,
                                           size_t out_capacity, uint32_t* d_pending, void* stream);
-lcf_status_t lcf_dpratio_resolve_pending(void* d_out, size_t shard_bytes, const uint32_t* d_pending,
-                                         const void* d_prefix, void* stream);
+lcf_status_t lcf_dpratio_find_roots(const lcf_dp_view* views, size_t count, size_t self, void* stream);
+lcf_status_t lcf_dpratio_gather_roots(const lcf_dp_view* views, size_t count, size_t self, void* stream);
+
+/* CUDA IPC plumbing for the sharded modes (one process per GPU on one node):
+ * lcf_ipc_export writes a 64-byte handle of the device allocation holding
+ * d_ptr and d_ptr's offset inside it; another process passes both to
+ * lcf_ipc_import and gets a device pointer to the same bytes (over NVLink when
+ * the GPUs differ), valid until lcf_ipc_close. A process cannot import its
+ * own export (use its pointer). Errors: INVALID_ARGUMENT (null / unknown
+ * pointer), CUDA (the driver refused). */
+lcf_status_t lcf_ipc_export(const void* d_ptr, void* handle64, uint64_t* offset);
+lcf_status_t lcf_ipc_import(const void* handle64, uint64_t offset, void** d_ptr);
+lcf_status_t lcf_ipc_close(void* d_ptr);
 
 /* Number of kernel launches the library enqueued since the process started
  * (bench/test accounting). */

@@ -6,6 +6,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <string>
 #include <mutex>
 #include <utility>
 #include <vector>
@@ -29,6 +30,9 @@ struct Workspace {
   size_t status_cap = 0;
   uint32_t* tile_flag = nullptr;         // DPratio decode tile completion flags
   size_t tile_cap = 0;
+  uint32_t* pend = nullptr;              // DPratio decode pending-word bitmap (1 bit per word)
+  size_t pend_cap = 0;
+  uint32_t* any_pend = nullptr;          // DPratio decode: epoch of the newest launch with a pending word
   uint32_t* err = nullptr;               // (epoch << 8 | bits) of the newest failure
   uint32_t epoch = 0, checked_epoch = 0;
   void* scratch[4] = {nullptr, nullptr, nullptr, nullptr};  // grown on demand
@@ -64,7 +68,8 @@ Workspace* get_ws(cudaStream_t stream, lcf_status_t* st) {
   ws->device = dev;
   ws->stream = stream;
   if (!cuda_ok(cudaMalloc(&ws->ticket, 2 * sizeof(unsigned long long))) ||
-      !cuda_ok(cudaMalloc(&ws->err, sizeof(uint32_t))) ||
+      !cuda_ok(cudaMalloc(&ws->err, sizeof(uint32_t))) || !cuda_ok(cudaMalloc(&ws->any_pend, sizeof(uint32_t))) ||
+      !cuda_ok(cudaMemsetAsync(ws->any_pend, 0, sizeof(uint32_t), stream)) ||
       !cuda_ok(cudaMemsetAsync(ws->ticket, 0, 2 * sizeof(unsigned long long), stream)) ||
       !cuda_ok(cudaMemsetAsync(ws->err, 0, sizeof(uint32_t), stream))) {
     *st = LCF_ERROR_OUT_OF_MEMORY;
@@ -95,6 +100,7 @@ uint32_t next_epoch(Workspace* ws) {
   if (++ws->epoch >= kEpochLimit) {  // wrap: forget every status/flag word
     if (ws->status) cudaMemsetAsync(ws->status, 0, ws->status_cap * sizeof(uint64_t), ws->stream);
     if (ws->tile_flag) cudaMemsetAsync(ws->tile_flag, 0, ws->tile_cap * sizeof(uint32_t), ws->stream);
+    if (ws->any_pend) cudaMemsetAsync(ws->any_pend, 0, sizeof(uint32_t), ws->stream);
     cudaMemsetAsync(ws->err, 0, sizeof(uint32_t), ws->stream);
     ws->epoch = 1;
     ws->checked_epoch = 0;
@@ -277,6 +283,28 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
   return LCF_SUCCESS;
 }
 
+// The DPratio decode of tiles [first_tile, end_tile) (end 0: all) of the stream
+// at a.stream into a.out: the tile decoder, then the root resolution of the
+// words it left pending (single view: the whole output). Caller holds ws->mu.
+static lcf_status_t dpratio_decode_range(Workspace* ws, DecArgs a, const LaunchCtx& ctx, uint64_t max_tiles,
+                                         uint64_t end_tile, cudaStream_t stream) {
+  const uint64_t words = a.out_capacity / 8;
+  lcf_status_t st;
+  if ((st = grow(ws->pend, ws->pend_cap, (words + 31) / 32 + 1, stream, true))) return st;
+  a.pend = ws->pend;
+  a.any_pend = ws->any_pend;
+  launch_dpratio_decode(a, ctx, max_tiles, stream);
+  DpViews v{};
+  v.count = 1;
+  v.self = 0;
+  v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend};
+  const uint64_t lo = a.first_tile * 2048, hi = end_tile ? end_tile * 2048 : words;
+  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream);
+  launch_dp_gather_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream);
+  g_launches += 2;
+  return LCF_SUCCESS;
+}
+
 lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, size_t in_bytes, void* d_out,
                             size_t out_capacity, size_t* out_bytes, void* stream_) {
   cudaStream_t stream = (cudaStream_t)stream_;
@@ -327,7 +355,9 @@ lcf_status_t lcf_decompress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in
     case LCF_SPSPEED: launch_speed_decode<uint32_t>(a, ctx, grid, stream); break;
     case LCF_DPSPEED: launch_speed_decode<uint64_t>(a, ctx, grid, stream); break;
     case LCF_SPRATIO: launch_spratio_decode(a, ctx, grid, stream); break;
-    case LCF_DPRATIO: launch_dpratio_decode(a, ctx, grid / 2 + 1, stream); break;
+    case LCF_DPRATIO:
+      if ((st = dpratio_decode_range(ws, a, ctx, grid / 2 + 1, 0, stream))) return st;
+      break;
     default: return LCF_ERROR_INVALID_ARGUMENT;
   }
   ++g_launches;
@@ -589,7 +619,7 @@ static lcf_status_t decompress_host_dpratio_pipelined(const uint8_t* h_in, size_
       a.end_tile = t1;
       a.base_off = off;
       LaunchCtx ctx = make_ctx(ws);
-      launch_dpratio_decode(a, ctx, t1 - t0, ws->stream);
+      if ((st = dpratio_decode_range(ws, a, ctx, t1 - t0, t1, ws->stream))) return st;
       ++g_launches;
       if ((st = last_launch_status())) return st;
     }
@@ -639,7 +669,7 @@ static lcf_status_t compress_host_dpratio_pipelined(const uint8_t* h_in, size_t 
   cudaEvent_t* evH = ws->ev.data();
   cudaEvent_t* evC = ws->ev.data() + k;
   uint64_t* cnt_h = reinterpret_cast<uint64_t*>(ws->hstage);
-  if (!cuda_ok(cudaMemsetAsync(P[0], 0, 1u << 20, ws->stream))) return LCF_ERROR_CUDA;  // empty carry of slice 0
+  if (!fcm_empty_carry(P[0], ws->stream)) return LCF_ERROR_CUDA;  // slice 0 has no earlier slices
   uint64_t off = base;
   auto finish = [&](uint64_t i) -> lcf_status_t {
     const uint64_t t0 = i * st_tiles, nt = (t0 + st_tiles < T ? st_tiles : T - t0);
@@ -855,11 +885,86 @@ lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size
   return LCF_SUCCESS;
 }
 
-lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream_) {
+lcf_status_t lcf_dpratio_merge_summary_ptrs(const void* const* d_summaries, size_t count, void* d_carry,
+                                            void* stream_) {
   cudaStream_t stream = (cudaStream_t)stream_;
-  if (!d_carry || (count && !d_summaries) || count > 0xFFFFFFFFull) return LCF_ERROR_INVALID_ARGUMENT;
+  if (!d_carry || (count && !d_summaries) || count > 64) return LCF_ERROR_INVALID_ARGUMENT;
+  for (size_t r = 0; r < count; ++r)
+    if (!d_summaries[r]) return LCF_ERROR_INVALID_ARGUMENT;
   g_launches += launch_fcm_carry_merge(d_summaries, (uint32_t)count, d_carry, stream);
   return last_launch_status();
+}
+
+lcf_status_t lcf_dpratio_merge_summaries(const void* d_summaries, size_t count, void* d_carry, void* stream) {
+  if (!d_carry || (count && !d_summaries) || count > 64) return LCF_ERROR_INVALID_ARGUMENT;
+  const void* p[64];
+  for (size_t r = 0; r < count; ++r) p[r] = static_cast<const uint8_t*>(d_summaries) + r * fcm_carry_bytes();
+  return lcf_dpratio_merge_summary_ptrs(p, count, d_carry, stream);
+}
+
+// ---- CUDA IPC plumbing (include/lcf.h) ---------------------------------------
+// The export handle covers the whole allocation holding d_ptr (found with the
+// driver's cuMemGetAddressRange, fetched at run time so that the library
+// needs no link-time libcuda); the importer adds the offset back.
+namespace {
+typedef int (*AddrRangeFn)(unsigned long long*, size_t*, unsigned long long);
+std::mutex g_ipc_mu;
+// several tensors of one peer allocation map it once (the driver maps a
+// handle once per process): handle bytes → (base, imports); pointer → handle
+std::map<std::string, std::pair<void*, int>> g_ipc_maps;
+std::multimap<void*, std::string> g_ipc_ptrs;
+}  // namespace
+
+lcf_status_t lcf_ipc_export(const void* d_ptr, void* handle64, uint64_t* offset) {
+  if (!d_ptr || !handle64 || !offset) return LCF_ERROR_INVALID_ARGUMENT;
+  static AddrRangeFn range = [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      fn = nullptr;
+    return reinterpret_cast<AddrRangeFn>(fn);
+  }();
+  if (!range) return LCF_ERROR_CUDA;
+  unsigned long long base = 0;
+  size_t size = 0;
+  if (range(&base, &size, (unsigned long long)(uintptr_t)d_ptr) != 0) return LCF_ERROR_INVALID_ARGUMENT;
+  cudaIpcMemHandle_t h;
+  if (!cuda_ok(cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base)))) return LCF_ERROR_CUDA;
+  static_assert(sizeof(h) == 64, "64-byte IPC handle");
+  memcpy(handle64, &h, 64);
+  *offset = (uint64_t)((uintptr_t)d_ptr - base);
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_ipc_import(const void* handle64, uint64_t offset, void** d_ptr) {
+  if (!handle64 || !d_ptr) return LCF_ERROR_INVALID_ARGUMENT;
+  const std::string key(static_cast<const char*>(handle64), 64);
+  std::lock_guard<std::mutex> g(g_ipc_mu);
+  auto it = g_ipc_maps.find(key);
+  if (it == g_ipc_maps.end()) {
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle64, 64);
+    void* base = nullptr;
+    if (!cuda_ok(cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess))) return LCF_ERROR_CUDA;
+    it = g_ipc_maps.emplace(key, std::make_pair(base, 0)).first;
+  }
+  ++it->second.second;
+  *d_ptr = static_cast<uint8_t*>(it->second.first) + offset;
+  g_ipc_ptrs.emplace(*d_ptr, key);
+  return LCF_SUCCESS;
+}
+
+lcf_status_t lcf_ipc_close(void* d_ptr) {
+  std::lock_guard<std::mutex> g(g_ipc_mu);
+  auto p = g_ipc_ptrs.find(d_ptr);
+  if (p == g_ipc_ptrs.end()) return LCF_ERROR_INVALID_ARGUMENT;
+  auto it = g_ipc_maps.find(p->second);
+  g_ipc_ptrs.erase(p);
+  if (--it->second.second > 0) return LCF_SUCCESS;
+  void* base = it->second.first;
+  g_ipc_maps.erase(it);
+  return cuda_ok(cudaIpcCloseMemHandle(base)) ? LCF_SUCCESS : LCF_ERROR_CUDA;
 }
 
 lcf_status_t lcf_dpratio_compress_shard(const void* d_x, size_t shard_bytes, size_t total_in_bytes,
@@ -927,19 +1032,51 @@ lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uin
   a.tile_flag = ws->tile_flag;
   a.gbase = first_word;
   a.pend = d_pending;
+  a.any_pend = ws->any_pend;
   LaunchCtx ctx = make_ctx(ws);
   launch_dpratio_decode(a, ctx, grid / 2 + 1, stream);
   ++g_launches;
   return last_launch_status();
 }
 
-lcf_status_t lcf_dpratio_resolve_pending(void* d_out, size_t shard_bytes, const uint32_t* d_pending,
-                                         const void* d_prefix, void* stream_) {
-  if (shard_bytes % 8 || (shard_bytes && (!d_out || !d_pending || !d_prefix))) return LCF_ERROR_INVALID_ARGUMENT;
-  launch_dp_resolve_pending(static_cast<uint64_t*>(d_out), shard_bytes / 8, d_pending,
-                            static_cast<const uint64_t*>(d_prefix), (cudaStream_t)stream_);
-  ++g_launches;
+// The views of lcf_dpratio_find_roots / gather_roots (include/lcf.h).
+static lcf_status_t dp_views(const lcf_dp_view* views, size_t count, size_t self, DpViews& v) {
+  if (!views || count == 0 || count > kMaxViews || self >= count) return LCF_ERROR_INVALID_ARGUMENT;
+  v.count = (uint32_t)count;
+  v.self = (uint32_t)self;
+  for (size_t q = 0; q < count; ++q) {
+    const lcf_dp_view& w = views[q];
+    if (q ? w.first_word != views[q - 1].first_word + views[q - 1].n_words : w.first_word != 0)
+      return LCF_ERROR_INVALID_ARGUMENT;  // sorted, contiguous from word 0
+    if (w.n_words && (!w.d_words || !w.d_pending)) return LCF_ERROR_INVALID_ARGUMENT;
+    v.v[q] = DpView{w.first_word, w.n_words, static_cast<uint64_t*>(w.d_words), w.d_pending};
+  }
+  if (views[self].first_word % 32) return LCF_ERROR_INVALID_ARGUMENT;
+  return LCF_SUCCESS;
+}
+
+static lcf_status_t dp_roots(const lcf_dp_view* views, size_t count, size_t self, void* stream_, bool gather) {
+  cudaStream_t stream = (cudaStream_t)stream_;
+  DpViews v{};
+  if (lcf_status_t s = dp_views(views, count, self, v)) return s;
+  lcf_status_t st = LCF_SUCCESS;
+  Workspace* ws = get_ws(stream, &st);
+  if (!ws) return st;
+  std::lock_guard<std::mutex> g(ws->mu);
+  LaunchCtx ctx = make_ctx(ws);
+  const uint64_t n = views[self].n_words;
+  if (gather) launch_dp_gather_roots(v, nullptr, 0, n, ctx, nullptr, stream);
+  else launch_dp_find_roots(v, nullptr, 0, n, ctx, nullptr, stream);
+  if (n) ++g_launches;
   return last_launch_status();
+}
+
+lcf_status_t lcf_dpratio_find_roots(const lcf_dp_view* views, size_t count, size_t self, void* stream) {
+  return dp_roots(views, count, self, stream, false);
+}
+
+lcf_status_t lcf_dpratio_gather_roots(const lcf_dp_view* views, size_t count, size_t self, void* stream) {
+  return dp_roots(views, count, self, stream, true);
 }
 
 lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_in_bytes,

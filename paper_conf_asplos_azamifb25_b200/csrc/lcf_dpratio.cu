@@ -721,7 +721,7 @@ struct DDecSmem {
 struct FcmScratch {  // pointer jumping (aliases S.rz)
   int32_t pj[2][kDT];  // target (−1 done)
   uint64_t vj[2][kDT];
-  uint8_t fj[2][kDT];  // shard decode: value is a pending global target
+  uint8_t fj[2][kDT];  // value is a pending global target
 };
 static_assert(sizeof(FcmScratch) <= kChunkBytes, "FCM scratch fits in rz");
 
@@ -851,7 +851,6 @@ __device__ __forceinline__ bool raze_diffms_inv(const uint8_t* rz, uint32_t off,
   return true;
 }
 
-template <bool SHARD>
 __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t tid) {
   const uint32_t lane = tid & 31;
   const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
@@ -955,17 +954,24 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
     if (tid == 0) trace_stamp(a, t, 4);
     if (tid == 0) trace_stamp(a, t, 5);
     // ---- FCM decode of the tile (L197): x[i] = Dist[i] ? x[i − Dist[i]] : V[i] ----
+    // Chains inside the tile are followed here (pointer jumping in shared
+    // memory). A reference into an earlier tile is read if that tile is
+    // complete; otherwise — and for a word before the stream's first word
+    // (shard decode) — the word is left PENDING: it holds the global index it
+    // copies and its bit is set in a.pend. No tile ever waits for another:
+    // dp_find_roots / dp_gather_roots (below) resolve the pending words after
+    // this kernel, so long cross-tile chains (a value repeated row after row)
+    // cost pointer jumps instead of a tile-by-tile serial dependency.
     bool bad = !ok;
+    const uint64_t gb = a.gbase;  // global index of this stream's word 0
     if (ok && nzD) {  // (no distances: x = V as it stands)
-      if (SHARD)
-        for (uint32_t w = tid; w < kTileWords / 32; w += kDT) S.pmask[w] = 0;
+      for (uint32_t w = tid; w < kTileWords / 32; w += kDT) S.pmask[w] = 0;
       bar_d();  // X complete (V's DIFFMS⁻¹ ends without a barrier)
-      const uint64_t gb = SHARD ? a.gbase : 0;  // global index of this stream's word 0
       for (uint32_t b = 0; b < m; b += kDT) {  // 256-element blocks in index order
         const uint32_t li = b + tid;
         int32_t p = -1;
         uint64_t val = 0;
-        uint8_t f = 0;  // (shard decode) val is a pending global target
+        uint8_t f = 0;  // val is a pending global target
         if (li < m) {
           const uint64_t d = Dw[li], gi = gb + t0 + li;
           if (d == 0) {
@@ -976,13 +982,19 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
             p = (int32_t)(gi - d - gb - t0 - b);  // inside this block: resolve below
           } else if (gi - d >= gb + t0) {
             const uint32_t lj = (uint32_t)(gi - d - gb - t0);
-            val = S.X[lj];  // earlier block of this tile: already final (or pending)
-            if (SHARD) f = (S.pmask[lj / 32] >> (lj % 32)) & 1;
-          } else if (!SHARD || gi - d >= gb) {  // earlier tile: wait for its flag, then read the output
-            const uint64_t j = gi - d - gb, tj = j / kTileWords;  // (tiles before first_tile: final already)
-            while (tj >= a.first_tile && ld_acquire_u32(a.tile_flag + tj) != ctx.epoch) __nanosleep(100);
-            val = ld_cg_u64(out + j);
-            if (SHARD) f = (__ldcg(a.pend + j / 32) >> (j % 32)) & 1;
+            val = S.X[lj];  // earlier block of this tile: final or pending
+            f = (S.pmask[lj / 32] >> (lj % 32)) & 1;
+          } else if (gi - d >= gb) {  // earlier tile of this stream
+            const uint64_t j = gi - d - gb, tj = j / kTileWords;
+            if (tj < a.first_tile) {  // an earlier launch on this stream: final
+              val = ld_cg_u64(out + j);
+            } else if (ld_acquire_u32(a.tile_flag + tj) == ctx.epoch) {  // complete: final or pending
+              val = ld_cg_u64(out + j);
+              f = (__ldcg(a.pend + j / 32) >> (j % 32)) & 1;
+            } else {  // still in flight: pending on it
+              val = gi - d;
+              f = 1;
+            }
           } else {  // before the shard: pending on the global word gi − d
             val = gi - d;
             f = 1;
@@ -992,13 +1004,13 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
         uint32_t par = 0;
         F.pj[0][tid] = p;
         F.vj[0][tid] = val;
-        if (SHARD) F.fj[0][tid] = f;
+        F.fj[0][tid] = f;
         while (bar_d_or(p >= 0)) {
           if (p >= 0) {
             const int32_t q = F.pj[par][p];
             if (q < 0) {
               val = F.vj[par][p];
-              if (SHARD) f = F.fj[par][p];
+              f = F.fj[par][p];
               p = -1;
             } else {
               p = q;
@@ -1006,16 +1018,22 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
           }
           F.pj[par ^ 1][tid] = p;
           F.vj[par ^ 1][tid] = val;
-          if (SHARD) F.fj[par ^ 1][tid] = f;
+          F.fj[par ^ 1][tid] = f;
           par ^= 1;
         }
-        if (li < m) S.X[li] = val;  // x, in place
-        if (SHARD && li < m && f) atomicOr(&S.pmask[li / 32], 1u << (li % 32));
+        if (li < m) S.X[li] = val;  // x (or a pending target), in place
+        if (li < m && f) atomicOr(&S.pmask[li / 32], 1u << (li % 32));
         bar_d();
       }
-      if (SHARD)  // the tile's pending bits, before its completion flag (released after a barrier)
-        for (uint32_t w = tid; w < (m + 31) / 32; w += kDT) a.pend[t0 / 32 + w] = S.pmask[w];
+      // the tile's pending bits, before its completion flag (released after a barrier)
+      for (uint32_t w = tid; w < (m + 31) / 32; w += kDT) {
+        const uint32_t pm = bad ? 0u : S.pmask[w];
+        a.pend[t0 / 32 + w] = pm;
+        if (pm) st_relaxed_u32(a.any_pend, ctx.epoch);  // some word of this launch is pending
+      }
       release(&S.empty_d[0]);
+    } else {
+      for (uint32_t w = tid; w < (m + 31) / 32; w += kDT) a.pend[t0 / 32 + w] = 0;
     }
     if (tid == 0) trace_stamp(a, t, 6);
     fence_proxy_async_smem();  // S.X (generic-proxy writes) → the bulk store
@@ -1035,7 +1053,6 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   }
 }
 
-template <bool SHARD>
 __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DDecSmem& S = *reinterpret_cast<DDecSmem*>(smem_raw);
@@ -1049,7 +1066,7 @@ __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs
   }
   __syncthreads();
   if (warp == 0) d_dec_loader(S, a, ctx, lane);
-  else d_dec_compute<SHARD>(S, a, ctx, threadIdx.x - 32);
+  else d_dec_compute(S, a, ctx, threadIdx.x - 32);
 }
 
 }  // namespace
@@ -1082,35 +1099,118 @@ int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, siz
 }
 
 namespace {
-// Pending words of a decoded shard take the final word of their global target
-// (prefix: the words before the shard, final).
-__global__ void __launch_bounds__(256) dp_resolve_pending_kernel(uint64_t* __restrict__ out, uint64_t n,
-                                                                const uint32_t* __restrict__ pend,
-                                                                const uint64_t* __restrict__ prefix) {
-  for (uint64_t i = blockIdx.x * 256ull + threadIdx.x; i < n; i += (uint64_t)gridDim.x * 256)
-    if ((pend[i / 32] >> (i % 32)) & 1) out[i] = prefix[out[i]];
+// ---- root resolution of pending words (L197's union-find "find") ----------------
+// After the tile decoder, a pending word holds the global index of the word it
+// copies (always a smaller index). dp_find_roots follows each pending word's
+// chain to its root — the first word on it that is not pending — and stores
+// the root index in the word, writing the partial result back every few hops
+// so that walks through it jump further (path compression, as the paper's
+// decoder shortens chains for other threads). Every stored index is an
+// ancestor on the chain, so a concurrent walker reading an old or a new value
+// stays correct; no value is written until dp_gather_roots, after every walk
+// has ended. Grid-stride in index order: earlier words are compressed first.
+__device__ __forceinline__ int dp_owner(const DpViews& V, uint64_t g) {
+  int q = (int)V.self;
+  while (q > 0 && g < V.v[q].first) --q;
+  return q;
+}
+
+__device__ __forceinline__ uint64_t dp_hi(const DpViews& V, const uint8_t* stream, uint64_t w_hi) {
+  const DpView& me = V.v[V.self];
+  uint64_t hi = w_hi < me.n ? w_hi : me.n;
+  if (stream) {  // the stream's word count (a malformed header was reported by the decoder)
+    const uint64_t nw = reinterpret_cast<const uint64_t*>(stream)[1] / 8;
+    hi = hi < nw ? hi : nw;
+  }
+  return hi;
+}
+
+__global__ void __launch_bounds__(256) dp_find_roots_kernel(const __grid_constant__ DpViews V, const uint8_t* stream,
+                                                           uint64_t w_lo, uint64_t w_hi, LaunchCtx ctx,
+                                                           const uint32_t* any_pend) {
+  if (any_pend && *any_pend != ctx.epoch) return;
+  const DpView& me = V.v[V.self];
+  const uint64_t hi = dp_hi(V, stream, w_hi);
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint64_t base = w_lo + (blockIdx.x * 256ull + threadIdx.x - lane); base < hi; base += gridDim.x * 256ull) {
+    const uint32_t bits = __ldcg(me.pend + base / 32);  // one bitmap word per warp (w_lo % 32 == 0)
+    const uint64_t li = base + lane;
+    if (!((bits >> lane) & 1) || li >= hi) continue;
+    uint64_t cur = me.first + li, t = __ldcg(me.out + li);
+    uint32_t hops = 0;
+    bool err = false;
+    for (;;) {
+      if (t >= cur) { err = true; break; }  // chains point strictly backwards
+      const DpView& w = V.v[dp_owner(V, t)];
+      if (t < w.first || t - w.first >= w.n) { err = true; break; }
+      const uint64_t lj = t - w.first;
+      if (!((ld_relaxed_sys_u32(w.pend + lj / 32) >> (lj % 32)) & 1)) break;  // final: the root
+      cur = t;
+      t = ld_relaxed_sys_u64(w.out + lj);
+      if ((++hops & 3) == 0) st_relaxed_sys_u64(me.out + li, t);
+    }
+    if (err) record_error(ctx, DERR_CORRUPT);
+    else st_relaxed_sys_u64(me.out + li, t);
+  }
+}
+
+// Pending words take their root's value (roots are never pending, so nothing
+// read here is being written); each bitmap word is cleared by its warp.
+__global__ void __launch_bounds__(256) dp_gather_roots_kernel(const __grid_constant__ DpViews V,
+                                                             const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                                                             LaunchCtx ctx, const uint32_t* any_pend) {
+  if (any_pend && *any_pend != ctx.epoch) return;
+  const DpView& me = V.v[V.self];
+  const uint64_t hi = dp_hi(V, stream, w_hi);
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint64_t base = w_lo + (blockIdx.x * 256ull + threadIdx.x - lane); base < hi; base += gridDim.x * 256ull) {
+    const uint32_t bits = __ldcg(me.pend + base / 32);
+    if (!bits) continue;  // warp-uniform
+    const uint64_t li = base + lane;
+    if (((bits >> lane) & 1) && li < hi) {
+      const uint64_t r = __ldcg(me.out + li);
+      const DpView& w = V.v[dp_owner(V, r)];
+      if (r >= me.first + li || r < w.first || r - w.first >= w.n) record_error(ctx, DERR_CORRUPT);
+      else me.out[li] = ld_relaxed_sys_u64(w.out + (r - w.first));
+    }
+    __syncwarp();
+    if (lane == 0) me.pend[base / 32] = 0;
+  }
+}
+
+int roots_grid(const void* kern, uint64_t words) {
+  const uint64_t cap = (uint64_t)resident_capacity(kern, 256, 0);
+  const uint64_t need = (words + 255) / 256;
+  return (int)(need < cap ? (need ? need : 1) : cap);
 }
 }  // namespace
 
-void launch_dp_resolve_pending(uint64_t* out, uint64_t n, const uint32_t* pend, const uint64_t* prefix,
-                               cudaStream_t st) {
-  if (!n) return;
-  KTrace kt("dpratio_resolve_pending", st);
-  dp_resolve_pending_kernel<<<(unsigned)umin64((n + 255) / 256, 148 * 16), 256, 0, st>>>(out, n, pend, prefix);
+void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
+  if (w_hi <= w_lo) return;
+  KTrace kt("dp_find_roots", st);
+  dp_find_roots_kernel<<<roots_grid((const void*)dp_find_roots_kernel, w_hi - w_lo), 256, 0, st>>>(
+      v, stream, w_lo, w_hi, ctx, any_pend);
+}
+
+void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
+  if (w_hi <= w_lo) return;
+  KTrace kt("dp_gather_roots", st);
+  dp_gather_roots_kernel<<<roots_grid((const void*)dp_gather_roots_kernel, w_hi - w_lo), 256, 0, st>>>(
+      v, stream, w_lo, w_hi, ctx, any_pend);
 }
 
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st) {
   const size_t smem = sizeof(DDecSmem);
   static const bool init = [&] {
-    cudaFuncSetAttribute(dpratio_decode_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(dpratio_decode_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(dpratio_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     return true;
   }();
   (void)init;
-  const int grid = persistent_grid(dpratio_decode_kernel<false>, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
+  const int grid = persistent_grid(dpratio_decode_kernel, kDDecThreads, smem, (max_tiles + kDBatch - 1) / kDBatch);
   KTrace kt("dpratio_decode", st);
-  if (a.pend) dpratio_decode_kernel<true><<<grid, kDDecThreads, smem, st>>>(a, ctx);
-  else dpratio_decode_kernel<false><<<grid, kDDecThreads, smem, st>>>(a, ctx);
+  dpratio_decode_kernel<<<grid, kDDecThreads, smem, st>>>(a, ctx);
 }
 
 }  // namespace lcf

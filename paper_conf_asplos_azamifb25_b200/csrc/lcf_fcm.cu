@@ -508,18 +508,22 @@ __global__ void __launch_bounds__(256) fcm_summary_kernel(const uint64_t* __rest
 }
 
 // Carry of shard g: per hash, walk the summaries of shards g−1, g−2, … 0 and
-// keep the first four entries (most recent first).
-__global__ void __launch_bounds__(256) fcm_carry_merge_kernel(const uint8_t* __restrict__ sums, uint32_t count,
+// keep the first four entries (most recent first). The summaries are read
+// through pointers (local, or peers' mapped by CUDA IPC): a hash whose four
+// entries come from shard g−1 never touches the older summaries.
+struct SumPtrs {
+  const uint8_t* p[64];
+};
+__global__ void __launch_bounds__(256) fcm_carry_merge_kernel(const __grid_constant__ SumPtrs S, uint32_t count,
                                                              uint8_t* __restrict__ out) {
   const uint64_t h = blockIdx.x * 256ull + threadIdx.x;
   if (h >= kHashes) return;
-  auto cnt_of = [&](const uint8_t* b) { return b; };
   auto idx_of = [&](const uint8_t* b) { return reinterpret_cast<const uint32_t*>(b + kHashes); };
   auto val_of = [&](const uint8_t* b) { return reinterpret_cast<const uint64_t*>(b + kHashes * 17); };
   uint32_t m = 0;
   for (int32_t r = (int32_t)count - 1; r >= 0 && m < 4; --r) {
-    const uint8_t* b = sums + (uint64_t)r * carry_bytes();
-    const uint32_t c = cnt_of(b)[h];
+    const uint8_t* b = S.p[r];
+    const uint32_t c = b[h];
     for (uint32_t q = 0; q < c && m < 4; ++q, ++m) {
       reinterpret_cast<uint32_t*>(out + kHashes)[4 * h + m] = idx_of(b)[4 * h + q];
       reinterpret_cast<uint64_t*>(out + kHashes * 17)[4 * h + m] = val_of(b)[4 * h + q];
@@ -537,6 +541,10 @@ size_t fcm_dist_workspace(uint64_t n) {
 }
 
 size_t fcm_carry_bytes() { return carry_bytes(); }
+
+// An empty carry (no earlier shard): every per-hash count is 0; the index and
+// value areas are never read for a count of 0.
+bool fcm_empty_carry(void* carry, cudaStream_t st) { return cudaMemsetAsync(carry, 0, kHashes, st) == cudaSuccess; }
 
 // The FCM distances of x[0, n) (sharded: a shard whose words x[−halo, 0)
 // precede it and whose first word has global index gbase; carry = the merged
@@ -619,10 +627,11 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
   return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out, false);
 }
 
-int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st) {
+int launch_fcm_carry_merge(const void* const* summaries, uint32_t count, void* carry, cudaStream_t st) {
+  SumPtrs S{};
+  for (uint32_t r = 0; r < count && r < 64; ++r) S.p[r] = static_cast<const uint8_t*>(summaries[r]);
   KTrace kt("fcm_carry_merge", st);
-  fcm_carry_merge_kernel<<<(unsigned)(kHashes / 256), 256, 0, st>>>(static_cast<const uint8_t*>(summaries), count,
-                                                                    static_cast<uint8_t*>(carry));
+  fcm_carry_merge_kernel<<<(unsigned)(kHashes / 256), 256, 0, st>>>(S, count, static_cast<uint8_t*>(carry));
   return 1;
 }
 

@@ -73,11 +73,29 @@ struct DecArgs {
   // 2·first_tile; earlier tiles are already final in `out` (an earlier launch
   // on the same stream) and only their payload bytes may be absent.
   uint64_t first_tile, end_tile, base_off;
-  // DPratio shard decode (NEXT-1): word 0 of this stream is global word gbase;
-  // a distance reaching before it is left pending: the output holds the global
-  // target index and `pend` (1 bit per word, zeroed) marks the word.
+  // DPratio: word 0 of this stream is global word gbase (0, or a shard's first
+  // word, NEXT-1). A word whose distance reaches before it, or into a tile not
+  // yet complete, is left pending: the output holds the global index it
+  // copies and its bit in `pend` (1 bit per word; every decoded tile writes
+  // its bitmap words) is set; any_pend ← epoch if any word is.
   uint64_t gbase;
   uint32_t* pend;
+  uint32_t* any_pend;
+};
+
+// The pending-word views of the DPratio root resolution (dp_find_roots /
+// dp_gather_roots in lcf_dpratio.cu): view q covers global words
+// [first, first + n) at `out` with bitmap `pend` (device pointers, local or
+// CUDA-IPC-mapped peers), sorted by first and contiguous.
+constexpr uint32_t kMaxViews = 64;
+struct DpView {
+  uint64_t first, n;
+  uint64_t* out;
+  uint32_t* pend;
+};
+struct DpViews {
+  uint32_t count, self;
+  DpView v[kMaxViews];
 };
 
 struct DecChunk {
@@ -166,13 +184,25 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
 // earlier shards (carry, nullable); `summary` (nullable) receives this
 // shard's summary (fcm_carry_bytes() bytes); match = false: summary only.
 size_t fcm_carry_bytes();
+bool fcm_empty_carry(void* carry, cudaStream_t st);
 int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
                      bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist, bool sorted = false);
-int launch_fcm_carry_merge(const void* summaries, uint32_t count, void* carry, cudaStream_t st);
+// summaries: host array of `count` (≤ 64) device pointers, shard order
+int launch_fcm_carry_merge(const void* const* summaries, uint32_t count, void* carry, cudaStream_t st);
 size_t dpratio_fcm_workspace(uint64_t n_words);
 int launch_dpratio_encode(const EncArgs& a, const LaunchCtx& ctx, void* ws, size_t ws_bytes, cudaStream_t st,
                           uint32_t halo = 0, uint64_t gbase = 0, const void* carry = nullptr, bool sorted = false);
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st);
-void launch_dp_resolve_pending(uint64_t* out, uint64_t n, const uint32_t* pend, const uint64_t* prefix, cudaStream_t st);
+// Root resolution of pending words of view `self`, local words [w_lo, w_hi)
+// (clamped to the stream header's word count when `stream` is given).
+// find: every pending word's target becomes its chain's root (a final word),
+// with path compression; gather: pending words take their root's value and
+// their bits are cleared. Every view's decode must be complete before any
+// find, and every find before any gather. any_pend (nullable): skip unless
+// *any_pend == ctx.epoch.
+void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
+void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
 
 }  // namespace lcf

@@ -23,7 +23,7 @@ import torch
 CONFIGS = {
     "tiny_512x512_f32": (1, (512, 512), torch.float32, {"f": 0}),
     "cesm_1800x3600_f32": (2, (1800, 3600), torch.float32, {"T": 0, "U": 1}),
-    "miranda_256x384x384_f64": (3, (256, 384, 384), torch.float64, {"density": 0, "velocity": 1}),
+    "miranda_256x384x384_f64": (3, (256, 384, 384), torch.float64, {"density": 0, "velocity": 1, "rt_density": 2}),
     "nyx_512x512x512_f32": (4, (512, 512, 512), torch.float32, {"baryon_density": 0, "velocity": 1}),
     "hacc_280953867_f32": (5, (280_953_867,), torch.float32, {"xx": 0, "vx": 1}),
 }
@@ -96,6 +96,8 @@ def field(config: str, name: str, device="cpu", origin=None, shape=None, replica
         else:
             f = 0.0 + 20.0 * ms + 1e-3 * 20.0 * eps
     elif config == "miranda_256x384x384_f64":
+        if name == "rt_density":
+            return _rt_density(g, device, shp, origin, full_shape, ms, eps)
         if name == "density":
             fronts = torch.tanh(8.0 * multiscale(shp, g, device, octaves=2, origin=origin, full_shape=full_shape))
             f = 2.0 + (1.0 + fronts) * (0.5 + 0.5 * ms) + 1e-10 * eps
@@ -109,6 +111,28 @@ def field(config: str, name: str, device="cpu", origin=None, shape=None, replica
     else:
         raise KeyError(config)
     return f.to(dtype)
+
+
+def _rt_density(g, device, shp, origin, full_shape, ms, eps):
+    """Rayleigh–Taylor-like density (the flow Miranda simulates): a stratified
+    background ρ0(z) along the fastest axis (z = last index / 384) plus a
+    perturbation confined to a mixing band around z = 0.5 whose half-width
+    δ(x, y) ∈ [0.12, 0.32] varies smoothly over the horizontal plane:
+        f = ρ0(z) + w(x, y, z)·(0.3·ms + 1e-10·ε),
+        ρ0(z) = 2 + tanh((z − 0.5)/0.08) + 0.25·z,
+        w = max(0, 1 − ((z − 0.5)/δ)²)³.
+    Outside the band w is exactly 0, so every (x, y) row repeats ρ0's bits
+    there: the exact repeats at a distance of one row that FCM finds (L300,
+    "repeating values … even when they are far apart"); about half the words
+    match, and each match chains back through all earlier rows."""
+    o = tuple(origin or (0, 0, 0))
+    z = torch.arange(o[2], o[2] + shp[2], dtype=torch.float64, device=device) / full_shape[2]
+    rho0 = 2.0 + torch.tanh((z - 0.5) / 0.08) + 0.25 * z  # a function of z alone: bitwise equal per row
+    m2 = multiscale(shp[:2], g, device, octaves=3, origin=o[:2], full_shape=full_shape[:2])
+    delta = (0.22 + 0.1 * torch.clamp(m2 / 1.5, -1.0, 1.0)).unsqueeze(-1)
+    w = torch.clamp(1.0 - ((z - 0.5) / delta) ** 2, min=0.0) ** 3
+    f = rho0 + w * (0.3 * ms + 1e-10 * eps)
+    return f.to(torch.float64)
 
 
 def _hacc(name, g, device, shp, origin):

@@ -30,6 +30,12 @@ class LcfError(RuntimeError):
 _lib = None
 
 
+class DpView(ctypes.Structure):
+    """lcf_dp_view (include/lcf.h): one shard's decoded words and pending bitmap."""
+    _fields_ = [("first_word", ctypes.c_uint64), ("n_words", ctypes.c_uint64), ("d_words", ctypes.c_void_p),
+                ("d_pending", ctypes.c_void_p)]
+
+
 def lib() -> ctypes.CDLL:
     global _lib
     if _lib is None:
@@ -64,8 +70,17 @@ def lib() -> ctypes.CDLL:
         L.lcf_dpratio_compress_shard.restype = i32
         L.lcf_dpratio_decompress_shard.argtypes = [vp, sz, u64, vp, sz, vp, vp]
         L.lcf_dpratio_decompress_shard.restype = i32
-        L.lcf_dpratio_resolve_pending.argtypes = [vp, sz, vp, vp, vp]
-        L.lcf_dpratio_resolve_pending.restype = i32
+        L.lcf_dpratio_merge_summary_ptrs.argtypes = [ctypes.POINTER(vp), sz, vp, vp]
+        L.lcf_dpratio_merge_summary_ptrs.restype = i32
+        for f in ("lcf_dpratio_find_roots", "lcf_dpratio_gather_roots"):
+            getattr(L, f).argtypes = [ctypes.POINTER(DpView), sz, sz, vp]
+            getattr(L, f).restype = i32
+        L.lcf_ipc_export.argtypes = [vp, ctypes.c_char_p, ctypes.POINTER(u64)]
+        L.lcf_ipc_export.restype = i32
+        L.lcf_ipc_import.argtypes = [ctypes.c_char_p, u64, ctypes.POINTER(vp)]
+        L.lcf_ipc_import.restype = i32
+        L.lcf_ipc_close.argtypes = [vp]
+        L.lcf_ipc_close.restype = i32
         L.lcf_launch_count.argtypes = []
         L.lcf_launch_count.restype = u64
         L.lcf_profile_enable.argtypes = [i32]
@@ -214,9 +229,47 @@ def lcf_dpratio_decompress_shard(d_in, in_bytes, first_word, d_out, out_capacity
                                               _ptr(d_pending), _stream(stream)), "lcf_dpratio_decompress_shard")
 
 
-def lcf_dpratio_resolve_pending(d_out, shard_bytes, d_pending, d_prefix, stream=None) -> None:
-    _check(lib().lcf_dpratio_resolve_pending(_ptr(d_out), shard_bytes, _ptr(d_pending), _ptr(d_prefix),
-                                             _stream(stream)), "lcf_dpratio_resolve_pending")
+def lcf_dpratio_merge_summary_ptrs(d_summaries, count, d_carry, stream=None) -> None:
+    """d_summaries: list of device pointers (tensors or ints), shard order."""
+    arr = (ctypes.c_void_p * max(1, count))(*[_ptr(p) for p in d_summaries[:count]])
+    _check(lib().lcf_dpratio_merge_summary_ptrs(arr, count, _ptr(d_carry), _stream(stream)),
+           "lcf_dpratio_merge_summary_ptrs")
+
+
+def _views(views):
+    """views: list of (first_word, n_words, d_words, d_pending)."""
+    arr = (DpView * len(views))()
+    for q, (f, n, w, p) in enumerate(views):
+        arr[q] = DpView(f, n, _ptr(w), _ptr(p))
+    return arr
+
+
+def lcf_dpratio_find_roots(views, self_index, stream=None) -> None:
+    _check(lib().lcf_dpratio_find_roots(_views(views), len(views), self_index, _stream(stream)),
+           "lcf_dpratio_find_roots")
+
+
+def lcf_dpratio_gather_roots(views, self_index, stream=None) -> None:
+    _check(lib().lcf_dpratio_gather_roots(_views(views), len(views), self_index, _stream(stream)),
+           "lcf_dpratio_gather_roots")
+
+
+def lcf_ipc_export(d_ptr):
+    """(64-byte handle, offset) of the device allocation holding d_ptr."""
+    h = ctypes.create_string_buffer(64)
+    off = ctypes.c_uint64()
+    _check(lib().lcf_ipc_export(_ptr(d_ptr), h, ctypes.byref(off)), "lcf_ipc_export")
+    return h.raw, int(off.value)
+
+
+def lcf_ipc_import(handle: bytes, offset: int) -> int:
+    p = ctypes.c_void_p()
+    _check(lib().lcf_ipc_import(handle, offset, ctypes.byref(p)), "lcf_ipc_import")
+    return int(p.value)
+
+
+def lcf_ipc_close(d_ptr: int) -> None:
+    _check(lib().lcf_ipc_close(d_ptr), "lcf_ipc_close")
 
 
 def lcf_write_header(algo, dtype, total_in_bytes, total_payload_bytes, d_stream, stream=None) -> None:

@@ -172,21 +172,21 @@ def dp_compress_piece(x_shard, n_total_words: int, first_word: int, carry, rank:
 
 
 def dp_simulate_shards(x, world: int) -> bytes:
-    """All ranks' steps on one device, in rank order (the exchange becomes a
-    stacked tensor): the assembled stream, for identity tests."""
+    """All ranks' steps on one device, in rank order (a summary pointer is a
+    plain device pointer here): the assembled stream, for identity tests."""
     import torch
     from . import lcf
     n = x.numel()
     sb = lcf.lcf_dpratio_summary_bytes()
-    sums = torch.empty(world * sb, dtype=torch.uint8, device=x.device)
+    sums = [torch.empty(sb, dtype=torch.uint8, device=x.device) for _ in range(world)]
     ranges = [dp_shard_words(n, world, g) for g in range(world)]
     for g, (f, k) in enumerate(ranges):
-        lcf.lcf_dpratio_shard_summary(x[f:f + k] if k else x, 8 * k, 8 * n, f, sums[g * sb:(g + 1) * sb])
+        lcf.lcf_dpratio_shard_summary(x[f:f + k] if k else x, 8 * k, 8 * n, f, sums[g])
     carry = torch.empty(sb, dtype=torch.uint8, device=x.device)
     tables, pays = [], []
     for g, (f, k) in enumerate(ranges):
         if g:
-            lcf.lcf_dpratio_merge_summaries(sums, g, carry)
+            lcf.lcf_dpratio_merge_summary_ptrs(sums[:g], g, carry)
         t, p, c = dp_compress_piece(x[f:f + k] if k else x[:0], n, f, carry if g else None, g)
         torch.cuda.synchronize()
         tables.append(t.cpu().numpy().tobytes())
@@ -201,27 +201,121 @@ def dp_simulate_shards(x, world: int) -> bytes:
     return hdr + tab + bytes(base - HEADER - 4 * C) + payload
 
 
+# ---- collectives and peer memory for the distributed DPratio calls ------------
+
+def _is_gloo(group=None) -> bool:
+    import torch.distributed as dist
+    return dist.get_backend(group) == "gloo"
+
+
+def _all_gather(t, group=None):
+    """all_gather_into_tensor of a small tensor; with gloo the collective runs
+    on a CPU copy (gloo has no CUDA all-gather-into-tensor)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    src = t.cpu() if _is_gloo(group) else t
+    out = torch.empty(world * src.numel(), dtype=src.dtype, device=src.device)
+    dist.all_gather_into_tensor(out, src.contiguous().reshape(-1), group=group)
+    return out.view((world,) + tuple(src.shape)).to(t.device)
+
+
+def _barrier(group=None):
+    import torch
+    import torch.distributed as dist
+    if torch.cuda.is_available():
+        torch.cuda.synchronize()
+    dist.barrier(group=group)
+
+
+def gather_halo(x_shard, first_word: int, group=None):
+    """The min(3, first_word) words before this rank's shard (FCM's hash
+    context, L172): every rank contributes its last ≤ 3 words, and
+    rank r takes the last words of ranks < r in order (a shard shorter than 3
+    words, or empty, passes the earlier ranks' words through). One all-gather
+    of 4 int64 per rank."""
+    import torch
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    k = x_shard.numel()
+    mine = torch.zeros(4, dtype=torch.int64, device=x_shard.device)
+    c = min(3, k)
+    mine[0] = c
+    if c:
+        mine[1:1 + c] = x_shard[k - c:].view(torch.int64)
+    tails = _all_gather(mine, group).cpu()
+    words = []
+    for r in range(rank):
+        cr = int(tails[r, 0])
+        words.extend(int(v) for v in tails[r, 1:1 + cr])
+    h = min(3, first_word)
+    assert len(words) >= h, "shards must be given in array order"
+    return torch.tensor(words[len(words) - h:], dtype=torch.int64, device=x_shard.device)
+
+
+class PeerTensors:
+    """Device pointers of every rank's copy of some tensors: this rank's own
+    pointers, and its peers' mapped by CUDA IPC (lcf_ipc_export / import; over
+    NVLink between GPUs, plain mappings on one GPU). The handles travel by
+    all_gather_object. close() unmaps."""
+
+    def __init__(self, tensors, group=None):
+        import torch.distributed as dist
+        from . import lcf
+        self.rank, world = dist.get_rank(group), dist.get_world_size(group)
+        mine = [lcf.lcf_ipc_export(t) for t in tensors]
+        allh = [None] * world
+        dist.all_gather_object(allh, mine, group=group)
+        self.ptrs, self._opened = [], []
+        for r in range(world):
+            if r == self.rank:
+                self.ptrs.append([t.data_ptr() for t in tensors])
+            else:
+                row = [lcf.lcf_ipc_import(h, off) for h, off in allh[r]]
+                self._opened.extend(row)
+                self.ptrs.append(row)
+
+    def close(self):
+        from . import lcf
+        for p in self._opened:
+            lcf.lcf_ipc_close(p)
+        self._opened = []
+
+
 def dp_compress_sharded(x_shard, n_total_words: int, first_word: int, group=None):
-    """The distributed version (one process per GPU, NCCL): the summary
-    all-gather, this rank's carry, its piece and the payload-count exchange.
-    Returns (table slice, payload piece, payload offset, total payload)."""
+    """The distributed version (one process per GPU): the 3-word halo from the
+    lower ranks, this rank's summary, its carry merged from the lower ranks'
+    summaries read in place over CUDA IPC (no summary all-gather), its piece,
+    and the payload-count exchange. Returns (table slice, payload piece,
+    payload offset, total payload) with host ints."""
     import torch
     import torch.distributed as dist
     from . import lcf
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    halo = gather_halo(x_shard, first_word, group)
+    h = halo.numel()
+    # [halo ‖ shard] in one buffer, the shard's first word 16-byte aligned
+    # (the allocation is: 4 words of headroom hold the ≤ 3 halo words)
+    buf = torch.empty(4 + max(1, x_shard.numel()), dtype=torch.int64, device=x_shard.device)
+    xs = buf[4:4 + x_shard.numel()]
+    xs.copy_(x_shard.view(torch.int64))
+    if h:
+        buf[4 - h:4] = halo
     sb = lcf.lcf_dpratio_summary_bytes()
     mine = torch.empty(sb, dtype=torch.uint8, device=x_shard.device)
-    lcf.lcf_dpratio_shard_summary(x_shard, x_shard.numel() * 8, 8 * n_total_words, first_word, mine)
-    sums = torch.empty(world * sb, dtype=torch.uint8, device=x_shard.device)
-    dist.all_gather_into_tensor(sums, mine, group=group)
+    nb = xs.numel() * 8
+    lcf.lcf_dpratio_shard_summary(xs, nb, 8 * n_total_words, first_word, mine)
+    _barrier(group)  # every summary written
+    peers = PeerTensors([mine], group)
     carry = None
     if rank:
         carry = torch.empty(sb, dtype=torch.uint8, device=x_shard.device)
-        lcf.lcf_dpratio_merge_summaries(sums, rank, carry)
-    table, payload, count = dp_compress_piece(x_shard, n_total_words, first_word, carry, rank)
-    counts = exchange_counts(count, group=group)
-    off = sum(counts[:rank])
-    return table, payload[:counts[rank]], off, sum(counts)
+        lcf.lcf_dpratio_merge_summary_ptrs([peers.ptrs[r][0] for r in range(rank)], rank, carry)
+    table, payload, count = dp_compress_piece(xs, n_total_words, first_word, carry, rank)
+    _barrier(group)  # every merge has read the summaries
+    peers.close()
+    counts = _all_gather(count, group).reshape(-1).cpu().tolist()
+    return table, payload[:counts[rank]], sum(counts[:rank]), sum(counts)
 
 
 def dp_shard_substream(stream: bytes, world: int, rank: int) -> bytes:
@@ -247,14 +341,17 @@ def dp_shard_substream(stream: bytes, world: int, rank: int) -> bytes:
 
 def dp_simulate_decode_shards(stream: bytes, world: int):
     """Sharded DPratio decompression on one device: every shard decodes its
-    sub-stream independently (cross-shard words left pending), then the shards
-    resolve their pending words in array order. Returns the int64 words."""
+    sub-stream independently (words whose chains leave a tile that is not yet
+    complete stay pending), then every shard finds its pending words' roots
+    through the views of all shards, then every shard gathers the roots'
+    values — the distributed protocol with the barriers as program order.
+    Returns the int64 words."""
     import numpy as np
     import torch
     from . import lcf
     n = int(np.frombuffer(stream[8:16], np.uint64)[0]) // 8
     out = torch.empty(max(n, 1), dtype=torch.int64, device="cuda")
-    pend, subs = [], []
+    views, subs = [], []
     for g in range(world):
         f, k = dp_shard_words(n, world, g)
         sub = torch.from_numpy(np.frombuffer(dp_shard_substream(stream, world, g), np.uint8).copy()).cuda()
@@ -262,70 +359,22 @@ def dp_simulate_decode_shards(stream: bytes, world: int):
         if k:
             lcf.lcf_dpratio_decompress_shard(sub, sub.numel(), f, out[f:f + k], 8 * k, p)
         subs.append(sub)
-        pend.append(p)
+        views.append((f, k, out[f:f + k] if k else out, p))
     lcf.lcf_check_stream()
-    for g in range(world):  # in array order: everything before shard g is final
-        f, k = dp_shard_words(n, world, g)
-        if k:
-            lcf.lcf_dpratio_resolve_pending(out[f:f + k], 8 * k, pend[g], out)
-    torch.cuda.synchronize()
+    for g in range(world):
+        lcf.lcf_dpratio_find_roots(views, g)
+    for g in range(world):
+        lcf.lcf_dpratio_gather_roots(views, g)
+    lcf.lcf_check_stream()
     return out[:n]
-
-
-def _owner(j, n: int, world: int):
-    """Rank owning global word index j (tensor) under dp_shard_words."""
-    import torch
-    firsts = torch.tensor([dp_shard_words(n, world, r)[0] for r in range(world)], dtype=torch.int64,
-                          device=j.device)
-    return torch.searchsorted(firsts, j, right=True) - 1
-
-
-def dp_resolve_pending_distributed(out_local, pend, first_word: int, n_total: int, group=None):
-    """Resolve a decoded shard's pending words (lcf_dpratio_decompress_shard)
-    across ranks: in rank order r = 1 … G−1, rank r asks every lower rank for
-    the final words at its pending targets; a lower rank is final by then
-    (its own step came first). Point-to-point messages only: the request and
-    answer volume is the number of pending words. Works on any backend (NCCL
-    with CUDA tensors, gloo with CPU tensors)."""
-    import torch
-    import torch.distributed as dist
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
-    dev = out_local.device
-    k = out_local.numel()
-    bits = pend.view(torch.int32)
-    pos = torch.arange(k, device=dev)
-    mask = ((bits[pos // 32] >> (pos % 32)) & 1).bool() if k else torch.zeros(0, dtype=torch.bool, device=dev)
-    idx = pos[mask]
-    tgt = out_local[idx].clone()
-    own = _owner(tgt, n_total, world) if idx.numel() else tgt
-    for r in range(1, world):
-        if rank == r:
-            for q in range(r):
-                sel = own == q
-                req = tgt[sel].contiguous()
-                cnt = torch.tensor([req.numel()], dtype=torch.int64, device=dev)
-                dist.send(cnt, q, group=group)
-                if req.numel():
-                    dist.send(req, q, group=group)
-                    vals = torch.empty_like(req)
-                    dist.recv(vals, q, group=group)
-                    out_local[idx[sel]] = vals
-        elif rank < r:
-            cnt = torch.empty(1, dtype=torch.int64, device=dev)
-            dist.recv(cnt, r, group=group)
-            c = int(cnt.item())
-            if c:
-                req = torch.empty(c, dtype=torch.int64, device=dev)
-                dist.recv(req, r, group=group)
-                dist.send(out_local[req - first_word].contiguous(), r, group=group)
-    return out_local
 
 
 def dp_decompress_sharded(sub_stream, first_word: int, n_total: int, group=None):
     """The distributed sharded DPratio decompression of this rank's sub-stream
-    (dp_shard_substream layout, CUDA uint8 tensor): decode with cross-shard
-    chains pending, then resolve them against the lower ranks. Returns the
-    rank's int64 words."""
+    (dp_shard_substream layout, CUDA uint8 tensor): decode with pending words,
+    then the root resolution over every rank's words and bitmap, read in place
+    over CUDA IPC (peer loads over NVLink; no message per pending word).
+    Returns the rank's int64 words."""
     import torch
     import torch.distributed as dist
     from . import lcf
@@ -336,5 +385,17 @@ def dp_decompress_sharded(sub_stream, first_word: int, n_total: int, group=None)
     pend = torch.zeros(max(1, (k + 31) // 32), dtype=torch.int32, device=sub_stream.device)
     if k:
         lcf.lcf_dpratio_decompress_shard(sub_stream, sub_stream.numel(), f, out, 8 * k, pend)
-        lcf.lcf_check_stream()
-    return dp_resolve_pending_distributed(out[:k], pend, f, n_total, group=group)
+    lcf.lcf_check_stream()
+    _barrier(group)  # a. every shard decoded
+    peers = PeerTensors([out, pend], group)
+    views = []
+    for r in range(world):
+        fr, kr = dp_shard_words(n_total, world, r)
+        views.append((fr, kr, peers.ptrs[r][0], peers.ptrs[r][1]))
+    lcf.lcf_dpratio_find_roots(views, rank)
+    _barrier(group)  # c. every walk ended
+    lcf.lcf_dpratio_gather_roots(views, rank)
+    lcf.lcf_check_stream()
+    _barrier(group)  # every peer read done before the mappings go
+    peers.close()
+    return out[:k]

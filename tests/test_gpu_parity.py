@@ -1,5 +1,7 @@
 """GPU parity: the sm_100a path (through the C ABI) vs the CPU oracle, bit-exact
 on streams, size tables and decompressed bits (-m gpu)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -59,42 +61,35 @@ def check_parity(L, orc, algo, words: np.ndarray, name=""):
     return len(s_gpu)
 
 
-def algos_available(L):
-    avail = []
+def test_all_codecs_built(L):
+    """Every codec runs on the device: a missing one fails here instead of
+    silently skipping its parity suite."""
     for a in GPU_ALGOS:
-        try:
-            x = torch.zeros(16, dtype=tdt(a), device="cuda")
-            L.compress(a, x)
-            avail.append(a)
-        except L.LcfError:
-            pass
-    return avail
+        x = torch.zeros(16, dtype=tdt(a), device="cuda")
+        s = L.compress(a, x)
+        assert torch.equal(L.decompress(a, s), x), a
 
 
 @pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_adversarial_parity(L, orc, algo):
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
     for name, words in datagen.adversarial(32 if algo.startswith("SP") else 64):
         check_parity(L, orc, algo, words, name)
 
 
 @pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_exhaustive_tiny_parity(L, orc, algo):
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
+    """Every 1-, 2- and 3-word stream over the 16 special values:
+    16 + 256 + 4096 streams per codec, GPU = oracle byte for byte."""
+    import itertools
     sp = datagen.F32_SPECIALS if algo.startswith("SP") else datagen.F64_SPECIALS
-    rng = np.random.default_rng(0)
     for r in (1, 2, 3):
-        for _ in range(60):
-            check_parity(L, orc, algo, sp[rng.integers(0, 16, r)], f"tiny{r}")
+        for combo in itertools.product(range(16), repeat=r):
+            check_parity(L, orc, algo, sp[list(combo)], f"tiny{combo}")
 
 
 @pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_random_width_subchunks(L, orc, algo):
     """Every MPLG width 0..W (both flag states) and ragged tails."""
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
     W = 32 if algo.startswith("SP") else 64
     dt = wdt(algo)
     rng = np.random.default_rng(W)
@@ -119,8 +114,6 @@ CONFIG_CASES = [("SPspeed", "tiny_512x512_f32", "f"), ("SPratio", "tiny_512x512_
 
 @pytest.mark.parametrize("algo,config,field", CONFIG_CASES)
 def test_config_field_parity(L, orc, algo, config, field):
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
     x = datagen.field(config, field, device="cuda")
     words = x.cpu().numpy().view(wdt(algo))
     n = check_parity(L, orc, algo, words, f"{config}/{field}")
@@ -131,8 +124,6 @@ def test_config_field_parity(L, orc, algo, config, field):
                                         ("DPratio", "density"), ("DPratio", "velocity")])
 def test_miranda_subvolume_parity(L, orc, algo, field):
     """Miranda-shaped f64 (a 32×384×384 slab of the full field, 4.7 M words)."""
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
     x = datagen.field("miranda_256x384x384_f64", field, device="cuda", origin=(0, 0, 0), shape=(32, 384, 384))
     check_parity(L, orc, algo, x.cpu().numpy().view(np.uint64), f"miranda/{field}")
 
@@ -141,8 +132,6 @@ def test_dpratio_mixed_match_tiles(L, orc):
     """Tiles with and without FCM matches interleaved (the encoder's all-zero
     Dist fast path and its per-CTA cached stream alternate with the general
     path), plus a ragged last tile."""
-    if "DPratio" not in algos_available(L):
-        pytest.skip("DPratio not built")
     x = datagen.field("miranda_256x384x384_f64", "density", shape=(2, 384, 384)).numpy().reshape(-1).view(np.uint64)
     x = x[: 2048 * 100 + 777].copy()
     T = 2048
@@ -158,8 +147,6 @@ def test_dpratio_raw_tiles_with_matches(L, orc):
     matches: copied 16-word runs from random earlier positions, copies of
     copies (chains across tiles), and a ragged last tile. Exercises the
     decoder's raw-V + FCM path and cross-tile chain resolution."""
-    if "DPratio" not in algos_available(L):
-        pytest.skip("DPratio not built")
     rng = np.random.default_rng(11)
     T = 2048
     x = rng.integers(0, 2**63, size=12 * T + 333, dtype=np.uint64)
@@ -203,24 +190,38 @@ def test_dpratio_fcm_long_hash_runs(L, orc):
     """FCM distances over long same-hash runs (one hash for 300 K positions,
     50 hashes recurring every 50 positions, matches at the 3rd/4th candidate
     or beyond the window) — stream identical to the oracle's."""
-    if "DPratio" not in algos_available(L):
-        pytest.skip("DPratio not built")
     check_parity(L, orc, "DPratio", fcm_stress_input(), "fcm_long_hash_runs")
 
 
-def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
-    """Full-size check: GPU stream vs oracle on a sample of chunks (compress_chunks)."""
+def oracle_pieces_threaded(orc, algo, words, n_chunks, per=256):
+    """The oracle's size table and padded payload for chunks [0, n_chunks) of
+    `words`, computed in chunk ranges on all host cores (the oracle's own
+    compress_chunks; ctypes releases the GIL). Chunks are context-free (L104),
+    so the concatenated pieces are the oracle's whole-stream table and payload."""
+    from concurrent.futures import ThreadPoolExecutor
+    ranges = [(c, min(per, n_chunks - c)) for c in range(0, n_chunks, per)]
+    with ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
+        parts = list(ex.map(lambda r: orc.compress_chunks(algo, words, r[0], r[1]), ranges))
+    return np.concatenate([t for t, _ in parts]), b"".join(p for _, p in parts)
+
+
+def full_stream_parity(L, orc, algo, x_dev):
+    """Full-size check: the whole GPU stream equals the oracle's byte for byte
+    (header fields, every size-table entry, every payload byte), and decodes."""
     s = L.compress(algo, x_dev)
-    stream = s.cpu().numpy().tobytes()
-    words = x_dev.cpu().numpy().view(wdt(algo))
-    h, table, chunks = fmt_ref.parse_stream(stream)
-    C = len(table)
-    rng = np.random.default_rng(seed)
-    picks = sorted(set([0, C - 1] + rng.integers(0, C, n_samples).tolist()))
-    for c in picks:
-        tab, pay = orc.compress_chunks(algo, words, c, 1)
-        assert tab[0] == table[c], (c, tab[0], table[c])
-        assert pay[:tab[0] & 0x7FFFFFFF] == chunks[c][1], c
+    stream = s.cpu().numpy()
+    words = x_dev.cpu().numpy().reshape(-1).view(wdt(algo))
+    C = L.lcf_num_chunks(algo, words.nbytes)
+    table, payload = oracle_pieces_threaded(orc, algo, words, C)
+    hdr = np.frombuffer(stream[:32].tobytes(), np.uint64)
+    algo_id = {"SPspeed": 0, "SPratio": 1, "DPspeed": 2, "DPratio": 3}[algo]
+    assert stream[:8].tobytes() == (0x3146434C).to_bytes(4, "little") + bytes([1, algo_id, words.itemsize, 0])
+    assert int(hdr[1]) == words.nbytes and int(hdr[2]) == C and int(hdr[3]) == len(payload)
+    assert np.array_equal(stream[32:32 + 4 * C].view(np.uint32), table)
+    base = (32 + 4 * C + 15) // 16 * 16
+    assert not stream[32 + 4 * C:base].any()
+    assert len(stream) == base + len(payload)
+    assert stream[base:].tobytes() == payload
     y = L.decompress(algo, s)
     assert torch.equal(y, x_dev.reshape(-1))
     return len(stream)
@@ -228,40 +229,69 @@ def sampled_chunk_parity(L, orc, algo, x_dev, n_samples=24, seed=0):
 
 @pytest.mark.parametrize("algo,config,field", [
     ("SPspeed", "nyx_512x512x512_f32", "baryon_density"), ("SPspeed", "nyx_512x512x512_f32", "velocity"),
-    ("SPspeed", "hacc_280953867_f32", "xx"), ("SPratio", "nyx_512x512x512_f32", "velocity"),
-    ("SPratio", "hacc_280953867_f32", "vx"), ("DPspeed", "miranda_256x384x384_f64", "density")])
-def test_full_size_sampled_parity(L, orc, algo, config, field):
-    if algo not in algos_available(L):
-        pytest.skip(f"{algo} not built")
+    ("SPspeed", "hacc_280953867_f32", "xx"), ("SPspeed", "hacc_280953867_f32", "vx"),
+    ("SPratio", "nyx_512x512x512_f32", "baryon_density"), ("SPratio", "nyx_512x512x512_f32", "velocity"),
+    ("SPratio", "hacc_280953867_f32", "xx"), ("SPratio", "hacc_280953867_f32", "vx"),
+    ("DPspeed", "miranda_256x384x384_f64", "density"), ("DPspeed", "miranda_256x384x384_f64", "rt_density")])
+def test_full_size_stream_parity(L, orc, algo, config, field):
+    """BASELINE configs[2]/[3] at full size, the bench's fields: whole streams
+    byte for byte against the oracle (sampled chunks were not
+    enough)."""
     x = datagen.field(config, field, device="cuda").reshape(-1)
     x = x.view(tdt(algo))
-    sampled_chunk_parity(L, orc, algo, x)
+    full_stream_parity(L, orc, algo, x)
     del x
     torch.cuda.empty_cache()
 
 
-def test_full_size_dpratio_stream(L, orc):
-    """The bench's DPratio workload at full size (Miranda density, 256×384×384
-    f64, 37.7 M words: 2304 FCM sort tiles, 18,432 encode tiles): the whole GPU
-    stream equals the oracle's byte for byte (the oracle needs ~1 min), and it
-    decodes back."""
-    if "DPratio" not in algos_available(L):
-        pytest.skip("DPratio not built")
-    x = datagen.field("miranda_256x384x384_f64", "density", device="cuda").reshape(-1).view(torch.int64)
+@pytest.mark.parametrize("field", ["density", "rt_density"])
+def test_full_size_dpratio_stream(L, orc, field):
+    """The bench's DPratio workload at full size (Miranda-shaped 256×384×384
+    f64, 37.7 M words: 2304 FCM sort tiles, 18,432 encode tiles) — density
+    (no FCM match) and rt_density (about half the words match, every match
+    chaining back through all earlier rows): the whole GPU stream equals the
+    oracle's byte for byte (the oracle needs ~1 min), and it decodes back,
+    also through the host-buffer path."""
+    x = datagen.field("miranda_256x384x384_f64", field, device="cuda").reshape(-1).view(torch.int64)
     s = L.compress("DPratio", x)
-    ref = orc.compress("DPratio", x.cpu().numpy().view(np.uint64))
+    hx = x.cpu().numpy().view(np.uint64)
+    ref = orc.compress("DPratio", hx)
     assert s.numel() == len(ref)
     assert np.array_equal(s.cpu().numpy(), np.frombuffer(ref, np.uint8))
     assert torch.equal(L.decompress("DPratio", s), x)
-    # the host-buffer path compresses in tile slices with carried FCM state: the same bytes
-    hx = x.cpu().numpy().view(np.uint64)
+    # the host-buffer path compresses in tile slices with carried FCM state and
+    # decodes in tile ranges: the same bytes, the same words
     hout = np.zeros(L.lcf_max_compressed_size("DPratio", None, hx.nbytes), np.uint8)
     nh = L.lcf_compress_host("DPratio", None, hx, hx.nbytes, hout, hout.nbytes)
     assert nh == len(ref) and hout[:nh].tobytes() == ref
+    hy = np.zeros_like(hx)
+    assert L.lcf_decompress_host("DPratio", None, hout, nh, hy, hy.nbytes) == hx.nbytes
+    assert np.array_equal(hy, hx)
     del x, s
     torch.cuda.empty_cache()
 
 
+def test_dpratio_long_chains(L, orc, monkeypatch):
+    """FCM decode on chains that cross many tiles (L197): a constant array
+    (every word copies its predecessor: one chain through the whole array), a
+    period-384 array (chains of row length), a period-5000 array (each hop
+    crosses tiles) and an rt_density slab — GPU stream = oracle, words back,
+    also through 3-tile host slices."""
+    rng = np.random.default_rng(3)
+    base = rng.integers(0, 2**63, size=5000, dtype=np.uint64)
+    cases = {"constant": np.full(40 * 2048 + 5, 0x400921FB54442D18, np.uint64),
+             "period384": np.resize(base[:384], 30 * 2048 + 100),
+             "period5000": np.resize(base, 30 * 2048 + 7)}
+    rt = datagen.field("miranda_256x384x384_f64", "rt_density", shape=(3, 64, 384)).numpy().reshape(-1)
+    cases["rt_slab"] = rt.view(np.uint64).copy()
+    monkeypatch.setenv("LCF_HOST_SLICE_BYTES", str(3 * 16384))
+    for name, w in cases.items():
+        check_parity(L, orc, "DPratio", w, name)
+        ref = orc.compress("DPratio", w)
+        back = np.zeros_like(w)
+        assert L.lcf_decompress_host("DPratio", None, np.frombuffer(ref, np.uint8).copy(), len(ref), back,
+                                     back.nbytes) == w.nbytes
+        assert np.array_equal(back, w), name
 @pytest.mark.parametrize("algo", SPEED_ALGOS)
 def test_async_path_and_corruption(L, orc, algo):
     words = datagen.smooth_1d(3 * 4096 + 77, np.float32 if algo == "SPspeed" else np.float64, seed=3)

@@ -122,10 +122,11 @@ def _dp_inputs():
         j = int(rng.integers(0, i - n))
         mixed[i:i + n] = mixed[j:j + n]
     slab = datagen.field("miranda_256x384x384_f64", "density", shape=(2, 384, 384)).numpy().reshape(-1).view(np.uint64)
-    return {"fcm_stress": fcm_stress_input(), "copies": mixed, "miranda_slab": slab.copy()}
+    rt = datagen.field("miranda_256x384x384_f64", "rt_density", shape=(4, 96, 384)).numpy().reshape(-1).view(np.uint64)
+    return {"fcm_stress": fcm_stress_input(), "copies": mixed, "miranda_slab": slab.copy(), "rt_slab": rt.copy()}
 
 
-@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab"])
+@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab", "rt_slab"])
 @pytest.mark.parametrize("world", [2, 3, 8])
 def test_dpratio_shards_assemble_to_global(L, orc, name, world):
     """Sharded DPratio (NEXT-1): shard summaries → per-shard carries → shard
@@ -139,12 +140,13 @@ def test_dpratio_shards_assemble_to_global(L, orc, name, world):
         assert got == orc.compress("DPratio", words)
 
 
-@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab"])
+@pytest.mark.parametrize("name", ["fcm_stress", "copies", "miranda_slab", "rt_slab"])
 @pytest.mark.parametrize("world", [2, 3, 8])
 def test_dpratio_shard_decode(L, name, world):
     """Sharded DPratio decompression (NEXT-1): each shard decodes its own
-    sub-stream with chains into earlier shards left pending, then the shards
-    resolve them in array order — the original words come back."""
+    sub-stream with chains leaving a tile left pending, then every shard
+    finds its pending words' roots through all shards' views, then gathers
+    them — the original words come back."""
     words = _dp_inputs()[name]
     x = torch.from_numpy(words.view(np.int64)).cuda()
     stream = L.compress("DPratio", x).cpu().numpy().tobytes()

@@ -36,9 +36,17 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-WORKLOAD = "cesm_1800x3600_f32[T,U]:SPspeed,SPratio + miranda_256x384x384_f64[density]:DPspeed,DPratio"
-SP_CONFIG, SP_FIELDS = "cesm_1800x3600_f32", ("T", "U")
-DP_CONFIG, DP_FIELDS = "miranda_256x384x384_f64", ("density",)
+# (config, fields, codecs): BASELINE.json configs[1] (CESM-ATM-shaped) and
+# configs[3] (NYX-shaped 512³ and the HACC-like 1-D arrays — the largest
+# single-GPU SP configuration) for the SP codecs; configs[2] (Miranda-shaped)
+# for the DP codecs, with `rt_density` the field whose exact repeats FCM finds
+FIELD_SETS = (
+    ("cesm_1800x3600_f32", ("T", "U"), ("SPspeed", "SPratio")),
+    ("nyx_512x512x512_f32", ("baryon_density", "velocity"), ("SPspeed", "SPratio")),
+    ("hacc_280953867_f32", ("xx", "vx"), ("SPspeed", "SPratio")),
+    ("miranda_256x384x384_f64", ("density", "rt_density"), ("DPspeed", "DPratio")),
+)
+WORKLOAD = " + ".join(f"{cfg}[{','.join(names)}]:{','.join(codecs)}" for cfg, names, codecs in FIELD_SETS)
 ALL_CODECS = ("SPspeed", "SPratio", "DPspeed", "DPratio")
 L2_FLUSH_BYTES = 256 << 20
 
@@ -106,28 +114,43 @@ def dist_env():
     return ws, rank, local
 
 
+def replica_bytes(cfg):
+    from paper_conf_asplos_azamifb25_b200 import datagen
+    _, shape, dtype, _ = datagen.CONFIGS[cfg]
+    n = 1
+    for d in shape:
+        n *= d
+    return n * (4 if dtype == torch.float32 else 8)
+
+
 def make_fields(world, rank, device):
     """Per-field inputs. N = 1: the config's field. N > 1 (weak scaling): the
-    global input is the concatenation of N independent fields of the config
-    (replicas); chunk-local codecs get this rank's chunk-range shard of it,
-    DPratio (whole-array FCM) gets replica `rank` whole."""
+    global input is the concatenation of N independent replicas of the field;
+    chunk-local codecs get this rank's chunk-range shard of it (generated from
+    the ≤ 3 replicas the shard overlaps), DPratio (whole-array FCM) gets
+    replica `rank` whole."""
     from paper_conf_asplos_azamifb25_b200 import datagen, sharded
     fields = []
-    for cfg, names, codecs in ((SP_CONFIG, SP_FIELDS, ("SPspeed", "SPratio")),
-                               (DP_CONFIG, DP_FIELDS, ("DPspeed", "DPratio"))):
+    for cfg, names, codecs in FIELD_SETS:
+        rb = replica_bytes(cfg)
         for nm in names:
-            reps = [datagen.field(cfg, nm, device=device, replica=r).reshape(-1) for r in range(world)]
-            wdt = torch.int32 if reps[0].dtype == torch.float32 else torch.int64
-            whole = torch.cat(reps).view(wdt) if world > 1 else reps[0].view(wdt)
-            total = whole.numel() * whole.element_size()
-            off, ln = sharded.shard_bytes(total, world, rank)
-            shard = whole.view(torch.uint8)[off:off + ln].view(wdt).clone()
-            own = reps[rank].view(wdt).clone()
-            del reps, whole
+            own = datagen.field(cfg, nm, device=device, replica=rank).reshape(-1)
+            wdt = torch.int32 if own.dtype == torch.float32 else torch.int64
+            own = own.view(wdt)
+            shard, total = own, rb
+            if world > 1:
+                total = world * rb
+                off, ln = sharded.shard_bytes(total, world, rank)
+                r0, r1 = off // rb, (off + max(ln, 1) - 1) // rb
+                parts = [own if r == rank else datagen.field(cfg, nm, device=device, replica=r).reshape(-1).view(wdt)
+                         for r in range(r0, r1 + 1)]
+                whole = torch.cat(parts) if len(parts) > 1 else parts[0]
+                shard = whole.view(torch.uint8)[off - r0 * rb:off - r0 * rb + ln].view(wdt).clone()
+                del parts, whole
             for codec in codecs:
                 x = own if (codec == "DPratio" or world == 1) else shard
                 fields.append((cfg, nm, codec, x, total))
-    torch.cuda.empty_cache()
+            torch.cuda.empty_cache()
     return fields
 
 
@@ -164,7 +187,9 @@ def kernel_bytes(j):
             "fcm_sort_scatter": 2 * 16 * words,       # 8-byte records (or x) in, records out
             "fcm_match": 8 * words,                   # sorted records in (x gathered, matches scattered)
             "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
-            "dpratio_decode": sb + n}                 # stream in, x out
+            "dpratio_decode": sb + n,                 # stream in, x out
+            "dp_find_roots": words // 8,              # the pending bitmap (the walks are data-dependent)
+            "dp_gather_roots": words // 8}
 
 
 def compress_op(lcf, j):
@@ -211,13 +236,7 @@ def run_lcf(args):
         cap = lcf.lcf_max_compressed_size(codec, None, nbytes)
         s = torch.empty(cap, dtype=torch.uint8, device=dev)
         y = torch.empty_like(x)
-        try:
-            n = lcf.lcf_compress(codec, None, x, nbytes, s, cap)
-        except lcf.LcfError as e:
-            if e.status == 1:
-                print(f"[bench] {codec} unavailable: {e}", file=sys.stderr)
-                continue
-            raise
+        n = lcf.lcf_compress(codec, None, x, nbytes, s, cap)  # every codec must run: no skip
         lcf.lcf_decompress(codec, None, s, n, y, nbytes)
         assert torch.equal(x, y), f"{codec}/{nm}: round trip failed"
         sharded_job = world > 1 and codec != "DPratio"
@@ -314,12 +333,12 @@ def run_lcf(args):
         value = world * tot_bytes / ms_step / 1e6
 
     transfer = None
-    if world > 1 and args.transfer:
+    if world > 1 and args.transfer:  # (on by default at N ≥ 2)
         try:
             transfer = run_transfer(jobs, rank, dev)
         except Exception as e:  # a measurement extra: never fail the bench line for it
             print(f"[bench] transfer measurement failed: {e!r}", file=sys.stderr)
-    e2e = run_e2e(lcf, jobs, args) if rank == 0 else None
+    e2e = run_e2e(lcf, jobs, args, world)
     cpu = run_cpu_baseline(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
     cpu_codec = run_cpu_codec(jobs) if (rank == 0 and world == 1 and not args.no_cpu_baseline) else None
     if rank == 0:
@@ -391,78 +410,118 @@ def run_transfer(jobs, rank, dev, reps: int = 3):
             "jobs": out}
 
 
-def run_e2e(lcf, jobs, args):
+def run_e2e(lcf, jobs, args, world=1):
     """Same metric through lcf_compress_host / lcf_decompress_host (pinned
-    host buffers; H2D of the step's inputs and D2H of its results inside)."""
+    host buffers; H2D of the step's inputs and D2H of its results inside),
+    on every rank at once; the step time is the max over ranks. Pinned
+    buffers are shared by the jobs of one field."""
+    bufs = {}
     host = []
     for j in jobs:
-        hx = torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True)
-        hx.copy_(j["x"].view(torch.uint8).cpu())
-        hs = torch.empty(j["cap"], dtype=torch.uint8, pin_memory=True)
-        hy = torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True)
-        host.append((j, hx, hs, hy))
+        key = j["x"].data_ptr()
+        if key not in bufs:
+            hx = torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True)
+            hx.copy_(j["x"].view(torch.uint8).cpu())
+            cap = max(jj["cap"] for jj in jobs if jj["x"].data_ptr() == key)
+            bufs[key] = (hx, torch.empty(cap, dtype=torch.uint8, pin_memory=True),
+                         torch.empty(j["nbytes"], dtype=torch.uint8, pin_memory=True))
+        host.append((j,) + bufs[key])
     h2d = d2h = 0
     times = []
-    for it in range(max(1, args.warmup) + max(1, args.steps)):
+    iters = 1 + min(3, max(1, args.steps))  # one warm-up, ≤ 3 timed (PCIe-bound, seconds each)
+    for it in range(iters):
         torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
         t0 = time.perf_counter()
         h2d = d2h = 0
         for j, hx, hs, hy in host:
-            n = lcf.lcf_compress_host(j["codec"], None, hx, j["nbytes"], hs, j["cap"])
+            n = lcf.lcf_compress_host(j["codec"], None, hx, j["nbytes"], hs, hs.numel())
             m = lcf.lcf_decompress_host(j["codec"], None, hs, n, hy, j["nbytes"])
             h2d += j["nbytes"] + n
             d2h += n + m
+            if it == iters - 1:
+                assert torch.equal(hx, hy), j["codec"]
         times.append(time.perf_counter() - t0)
-    for j, hx, hs, hy in host:
-        assert torch.equal(hx, hy), j["codec"]
-    t = statistics.median(times[max(1, args.warmup):])
-    total = sum(2 * j["nbytes"] for j, *_ in host)
+    t = statistics.median(times[1:])
+    if world > 1:
+        tt = torch.tensor([t], device="cuda")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        t = float(tt.item())
+    total = world * sum(2 * j["nbytes"] for j, *_ in host)
     return {"value": total / t / 1e9, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-            "ms_per_step": t * 1e3, "api": "lcf_compress_host + lcf_decompress_host"}
+            "ms_per_step": t * 1e3, "api": "lcf_compress_host + lcf_decompress_host",
+            "timing": "host wall clock per step (the calls synchronise), median of 3 after 1 warm-up"
+                      + (", max over ranks; bytes per step are rank 0's" if world > 1 else "")}
+
+
+def _host_words(j, nbytes):
+    words = j["x"][: nbytes // j["x"].element_size()].cpu().numpy()
+    return words.view(np.uint32 if words.dtype == np.int32 else np.uint64)
 
 
 def run_cpu_baseline(jobs, budget_s: float = 12.0):
-    """The oracle as it stands, single-threaded, on a bounded sample: the first
-    K chunks of every (codec, field) job, K sized for ~budget_s seconds."""
+    """The oracle as it stands on a bounded sample of the workload: the first
+    4 MiB of every (codec, field) job, single-threaded, repeated up to the
+    budget; plus the same oracle functions run chunk-parallel over all host
+    cores on the first 64 MiB of every chunk-local job — each
+    thread compresses and decompresses its own chunk range as an independent
+    stream (chunks are context-free, L104); DPratio's FCM is a whole-array
+    pass, so it has no chunk-parallel oracle figure."""
     import oracle
+    from concurrent.futures import ThreadPoolExecutor
     oracle.lib()
-    sample_bytes = 1 << 20
-    done_bytes, spent = 0, 0.0
-    per = []
-    for j in jobs:
-        words = j["x"][: sample_bytes // j["x"].element_size()].cpu().numpy()
-        words = words.view(np.uint32 if words.dtype == np.int32 else np.uint64)
-        t0 = time.perf_counter()
-        s = oracle.compress(j["codec"], words)
-        t1 = time.perf_counter()
-        y = oracle.decompress(j["codec"], s)
-        t2 = time.perf_counter()
-        assert np.array_equal(y, words)
-        per.append((j["codec"], words.nbytes, t1 - t0, t2 - t1))
-        done_bytes += 2 * words.nbytes
-        spent += t2 - t0
-    # scale the sample up to the budget
-    reps = max(1, int(budget_s / max(spent, 1e-3)))
-    reps = min(reps, 8)
-    if reps > 1:
-        for _ in range(reps - 1):
-            for j in jobs:
-                words = j["x"][: sample_bytes // j["x"].element_size()].cpu().numpy()
-                words = words.view(np.uint32 if words.dtype == np.int32 else np.uint64)
-                t0 = time.perf_counter()
-                s = oracle.compress(j["codec"], words)
-                oracle.decompress(j["codec"], s)
-                spent += time.perf_counter() - t0
-                done_bytes += 2 * words.nbytes
-    return {"value": done_bytes / spent / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {sample_bytes >> 20} MiB of every (codec, field) of the workload, compress+decompress, "
-                      f"x{reps}; {spent:.1f} s single-threaded"}
+    sample_bytes = 4 << 20
+    samples = [(j["codec"], _host_words(j, sample_bytes)) for j in jobs]
+    done_bytes, spent, reps = 0, 0.0, 0
+    while reps < 4 and (reps == 0 or spent * (reps + 1) / reps <= budget_s):
+        for codec, words in samples:
+            t0 = time.perf_counter()
+            s = oracle.compress(codec, words)
+            y = oracle.decompress(codec, s)
+            spent += time.perf_counter() - t0
+            done_bytes += 2 * words.nbytes
+            if reps == 0:
+                assert np.array_equal(y, words)
+        reps += 1
+    out = {"value": done_bytes / spent / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+           "sample": f"first {sample_bytes >> 20} MiB of every (codec, field) of the workload, compress+decompress, "
+                     f"x{reps}; {spent:.1f} s single-threaded"}
+    nt = os.cpu_count() or 1
+    big = [(j["codec"], _host_words(j, 64 << 20)) for j in jobs if j["codec"] != "DPratio"]
+    work = []
+    for codec, words in big:
+        cw = 16384 // words.itemsize
+        nc = -(-len(words) // cw)
+        per = -(-nc // nt)
+        work += [(codec, words[c * cw:(c + per) * cw]) for c in range(0, nc, per)]
+
+    def one(item):
+        codec, w = item
+        return np.array_equal(oracle.decompress(codec, oracle.compress(codec, w)), w)
+
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(max_workers=nt) as ex:
+        ok = all(ex.map(one, work))
+    t = time.perf_counter() - t0
+    assert ok
+    moved = 2 * sum(w.nbytes for _, w in big)
+    out["multicore"] = {"value": moved / t / 1e9, "unit": "GB/s", "cores": nt, "kind": "oracle, chunk-parallel",
+                        "sample": "first 64 MiB of every SPspeed/SPratio/DPspeed job, compress+decompress, "
+                                  f"{nt} threads over chunk ranges; {t:.1f} s"}
+    return out
+
+
+CPU_CODEC_FIELDS = ("cesm_1800x3600_f32/T", "cesm_1800x3600_f32/U", "miranda_256x384x384_f64/density",
+                    "miranda_256x384x384_f64/rt_density")
 
 
 def run_cpu_codec(jobs):
     """The multi-threaded CPU codec (liblcf_cpu.so) on the
-    whole workload, one step, all host cores: same metric; its streams must be
-    the GPU's bytes (the paper's CPU/GPU compatibility, L354)."""
+    CESM and Miranda jobs of the workload (whole fields; the NYX/HACC jobs are
+    left out to bound the run), one step, all host cores: same metric; its
+    streams must be the GPU's bytes (the paper's CPU/GPU compatibility, L354)."""
+    jobs = [j for j in jobs if j["field"] in CPU_CODEC_FIELDS]
     from paper_conf_asplos_azamifb25_b200 import lcf_cpu
     lcf_cpu.lib()
     nt = os.cpu_count() or 1
@@ -480,7 +539,8 @@ def run_cpu_codec(jobs):
         total += 2 * words.nbytes
         same = same and s.tobytes() == s_gpu.tobytes() and np.array_equal(y, words)
     return {"value": total / spent / 1e9, "unit": "GB/s", "cores": nt, "kind": "cpu_codec (liblcf_cpu.so)",
-            "streams_equal_gpu": bool(same), "sample": "the whole workload, one step (compress + decompress)"}
+            "streams_equal_gpu": bool(same),
+            "sample": "whole CESM T/U and Miranda density/rt_density fields with their codecs, compress + decompress"}
 
 
 def run_reference(args):
@@ -492,14 +552,20 @@ def run_reference(args):
     from paper_conf_asplos_azamifb25_b200 import datagen
     oracle.lib()
     sample_bytes = 1 << 20
+    cuda = torch.cuda.is_available()
     samples = []
-    for cfg, names, codecs in ((SP_CONFIG, SP_FIELDS, ("SPspeed", "SPratio")),
-                               (DP_CONFIG, DP_FIELDS, ("DPspeed", "DPratio"))):
+    for cfg, names, codecs in FIELD_SETS:
         for nm in names:
-            if cfg == DP_CONFIG:
-                x = datagen.field(cfg, nm, device="cpu", origin=(0, 0, 0), shape=(2, 384, 384))
-            else:
-                x = datagen.field(cfg, nm, device="cpu")
+            if cuda:  # the lcf arm's exact fields (generated on the device, as there)
+                x = datagen.field(cfg, nm, device="cuda").reshape(-1)[: sample_bytes // 4].cpu()
+            elif cfg.startswith("hacc"):  # (generated whole; a prefix of a shorter array of the same kind)
+                x = datagen._hacc(nm, datagen._gen(datagen.seed_of(5, {"xx": 0, "vx": 1}[nm]), "cpu"), "cpu",
+                                  (sample_bytes // 4,), None)
+            else:  # the leading planes of the field, drawn on the host
+                shape = datagen.CONFIGS[cfg][1]
+                sub = (max(1, (sample_bytes // (4 if cfg.endswith("f32") else 8)) // (shape[-1] * (
+                    shape[-2] if len(shape) == 3 else 1)) + 1),) + tuple(shape[1:])
+                x = datagen.field(cfg, nm, device="cpu", origin=(0,) * len(shape), shape=sub)
             w = x.numpy().reshape(-1).view(np.uint32 if x.dtype == torch.float32 else np.uint64)
             w = w[: sample_bytes // w.itemsize].copy()
             for c in codecs:
@@ -521,11 +587,43 @@ def run_reference(args):
         "impl": "reference", "metric": "compress+decompress throughput (uncompressed GB/s)", "value": v,
         "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/u64 (f32/f64 bits)",
-        "data": "synthetic", "config": {"workload": WORKLOAD, "sample": "first 1 MiB of every (codec, field)"},
+        "data": "synthetic", "config": {"workload": WORKLOAD, "sample": "first 1 MiB of every (codec, field)",
+                                        "l2": "n/a (host oracle)"},
         "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
                          "sample": "first 1 MiB of every (codec, field) of the workload per step"},
         "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }))
+
+
+def spawn_ranks(args) -> int:
+    """`--gpus N` without a launcher: re-run this script under
+    torch.distributed.run with N processes on this node (127.0.0.1), one per
+    GPU; rank 0's JSON line is the output."""
+    import socket
+    sock = socket.socket()
+    sock.bind(("127.0.0.1", 0))
+    port = sock.getsockname()[1]
+    sock.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def dry_run(args):
+    """--dry-run: the multi-rank plumbing only (process group, rank layout,
+    the max-over-ranks reduction) — no device work; gloo when there is no GPU."""
+    import torch.distributed as dist
+    world, rank, local = dist_env()
+    if world > 1:
+        dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
+    t = torch.tensor([float(rank + 1)])
+    if world > 1 and not torch.cuda.is_available():
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": world, "max_over_ranks": float(t.item()),
+                          "backend": dist.get_backend() if world > 1 else None}))
+    if world > 1:
+        dist.destroy_process_group()
 
 
 def main():
@@ -536,12 +634,23 @@ def main():
     ap.add_argument("--impl", default="lcf", choices=["lcf", "reference"])
     ap.add_argument("--codecs", default=",".join(ALL_CODECS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--transfer", action="store_true",
-                    help="N >= 2: also time rank 0 -> rank 1 raw vs compressed NCCL transfer (transfer.py)")
+    ap.add_argument("--no-transfer", action="store_true",
+                    help="N >= 2: skip the rank 0 -> rank 1 raw vs compressed NCCL transfer (transfer.py)")
+    ap.add_argument("--dry-run", action="store_true", help="multi-rank plumbing only (tests)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
-    if args.impl == "reference":
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        if not args.dry_run and args.impl == "lcf" and torch.cuda.device_count() < args.gpus:
+            sys.exit(f"bench.py --gpus {args.gpus}: only {torch.cuda.device_count()} CUDA devices visible")
+        sys.exit(spawn_ranks(args))
+    if world != args.gpus and not (args.impl == "reference" and world == 1):
+        sys.exit(f"bench.py --gpus {args.gpus} launched with WORLD_SIZE={world}")
+    args.transfer = not args.no_transfer
+    if args.dry_run:
+        dry_run(args)
+    elif args.impl == "reference":
         run_reference(args)
     else:
         run_lcf(args)

@@ -1125,6 +1125,7 @@ __device__ __forceinline__ uint64_t dp_hi(const DpViews& V, const uint8_t* strea
   return hi;
 }
 
+template <bool kSingle>
 __global__ void __launch_bounds__(256) dp_find_roots_kernel(const __grid_constant__ DpViews V, const uint8_t* stream,
                                                            uint64_t w_lo, uint64_t w_hi, LaunchCtx ctx,
                                                            const uint32_t* any_pend) {
@@ -1137,20 +1138,31 @@ __global__ void __launch_bounds__(256) dp_find_roots_kernel(const __grid_constan
     const uint64_t li = base + lane;
     if (!((bits >> lane) & 1) || li >= hi) continue;
     uint64_t cur = me.first + li, t = __ldcg(me.out + li);
-    uint32_t hops = 0;
     bool err = false;
     for (;;) {
       if (t >= cur) { err = true; break; }  // chains point strictly backwards
-      const DpView& w = V.v[dp_owner(V, t)];
+      const DpView& w = V.v[kSingle ? 0 : dp_owner(V, t)];
       if (t < w.first || t - w.first >= w.n) { err = true; break; }
       const uint64_t lj = t - w.first;
-      if (!((ld_relaxed_sys_u32(w.pend + lj / 32) >> (lj % 32)) & 1)) break;  // final: the root
+      // the bit and the word are fetched together (one round trip per hop)
+      uint32_t pw;
+      uint64_t nt;
+      if (kSingle) {
+        pw = __ldcg(w.pend + lj / 32);
+        nt = ld_relaxed_u64(w.out + lj);
+      } else {
+        pw = ld_relaxed_sys_u32(w.pend + lj / 32);
+        nt = ld_relaxed_sys_u64(w.out + lj);
+      }
+      if (!((pw >> (lj % 32)) & 1)) break;  // final: the root
       cur = t;
-      t = ld_relaxed_sys_u64(w.out + lj);
-      if ((++hops & 3) == 0) st_relaxed_sys_u64(me.out + li, t);
+      t = nt;
+      // every hop is written back: walkers through this word jump to where
+      // this walk has got (concurrent pointer doubling)
+      if (kSingle) st_relaxed_u64(me.out + li, t);
+      else st_relaxed_sys_u64(me.out + li, t);
     }
     if (err) record_error(ctx, DERR_CORRUPT);
-    else st_relaxed_sys_u64(me.out + li, t);
   }
 }
 
@@ -1189,8 +1201,12 @@ void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo
                           const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
   if (w_hi <= w_lo) return;
   KTrace kt("dp_find_roots", st);
-  dp_find_roots_kernel<<<roots_grid((const void*)dp_find_roots_kernel, w_hi - w_lo), 256, 0, st>>>(
-      v, stream, w_lo, w_hi, ctx, any_pend);
+  if (v.count == 1)
+    dp_find_roots_kernel<true><<<roots_grid((const void*)dp_find_roots_kernel<true>, w_hi - w_lo), 256, 0, st>>>(
+        v, stream, w_lo, w_hi, ctx, any_pend);
+  else
+    dp_find_roots_kernel<false><<<roots_grid((const void*)dp_find_roots_kernel<false>, w_hi - w_lo), 256, 0, st>>>(
+        v, stream, w_lo, w_hi, ctx, any_pend);
 }
 
 void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,

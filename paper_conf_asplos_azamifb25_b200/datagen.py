@@ -211,3 +211,32 @@ def adversarial(word_bits: int, seed: int = 7):
     for n in (1, 2, 3, 31, 32, 33, 63, 64, 65, 127, 128, 129, cw - 1, cw, cw + 1, 3 * cw + 1035):
         out.append((f"tail_{n}", smooth(n, 4 + n)))
     return out
+
+
+# --- every f32 bit pattern once -------------------------------------
+# word i = P(i) for i in [0, 2^32), P the "lowbias32" integer mixer (xor-shift
+# and odd-multiplier steps, each a bijection of u32): a seeded-looking order in
+# which every 32-bit pattern appears exactly once. Host (numpy) and device
+# (torch) give the same words.
+_MIX = (16, 0x7FEB352D, 15, 0x846CA68B, 16)
+
+
+def all_f32_patterns(start: int, count: int, device=None):
+    """Words [start, start + count) of the permutation; numpy uint32 on the
+    host (device None), else an int32 torch tensor on `device`."""
+    if device is None:
+        x = np.arange(start, start + count, dtype=np.uint64).astype(np.uint32)
+        x ^= x >> np.uint32(_MIX[0])
+        x *= np.uint32(_MIX[1])
+        x ^= x >> np.uint32(_MIX[2])
+        x *= np.uint32(_MIX[3])
+        x ^= x >> np.uint32(_MIX[4])
+        return x
+    m = 0xFFFFFFFF
+    x = torch.arange(start, start + count, dtype=torch.int64, device=device)
+    x = x ^ (x >> _MIX[0])
+    x = (x * _MIX[1]) & m
+    x = x ^ (x >> _MIX[2])
+    x = (x * _MIX[3]) & m
+    x = x ^ (x >> _MIX[4])
+    return x.to(torch.int32)  # wraps to the same 32 bits

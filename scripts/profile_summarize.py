@@ -10,7 +10,7 @@ import subprocess
 import sys
 from collections import defaultdict
 
-tag = sys.argv[1] if len(sys.argv) > 1 else "r1"
+tag = sys.argv[1] if len(sys.argv) > 1 else "r2"
 src = f"gpurun_out/prof_{tag}"
 os.makedirs("profiles", exist_ok=True)
 
@@ -23,11 +23,14 @@ def short(name):
     for k in ("speed_encode_kernel<unsigned int>", "speed_encode_kernel<unsigned long>",
               "speed_decode_kernel<unsigned int>", "speed_decode_kernel<unsigned long>",
               "spratio_encode_kernel", "spratio_decode_kernel", "dpratio_encode_kernel", "dpratio_decode_kernel",
-              "fcm_hash_kernel", "fcm_match_kernel", "DeviceRadixSortOnesweepKernel", "DeviceRadixSortHistogramKernel",
+              "fcm_hash_kernel", "fcm_match_kernel", "dp_find_roots_kernel", "dp_gather_roots_kernel",
+              "fcm_carry_merge_kernel", "fcm_summary_kernel", "DeviceRadixSortOnesweepKernel", "DeviceRadixSortHistogramKernel",
               "DeviceRadixSortExclusiveSumKernel", "write_header_kernel"):
         if k in name:
             return (k.replace("_kernel<unsigned int>", "_u32").replace("_kernel<unsigned long>", "_u64")
                     .replace("_kernel", ""))
+    if "spratio_encode" in name or "spratio_decode" in name:
+        return "spratio_encode" if "encode" in name else "spratio_decode"
     return None
 
 

@@ -47,10 +47,21 @@ template <int J, uint32_t M> __device__ __forceinline__ void tp_stage(uint32_t (
     A[k + J] ^= t << J;
   }
 }
+// The 16- and 8-bit stages move whole bytes: one byte permute per word
+// instead of the shift/xor/mask sequence.
+template <int J, uint32_t SLO, uint32_t SHI> __device__ __forceinline__ void tp_stage_bytes(uint32_t (&A)[32]) {
+#pragma unroll
+  for (int k = 0; k < 32; ++k) {
+    if (k & J) continue;
+    const uint32_t lo = __byte_perm(A[k], A[k + J], SLO), hi = __byte_perm(A[k], A[k + J], SHI);
+    A[k] = lo;
+    A[k + J] = hi;
+  }
+}
 // A[i] = row i with column c at bit 31−c  →  A'[c] bit (31−i) = A[i] bit (31−c)
 __device__ __forceinline__ void transpose32(uint32_t (&A)[32]) {
-  tp_stage<16, 0x0000FFFFu>(A);
-  tp_stage<8, 0x00FF00FFu>(A);
+  tp_stage_bytes<16, 0x3276u, 0x1054u>(A);  // ≡ tp_stage<16, 0x0000FFFF>
+  tp_stage_bytes<8, 0x3715u, 0x2604u>(A);   // ≡ tp_stage<8, 0x00FF00FF>
   tp_stage<4, 0x0F0F0F0Fu>(A);
   tp_stage<2, 0x33333333u>(A);
   tp_stage<1, 0x55555555u>(A);
@@ -269,12 +280,12 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
       trace_stamp(a, t, 2);
     }
     if (g == 0) trace_stamp(a, t, 3);
-    uint8_t* ob = reinterpret_cast<uint8_t*>(S.in[s]);
     if (cw == 0 && lane == 0) {
       S.out_chunk[s] = t;
       S.out_len[s] = len;
       S.out_raw[s] = raw;
     }
+    uint8_t* ob = reinterpret_cast<uint8_t*>(S.in[s]);
     if (raw) {  // the stage still holds the raw chunk: zero its padding
       if (g < round16(len) - len) ob[len + g] = 0;
     } else {
@@ -319,7 +330,7 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
   }
 }
 
-__global__ void __launch_bounds__(kREncThreads) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kREncThreads, 4) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

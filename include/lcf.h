@@ -178,8 +178,10 @@ lcf_status_t lcf_write_header(lcf_algo_t algo, lcf_dtype_t dtype, size_t total_i
  * follows FCM chains inside a tile (L197); a word whose distance leaves its
  * tile is read if that tile is already complete, else it is left PENDING:
  * d_out holds the global index of the word it copies and its bit in
- * d_pending is set (u32 bitmap of ceil(out_capacity / 8 / 32) words, fully
- * written by the call). Asynchronous; malformed input is reported by
+ * d_pending is set. d_pending holds 2·ceil(n / 32) u32 words, n =
+ * out_capacity / 8: the pending bitmap, then a bitmap marking the words that
+ * pending words point at (the chain nodes, walked first by find_roots); the
+ * call clears and writes both. Asynchronous; malformed input is reported by
  * lcf_check_stream. The pending words are then resolved over all shards, each
  * described by an lcf_dp_view (its words and bitmap — local pointers or
  * CUDA-IPC-mapped peer pointers; views sorted by first_word, contiguous from
@@ -200,7 +202,7 @@ typedef struct {
   uint64_t first_word;  /* global index of the view's word 0 */
   uint64_t n_words;     /* words in the view */
   void* d_words;        /* its decoded words (u64), device */
-  uint32_t* d_pending;  /* its pending bitmap, device */
+  uint32_t* d_pending;  /* its 2·ceil(n_words / 32) bitmap words (see above), device */
 } lcf_dp_view;
 size_t lcf_dpratio_summary_bytes(void);
 lcf_status_t lcf_dpratio_shard_summary(const void* d_x, size_t shard_bytes, size_t total_in_bytes, uint64_t first_word,

@@ -288,20 +288,22 @@ lcf_status_t lcf_compress(lcf_algo_t algo, lcf_dtype_t dtype, const void* d_in, 
 // words it left pending (single view: the whole output). Caller holds ws->mu.
 static lcf_status_t dpratio_decode_range(Workspace* ws, DecArgs a, const LaunchCtx& ctx, uint64_t max_tiles,
                                          uint64_t end_tile, cudaStream_t stream) {
-  const uint64_t words = a.out_capacity / 8;
+  const uint64_t words = a.out_capacity / 8, W = (words + 31) / 32 + 1;
   lcf_status_t st;
-  if ((st = grow(ws->pend, ws->pend_cap, (words + 31) / 32 + 1, stream, true))) return st;
+  if ((st = grow(ws->pend, ws->pend_cap, 2 * W, stream, true))) return st;  // pending bits ‖ chain-node marks
   a.pend = ws->pend;
+  a.tgt = ws->pend + W;
   a.any_pend = ws->any_pend;
   launch_dpratio_decode(a, ctx, max_tiles, stream);
   DpViews v{};
   v.count = 1;
   v.self = 0;
-  v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend};
+  v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend, ws->pend + W};
   const uint64_t lo = a.first_tile * 2048, hi = end_tile ? end_tile * 2048 : words;
-  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream);
+  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 0);  // chain nodes
+  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 1);  // the rest
   launch_dp_gather_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream);
-  g_launches += 2;
+  g_launches += 3;
   return LCF_SUCCESS;
 }
 
@@ -1021,7 +1023,8 @@ lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uin
   if ((st = grow(ws->status, ws->status_cap, grid, stream, true)) ||
       (st = grow(ws->tile_flag, ws->tile_cap, grid / 2 + 1, stream, true)))
     return st;
-  if (!cuda_ok(cudaMemsetAsync(d_pending, 0, 4 * ((out_capacity / 8 + 31) / 32), stream))) return LCF_ERROR_CUDA;
+  const uint64_t W = (out_capacity / 8 + 31) / 32;  // d_pending: pending bits ‖ chain-node marks
+  if (!cuda_ok(cudaMemsetAsync(d_pending, 0, 2 * 4 * W, stream))) return LCF_ERROR_CUDA;
   DecArgs a{};
   a.stream = static_cast<const uint8_t*>(d_in);
   a.stream_bytes = in_bytes;
@@ -1032,6 +1035,7 @@ lcf_status_t lcf_dpratio_decompress_shard(const void* d_in, size_t in_bytes, uin
   a.tile_flag = ws->tile_flag;
   a.gbase = first_word;
   a.pend = d_pending;
+  a.tgt = d_pending + W;
   a.any_pend = ws->any_pend;
   LaunchCtx ctx = make_ctx(ws);
   launch_dpratio_decode(a, ctx, grid / 2 + 1, stream);
@@ -1049,7 +1053,8 @@ static lcf_status_t dp_views(const lcf_dp_view* views, size_t count, size_t self
     if (q ? w.first_word != views[q - 1].first_word + views[q - 1].n_words : w.first_word != 0)
       return LCF_ERROR_INVALID_ARGUMENT;  // sorted, contiguous from word 0
     if (w.n_words && (!w.d_words || !w.d_pending)) return LCF_ERROR_INVALID_ARGUMENT;
-    v.v[q] = DpView{w.first_word, w.n_words, static_cast<uint64_t*>(w.d_words), w.d_pending};
+    v.v[q] = DpView{w.first_word, w.n_words, static_cast<uint64_t*>(w.d_words), w.d_pending,
+                    w.d_pending + (w.n_words + 31) / 32};
   }
   if (views[self].first_word % 32) return LCF_ERROR_INVALID_ARGUMENT;
   return LCF_SUCCESS;
@@ -1065,9 +1070,14 @@ static lcf_status_t dp_roots(const lcf_dp_view* views, size_t count, size_t self
   std::lock_guard<std::mutex> g(ws->mu);
   LaunchCtx ctx = make_ctx(ws);
   const uint64_t n = views[self].n_words;
-  if (gather) launch_dp_gather_roots(v, nullptr, 0, n, ctx, nullptr, stream);
-  else launch_dp_find_roots(v, nullptr, 0, n, ctx, nullptr, stream);
-  if (n) ++g_launches;
+  if (gather) {
+    launch_dp_gather_roots(v, nullptr, 0, n, ctx, nullptr, stream);
+    if (n) ++g_launches;
+  } else {
+    launch_dp_find_roots(v, nullptr, 0, n, ctx, nullptr, stream, 0);  // chain nodes first
+    launch_dp_find_roots(v, nullptr, 0, n, ctx, nullptr, stream, 1);
+    if (n) g_launches += 2;
+  }
   return last_launch_status();
 }
 

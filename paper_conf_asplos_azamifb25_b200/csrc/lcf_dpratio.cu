@@ -1023,6 +1023,21 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
         }
         if (li < m) S.X[li] = val;  // x (or a pending target), in place
         if (li < m && f) atomicOr(&S.pmask[li / 32], 1u << (li % 32));
+        // mark the word a pending word points at (a chain node, walked first by
+        // dp_find_roots); lanes hitting the same bitmap word send one OR
+        const bool mk = li < m && f && val >= gb && val - gb < n_words;
+        const uint32_t mkmask = __ballot_sync(0xFFFFFFFFu, mk);
+        if (mk) {
+          const uint64_t lt = val - gb;
+          const uint32_t key = (uint32_t)(lt / 32), lead = __ffs(mkmask) - 1;
+          const uint32_t key0 = __shfl_sync(mkmask, key, lead);
+          if (__all_sync(mkmask, key == key0)) {  // the usual case: one bitmap word for the warp
+            const uint32_t bitsum = __reduce_or_sync(mkmask, 1u << (lt % 32));
+            if ((threadIdx.x & 31) == lead) atomicOr(a.tgt + key, bitsum);
+          } else {
+            atomicOr(a.tgt + key, 1u << (lt % 32));
+          }
+        }
         bar_d();
       }
       // the tile's pending bits, before its completion flag (released after a barrier)
@@ -1080,10 +1095,12 @@ int launch_dpratio_encode(const EncArgs& a0, const LaunchCtx& ctx, void* ws, siz
   int launches = 0;
   if (n) {
     uint32_t* dist = nullptr;  // FCM distances (L170–185), lcf_fcm.cu; a shard's with its carry
+    const uint64_t* srt = nullptr;
     launches += launch_fcm_shard(reinterpret_cast<const uint64_t*>(a0.in), n, halo, gbase, carry, nullptr, true, ws,
-                                 ws_bytes, st, &dist, sorted);
+                                 ws_bytes, st, &dist, sorted, &srt);
     EncArgs a = a0;
     a.fcm_dist = dist;
+    (void)srt;
     const size_t smem = sizeof(DEncSmem);
     static const bool init = [&] {
       cudaFuncSetAttribute(dpratio_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1128,13 +1145,18 @@ __device__ __forceinline__ uint64_t dp_hi(const DpViews& V, const uint8_t* strea
 template <bool kSingle>
 __global__ void __launch_bounds__(256) dp_find_roots_kernel(const __grid_constant__ DpViews V, const uint8_t* stream,
                                                            uint64_t w_lo, uint64_t w_hi, LaunchCtx ctx,
-                                                           const uint32_t* any_pend) {
+                                                           const uint32_t* any_pend, int mode) {
   if (any_pend && *any_pend != ctx.epoch) return;
   const DpView& me = V.v[V.self];
   const uint64_t hi = dp_hi(V, stream, w_hi);
   const uint32_t lane = threadIdx.x & 31;
   for (uint64_t base = w_lo + (blockIdx.x * 256ull + threadIdx.x - lane); base < hi; base += gridDim.x * 256ull) {
-    const uint32_t bits = __ldcg(me.pend + base / 32);  // one bitmap word per warp (w_lo % 32 == 0)
+    uint32_t bits = __ldcg(me.pend + base / 32);  // one bitmap word per warp (w_lo % 32 == 0)
+    if (!bits) continue;
+    if (mode != 2) {
+      const uint32_t nodes = __ldcg(me.tgt + base / 32);
+      bits &= mode == 0 ? nodes : ~nodes;
+    }
     const uint64_t li = base + lane;
     if (!((bits >> lane) & 1) || li >= hi) continue;
     uint64_t cur = me.first + li, t = __ldcg(me.out + li);
@@ -1177,7 +1199,10 @@ __global__ void __launch_bounds__(256) dp_gather_roots_kernel(const __grid_const
   const uint32_t lane = threadIdx.x & 31;
   for (uint64_t base = w_lo + (blockIdx.x * 256ull + threadIdx.x - lane); base < hi; base += gridDim.x * 256ull) {
     const uint32_t bits = __ldcg(me.pend + base / 32);
-    if (!bits) continue;  // warp-uniform
+    if (!bits) {  // warp-uniform; a chain node that is not pending may still be marked
+      if (lane == 0) me.tgt[base / 32] = 0;
+      continue;
+    }
     const uint64_t li = base + lane;
     if (((bits >> lane) & 1) && li < hi) {
       const uint64_t r = __ldcg(me.out + li);
@@ -1186,7 +1211,10 @@ __global__ void __launch_bounds__(256) dp_gather_roots_kernel(const __grid_const
       else me.out[li] = ld_relaxed_sys_u64(w.out + (r - w.first));
     }
     __syncwarp();
-    if (lane == 0) me.pend[base / 32] = 0;
+    if (lane == 0) {
+      me.pend[base / 32] = 0;
+      me.tgt[base / 32] = 0;
+    }
   }
 }
 
@@ -1198,15 +1226,15 @@ int roots_grid(const void* kern, uint64_t words) {
 }  // namespace
 
 void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
-                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
+                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st, int mode) {
   if (w_hi <= w_lo) return;
   KTrace kt("dp_find_roots", st);
   if (v.count == 1)
     dp_find_roots_kernel<true><<<roots_grid((const void*)dp_find_roots_kernel<true>, w_hi - w_lo), 256, 0, st>>>(
-        v, stream, w_lo, w_hi, ctx, any_pend);
+        v, stream, w_lo, w_hi, ctx, any_pend, mode);
   else
     dp_find_roots_kernel<false><<<roots_grid((const void*)dp_find_roots_kernel<false>, w_hi - w_lo), 256, 0, st>>>(
-        v, stream, w_lo, w_hi, ctx, any_pend);
+        v, stream, w_lo, w_hi, ctx, any_pend, mode);
 }
 
 void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,

@@ -19,20 +19,23 @@
 //   sort_scatter per-warp digit counts → per-warp offsets inside the tile's
 //                digit run; then each warp walks its records in order and
 //                ranks equal digits with __match_any_sync → stable scatter
+#include "lcf_fcm.cuh"
 #include "lcf_kernels.cuh"
 
 namespace lcf {
 namespace {
 
-constexpr uint64_t FCM_K1 = 0x9E3779B97F4A7C15ull, FCM_K2 = 0xC2B2AE3D27D4EB4Full, FCM_K3 = 0x165667B19E3779F9ull;
+using fcm::hi_mul;
+using fcm::kRecFpShift;
+using fcm::kRecHashShift;
+using fcm::kRecIdxMask;
+constexpr uint64_t FCM_K1 = fcm::K1, FCM_K2 = fcm::K2, FCM_K3 = fcm::K3;
 constexpr int kDigitBits = 10, kDigits = 1 << kDigitBits;
 #ifndef LCF_WARP_RECS
 #define LCF_WARP_RECS 1024
 #endif
 constexpr int kSortWarps = 16, kSortThreads = kSortWarps * 32, kWarpRecs = LCF_WARP_RECS;
 constexpr uint32_t kTile = kSortWarps * kWarpRecs;
-constexpr int kRecHashShift = 44, kRecFpShift = 32;
-constexpr uint64_t kRecIdxMask = 0xFFFFFFFFull;
 constexpr uint32_t kNoDigit = kDigits;  // records past n
 constexpr int kMatchBlock = 256;
 constexpr int kScanWarps = 32, kScanBlocks = kDigits / 8;  // 8 digits per CTA (sort_scan_kernel)
@@ -49,7 +52,6 @@ __device__ __forceinline__ uint64_t make_rec(uint64_t xi, uint32_t hw, uint64_t 
   const uint32_t fp = (f ^ (f >> 12) ^ (f >> 24)) & 0xFFFu;
   return (h << kRecHashShift) | ((uint64_t)fp << kRecFpShift) | i;
 }
-__device__ __forceinline__ uint32_t hi_mul(uint64_t a, uint64_t k) { return (uint32_t)((a * k) >> 32); }
 
 // Lanes of the warp holding the same digit as this lane (valid lanes only):
 // ten ballots, one per digit bit — ALU-pipe votes instead of __match_any_sync,
@@ -447,6 +449,27 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
       uint32_t d = 0, used = 0;
       uint64_t xi = 0;
       bool have = false;
+      if constexpr (!CARRY) {
+        // deferred (no gather of x here): the nearest candidate with the same
+        // hash and fingerprint, flagged if another one follows in the window;
+        // the DPratio encoder compares the words in index order (L2-near for
+        // repeats a few rows apart) and falls back to fcm::match_one only when
+        // the nearest fails and another candidate exists
+#pragma unroll
+        for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
+          if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
+          const uint32_t hb = hw[4 + j - back];
+          if ((hb ^ hk) >> 12) break;  // left the hash's run
+          if (hb == hk) {
+            if (d) {
+              d |= fcm::kMulti;
+              break;
+            }
+            d = i - (uint32_t)(r[4 + j - back] & kRecIdxMask);
+          }
+        }
+        if (d) dist[i] = d;
+      } else {
 #pragma unroll
       for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
         if ((uint64_t)back > k) break;        // sorted position k has only k predecessors
@@ -481,6 +504,7 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
         }
       }
       if (d) dist[i] = d;
+      }
     }
   }
 }
@@ -532,6 +556,39 @@ __global__ void __launch_bounds__(256) fcm_carry_merge_kernel(const __grid_const
   out[h] = (uint8_t)m;
 }
 
+// The deferred candidates of the match kernel (distance | fcm::kMulti), in
+// index order: x[i] is read coalesced and x[i − d] is L2-near for repeats a
+// few rows back (a gather in sorted order costs two random sectors per
+// candidate). A failed nearest candidate with another one in its window falls
+// back to the full match of that word (fcm::match_one, rare).
+__global__ void __launch_bounds__(256) fcm_verify_kernel(const uint64_t* __restrict__ x, uint64_t n,
+                                                        const uint64_t* __restrict__ rec, uint32_t* __restrict__ dist,
+                                                        uint32_t halo) {
+  const uint64_t q4 = (n + 3) / 4;
+  for (uint64_t q = blockIdx.x * 256ull + threadIdx.x; q < q4; q += (uint64_t)gridDim.x * 256) {
+    uint4 dv;
+    if (4 * q + 4 <= n) {
+      dv = __ldcs(reinterpret_cast<const uint4*>(dist) + q);
+    } else {
+      dv.x = dist[4 * q];
+      dv.y = 4 * q + 1 < n ? dist[4 * q + 1] : 0u;
+      dv.z = 4 * q + 2 < n ? dist[4 * q + 2] : 0u;
+      dv.w = 4 * q + 3 < n ? dist[4 * q + 3] : 0u;
+    }
+    if (!(dv.x | dv.y | dv.z | dv.w)) continue;
+    const uint32_t raw[4] = {dv.x, dv.y, dv.z, dv.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if (!raw[j]) continue;
+      const uint64_t i = 4 * q + j;
+      const uint32_t d = raw[j] & ~fcm::kMulti;
+      uint32_t v = d <= i && x[i - d] == x[i] ? d : 0u;
+      if (!v && (raw[j] & fcm::kMulti)) v = fcm::match_one(x, rec, n, (uint32_t)i, halo);
+      if (v != raw[j]) dist[i] = v;
+    }
+  }
+}
+
 uint64_t n_tiles_of(uint64_t n) { return (n + kTile - 1) / kTile; }
 
 }  // namespace
@@ -551,7 +608,8 @@ bool fcm_empty_carry(void* carry, cudaStream_t st) { return cudaMemsetAsync(carr
 // summaries of the earlier shards, or null). summary (optional) receives this
 // shard's own summary; with match false only the summary is made.
 int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
-                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out, bool sorted) {
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out, bool sorted,
+                     const uint64_t** sorted_out) {
   (void)ws_bytes;
   uint8_t* p = static_cast<uint8_t*>(ws);
   uint64_t* rec_a = reinterpret_cast<uint64_t*>(p);
@@ -561,6 +619,7 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
   uint32_t* tot = reinterpret_cast<uint32_t*>(p + 2 * round16(8 * n) + round16(4 * T * kDigits));
   uint32_t* dist = reinterpret_cast<uint32_t*>(rec_a);  // pass-1 records are dead after pass 2
   *dist_out = dist;
+  if (sorted_out) *sorted_out = rec_b;
   if (n == 0) {
     if (summary) cudaMemsetAsync(summary, 0, kHashes, st);  // no entries
     return 0;
@@ -620,11 +679,17 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
     if (carry) fcm_match_kernel<true><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
     else fcm_match_kernel<false><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
   }
+  if (!carry) {  // deferred candidates → distances
+    KTrace kt("fcm_verify", st);
+    const int vblocks = (int)umin64(((n + 3) / 4 + 255) / 256, 148 * 8);
+    fcm_verify_kernel<<<vblocks, 256, 0, st>>>(x, n, rec_b, dist, halo);
+    ++launches;
+  }
   return launches + 1;
 }
 
 int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist_out) {
-  return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out, false);
+  return launch_fcm_shard(x, n, 0, 0, nullptr, nullptr, true, ws, ws_bytes, st, dist_out, false, nullptr);
 }
 
 int launch_fcm_carry_merge(const void* const* summaries, uint32_t count, void* carry, cudaStream_t st) {

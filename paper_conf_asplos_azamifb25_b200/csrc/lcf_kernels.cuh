@@ -80,6 +80,7 @@ struct DecArgs {
   // its bitmap words) is set; any_pend ← epoch if any word is.
   uint64_t gbase;
   uint32_t* pend;
+  uint32_t* tgt;       // bitmap of the words some pending word points at (chain nodes)
   uint32_t* any_pend;
 };
 
@@ -92,6 +93,7 @@ struct DpView {
   uint64_t first, n;
   uint64_t* out;
   uint32_t* pend;
+  uint32_t* tgt;  // chain-node marks (same indexing as pend)
 };
 struct DpViews {
   uint32_t count, self;
@@ -186,7 +188,8 @@ int launch_fcm_dist(const uint64_t* x, uint64_t n, void* ws, size_t ws_bytes, cu
 size_t fcm_carry_bytes();
 bool fcm_empty_carry(void* carry, cudaStream_t st);
 int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbase, const void* carry, void* summary,
-                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist, bool sorted = false);
+                     bool match, void* ws, size_t ws_bytes, cudaStream_t st, uint32_t** dist, bool sorted = false,
+                     const uint64_t** sorted_out = nullptr);
 // summaries: host array of `count` (≤ 64) device pointers, shard order
 int launch_fcm_carry_merge(const void* const* summaries, uint32_t count, void* carry, cudaStream_t st);
 size_t dpratio_fcm_workspace(uint64_t n_words);
@@ -196,12 +199,14 @@ void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
 // Root resolution of pending words of view `self`, local words [w_lo, w_hi)
 // (clamped to the stream header's word count when `stream` is given).
 // find: every pending word's target becomes its chain's root (a final word),
-// with path compression; gather: pending words take their root's value and
-// their bits are cleared. Every view's decode must be complete before any
+// with path compression — mode 0 walks the marked chain nodes only, mode 1
+// the other pending words (whose walks then end after a hop or two), mode 2
+// all of them; gather: pending words take their root's value and both
+// bitmaps are cleared. Every view's decode must be complete before any
 // find, and every find before any gather. any_pend (nullable): skip unless
 // *any_pend == ctx.epoch.
 void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
-                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
+                          const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st, int mode = 2);
 void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
                             const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
 

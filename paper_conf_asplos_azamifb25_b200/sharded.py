@@ -355,7 +355,7 @@ def dp_simulate_decode_shards(stream: bytes, world: int):
     for g in range(world):
         f, k = dp_shard_words(n, world, g)
         sub = torch.from_numpy(np.frombuffer(dp_shard_substream(stream, world, g), np.uint8).copy()).cuda()
-        p = torch.empty(max(1, (k + 31) // 32), dtype=torch.int32, device="cuda")
+        p = torch.empty(max(1, 2 * ((k + 31) // 32)), dtype=torch.int32, device="cuda")
         if k:
             lcf.lcf_dpratio_decompress_shard(sub, sub.numel(), f, out[f:f + k], 8 * k, p)
         subs.append(sub)
@@ -382,7 +382,7 @@ def dp_decompress_sharded(sub_stream, first_word: int, n_total: int, group=None)
     f, k = dp_shard_words(n_total, world, rank)
     assert f == first_word
     out = torch.empty(max(k, 1), dtype=torch.int64, device=sub_stream.device)
-    pend = torch.zeros(max(1, (k + 31) // 32), dtype=torch.int32, device=sub_stream.device)
+    pend = torch.zeros(max(1, 2 * ((k + 31) // 32)), dtype=torch.int32, device=sub_stream.device)
     if k:
         lcf.lcf_dpratio_decompress_shard(sub_stream, sub_stream.numel(), f, out, 8 * k, pend)
     lcf.lcf_check_stream()

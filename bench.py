@@ -189,6 +189,7 @@ def kernel_bytes(j):
             "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
             "dpratio_decode": sb + n,                 # stream in, x out
             "dp_find_roots": words // 8,              # the pending bitmap (the walks are data-dependent)
+            "dp_gather_leaves": words // 8,
             "dp_gather_roots": words // 8}
 
 

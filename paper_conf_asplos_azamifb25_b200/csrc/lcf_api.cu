@@ -32,6 +32,10 @@ struct Workspace {
   size_t tile_cap = 0;
   uint32_t* pend = nullptr;              // DPratio decode pending-word bitmap (1 bit per word)
   size_t pend_cap = 0;
+  uint32_t* tgt = nullptr;               // DPratio decode chain-node marks (1 bit per word)
+  size_t tgt_cap = 0;
+  uint32_t* nodes = nullptr;             // DPratio decode chain-node list: [0] count, then indices
+  size_t nodes_cap = 0;
   uint32_t* any_pend = nullptr;          // DPratio decode: epoch of the newest launch with a pending word
   uint32_t* err = nullptr;               // (epoch << 8 | bits) of the newest failure
   uint32_t epoch = 0, checked_epoch = 0;
@@ -290,20 +294,32 @@ static lcf_status_t dpratio_decode_range(Workspace* ws, DecArgs a, const LaunchC
                                          uint64_t end_tile, cudaStream_t stream) {
   const uint64_t words = a.out_capacity / 8, W = (words + 31) / 32 + 1;
   lcf_status_t st;
-  if ((st = grow(ws->pend, ws->pend_cap, 2 * W, stream, true))) return st;  // pending bits ‖ chain-node marks
+  // (each bitmap in its own buffer: the layout must not depend on the call's
+  // size, since every call leaves both bitmaps zero only where it wrote)
+  if ((st = grow(ws->pend, ws->pend_cap, W, stream, true)) || (st = grow(ws->tgt, ws->tgt_cap, W, stream, true)) ||
+      (st = grow(ws->nodes, ws->nodes_cap, words + 4, stream, false)))
+    return st;
+  uint32_t* cnt = ws->nodes;
   a.pend = ws->pend;
-  a.tgt = ws->pend + W;
+  a.tgt = ws->tgt;
   a.any_pend = ws->any_pend;
+  a.n_nodes = cnt;
+  a.nodes = cnt + 4;
+  if (!cuda_ok(cudaMemsetAsync(cnt, 0, 4, stream))) return LCF_ERROR_CUDA;
   launch_dpratio_decode(a, ctx, max_tiles, stream);
   DpViews v{};
   v.count = 1;
   v.self = 0;
-  v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend, ws->pend + W};
-  const uint64_t lo = a.first_tile * 2048, hi = end_tile ? end_tile * 2048 : words;
-  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 0);  // chain nodes
-  launch_dp_find_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 1);  // the rest
-  launch_dp_gather_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream);
+  v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend, ws->tgt};
+  const uint64_t lo = a.first_tile * 2048, hi = end_tile && end_tile * 2048 < words ? end_tile * 2048 : words;
+  launch_dp_nodes(v.v[0], a.nodes, cnt, words, ctx, ws->any_pend, false, stream);  // chain nodes → roots
+  launch_dp_gather_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 0);       // leaves, via their chain node
+  launch_dp_nodes(v.v[0], a.nodes, cnt, words, ctx, ws->any_pend, true, stream);   // chain nodes
   g_launches += 3;
+  // both bitmaps of the range back to zero (the next launch writes its tiles' words)
+  if (hi > lo && (!cuda_ok(cudaMemsetAsync(ws->pend + lo / 32, 0, 4 * ((hi + 31) / 32 - lo / 32), stream)) ||
+                  !cuda_ok(cudaMemsetAsync(ws->tgt + lo / 32, 0, 4 * ((hi + 31) / 32 - lo / 32), stream))))
+    return LCF_ERROR_CUDA;
   return LCF_SUCCESS;
 }
 

@@ -1033,9 +1033,16 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
           const uint32_t key0 = __shfl_sync(mkmask, key, lead);
           if (__all_sync(mkmask, key == key0)) {  // the usual case: one bitmap word for the warp
             const uint32_t bitsum = __reduce_or_sync(mkmask, 1u << (lt % 32));
-            if ((threadIdx.x & 31) == lead) atomicOr(a.tgt + key, bitsum);
+            if ((threadIdx.x & 31) == lead) {
+              const uint32_t fresh = bitsum & ~atomicOr(a.tgt + key, bitsum);
+              if (a.nodes && fresh) {  // first marks: onto the chain-node list
+                uint32_t k = atomicAdd(a.n_nodes, (uint32_t)__popc(fresh));
+                for (uint32_t b = fresh; b; b &= b - 1) a.nodes[k++] = 32 * key + (__ffs(b) - 1);
+              }
+            }
           } else {
-            atomicOr(a.tgt + key, 1u << (lt % 32));
+            const uint32_t bit = 1u << (lt % 32);
+            if (!(atomicOr(a.tgt + key, bit) & bit) && a.nodes) a.nodes[atomicAdd(a.n_nodes, 1u)] = (uint32_t)lt;
           }
         }
         bar_d();
@@ -1189,32 +1196,90 @@ __global__ void __launch_bounds__(256) dp_find_roots_kernel(const __grid_constan
 }
 
 // Pending words take their root's value (roots are never pending, so nothing
-// read here is being written); each bitmap word is cleared by its warp.
+// read here is being written). mode 2: every pending word (its pointer is its
+// root after the walks of modes 0 and 1); then each bitmap word is cleared.
+// Single view, chain nodes walked by mode 0 only: mode 0 gathers the other
+// pending words (leaves) through their chain node — the leaf points at a chain
+// node (marked by the decoder) or at a final word, and the chain node at its
+// root — and writes only leaves; mode 1 then gathers the chain nodes and
+// clears the bitmaps.
 __global__ void __launch_bounds__(256) dp_gather_roots_kernel(const __grid_constant__ DpViews V,
                                                              const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
-                                                             LaunchCtx ctx, const uint32_t* any_pend) {
+                                                             LaunchCtx ctx, const uint32_t* any_pend, int mode) {
   if (any_pend && *any_pend != ctx.epoch) return;
   const DpView& me = V.v[V.self];
   const uint64_t hi = dp_hi(V, stream, w_hi);
   const uint32_t lane = threadIdx.x & 31;
+  const bool clear = mode != 0;
   for (uint64_t base = w_lo + (blockIdx.x * 256ull + threadIdx.x - lane); base < hi; base += gridDim.x * 256ull) {
-    const uint32_t bits = __ldcg(me.pend + base / 32);
+    uint32_t bits = __ldcg(me.pend + base / 32);
     if (!bits) {  // warp-uniform; a chain node that is not pending may still be marked
-      if (lane == 0) me.tgt[base / 32] = 0;
+      if (clear && lane == 0) me.tgt[base / 32] = 0;
       continue;
+    }
+    if (mode != 2) {
+      const uint32_t nodes = __ldcg(me.tgt + base / 32);
+      bits &= mode == 1 ? nodes : ~nodes;
     }
     const uint64_t li = base + lane;
     if (((bits >> lane) & 1) && li < hi) {
-      const uint64_t r = __ldcg(me.out + li);
+      uint64_t r = __ldcg(me.out + li);
+      if (mode == 0 && r < me.first + li && r >= me.first) {  // a leaf: through its chain node
+        const uint64_t lr = r - me.first;
+        if ((__ldcg(me.pend + lr / 32) >> (lr % 32)) & 1) r = __ldcg(me.out + lr);
+      }
       const DpView& w = V.v[dp_owner(V, r)];
       if (r >= me.first + li || r < w.first || r - w.first >= w.n) record_error(ctx, DERR_CORRUPT);
       else me.out[li] = ld_relaxed_sys_u64(w.out + (r - w.first));
     }
-    __syncwarp();
-    if (lane == 0) {
-      me.pend[base / 32] = 0;
-      me.tgt[base / 32] = 0;
+    if (clear) {
+      __syncwarp();
+      if (lane == 0) {
+        me.pend[base / 32] = 0;
+        me.tgt[base / 32] = 0;
+      }
     }
+  }
+}
+
+// The chain-node list of a single-view decode: the walk runs over the list
+// (a few percent of the pending words on repeat-heavy data) instead of
+// scanning every bitmap word, in list order (≈ index order: tiles append as
+// they are decoded), writing back every hop.
+__global__ void __launch_bounds__(256) dp_walk_nodes_kernel(DpView me, const uint32_t* __restrict__ nodes,
+                                                           const uint32_t* __restrict__ n_nodes, uint64_t cap,
+                                                           LaunchCtx ctx, const uint32_t* any_pend) {
+  if (any_pend && *any_pend != ctx.epoch) return;
+  const uint64_t cnt = umin64(*n_nodes, cap);
+  for (uint64_t k = blockIdx.x * 256ull + threadIdx.x; k < cnt; k += (uint64_t)gridDim.x * 256) {
+    const uint64_t c = nodes[k];
+    if (c >= me.n || !((__ldcg(me.pend + c / 32) >> (c % 32)) & 1)) continue;  // a final word
+    uint64_t cur = c, t = __ldcg(me.out + c);
+    bool err = false;
+    for (;;) {
+      if (t >= cur) { err = true; break; }
+      const uint32_t pw = __ldcg(me.pend + t / 32);
+      const uint64_t nt = ld_relaxed_u64(me.out + t);
+      if (!((pw >> (t % 32)) & 1)) break;  // the root
+      cur = t;
+      t = nt;
+      st_relaxed_u64(me.out + c, t);
+    }
+    if (err) record_error(ctx, DERR_CORRUPT);
+  }
+}
+
+__global__ void __launch_bounds__(256) dp_gather_nodes_kernel(DpView me, const uint32_t* __restrict__ nodes,
+                                                             const uint32_t* __restrict__ n_nodes, uint64_t cap,
+                                                             LaunchCtx ctx, const uint32_t* any_pend) {
+  if (any_pend && *any_pend != ctx.epoch) return;
+  const uint64_t cnt = umin64(*n_nodes, cap);
+  for (uint64_t k = blockIdx.x * 256ull + threadIdx.x; k < cnt; k += (uint64_t)gridDim.x * 256) {
+    const uint64_t c = nodes[k];
+    if (c >= me.n || !((__ldcg(me.pend + c / 32) >> (c % 32)) & 1)) continue;
+    const uint64_t r = __ldcg(me.out + c);
+    if (r >= c) record_error(ctx, DERR_CORRUPT);
+    else me.out[c] = __ldcg(me.out + r);
   }
 }
 
@@ -1237,12 +1302,26 @@ void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo
         v, stream, w_lo, w_hi, ctx, any_pend, mode);
 }
 
+void launch_dp_nodes(const DpView& v, const uint32_t* nodes, const uint32_t* n_nodes, uint64_t cap,
+                     const LaunchCtx& ctx, const uint32_t* any_pend, bool gather, cudaStream_t st) {
+  if (!cap) return;
+  if (gather) {
+    KTrace kt("dp_gather_nodes", st);
+    dp_gather_nodes_kernel<<<roots_grid((const void*)dp_gather_nodes_kernel, cap), 256, 0, st>>>(v, nodes, n_nodes, cap,
+                                                                                               ctx, any_pend);
+  } else {
+    KTrace kt("dp_walk_nodes", st);
+    dp_walk_nodes_kernel<<<roots_grid((const void*)dp_walk_nodes_kernel, cap), 256, 0, st>>>(v, nodes, n_nodes, cap,
+                                                                                           ctx, any_pend);
+  }
+}
+
 void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
-                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
+                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st, int mode) {
   if (w_hi <= w_lo) return;
-  KTrace kt("dp_gather_roots", st);
+  KTrace kt(mode == 0 ? "dp_gather_leaves" : "dp_gather_roots", st);
   dp_gather_roots_kernel<<<roots_grid((const void*)dp_gather_roots_kernel, w_hi - w_lo), 256, 0, st>>>(
-      v, stream, w_lo, w_hi, ctx, any_pend);
+      v, stream, w_lo, w_hi, ctx, any_pend, mode);
 }
 
 void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_tiles, cudaStream_t st) {

@@ -82,6 +82,10 @@ struct DecArgs {
   uint32_t* pend;
   uint32_t* tgt;       // bitmap of the words some pending word points at (chain nodes)
   uint32_t* any_pend;
+  // (optional) list of the chain nodes, appended as they are first marked,
+  // and its length (zeroed before the launch)
+  uint32_t* nodes;
+  uint32_t* n_nodes;
 };
 
 // The pending-word views of the DPratio root resolution (dp_find_roots /
@@ -202,12 +206,19 @@ void launch_dpratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
 // with path compression — mode 0 walks the marked chain nodes only, mode 1
 // the other pending words (whose walks then end after a hop or two), mode 2
 // all of them; gather: pending words take their root's value and both
-// bitmaps are cleared. Every view's decode must be complete before any
+// bitmaps are cleared (mode 2; single view: mode 0 the leaves through their
+// chain nodes — no leaf walk needed — then mode 1 the chain nodes). Every view's decode must be complete before any
 // find, and every find before any gather. any_pend (nullable): skip unless
 // *any_pend == ctx.epoch.
 void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
                           const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st, int mode = 2);
 void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
-                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
+                            const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st, int mode = 2);
+// Single view with the decoder's chain-node list (nodes[0, *n_nodes), local
+// indices): walk the chain nodes to their roots (gather = false), or give them
+// their roots' values (gather = true; after the leaves' gather). `cap` bounds
+// the list (max_words).
+void launch_dp_nodes(const DpView& v, const uint32_t* nodes, const uint32_t* n_nodes, uint64_t cap,
+                     const LaunchCtx& ctx, const uint32_t* any_pend, bool gather, cudaStream_t st);
 
 }  // namespace lcf

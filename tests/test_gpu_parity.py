@@ -452,3 +452,15 @@ def test_dtype_and_argument_errors(L):
     with pytest.raises(L.LcfError) as e:
         L.lcf_compress("SPspeed", "float32", x, 400, o, 100)
     assert e.value.status == 3
+
+
+def test_dpratio_decode_call_sizes(L, orc):
+    """DPratio decodes of different sizes on one stream, chains in every one
+    (the decoder's per-stream bitmaps and chain-node list must come back clean
+    whatever the previous call's size was)."""
+    rng = np.random.default_rng(11)
+    base = rng.integers(0, 2**63, size=3000, dtype=np.uint64)
+    for n in (60 * 2048 + 3, 5 * 2048, 90 * 2048 + 1000, 2048 + 7, 33 * 2048):
+        w = np.resize(base[: 300 + n % 2000], n)
+        w[n // 3: n // 3 + 500] = rng.integers(0, 2**63, size=500, dtype=np.uint64)  # a break in the chains
+        check_parity(L, orc, "DPratio", w, f"size{n}")

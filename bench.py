@@ -185,7 +185,10 @@ def kernel_bytes(j):
     return {"fcm_sort_hist": 2 * 8 * words,           # x (pass 1) or pass-1 records (pass 2) in
             "fcm_sort_scan": 2 * 8 * 1024 * tiles,    # the tile × digit count matrix, read and rewritten
             "fcm_sort_scatter": 2 * 16 * words,       # 8-byte records (or x) in, records out
-            "fcm_match": 8 * words,                   # sorted records in (x gathered, matches scattered)
+            "fcm_match": 8 * words,                   # sorted records in (candidates scattered)
+            "fcm_verify": 4 * words,                  # the candidate array in (x read only at candidates)
+            "dp_walk_nodes": 0,                       # (data-dependent: the chain-node list)
+            "dp_gather_nodes": 0,
             "dpratio_encode": 12 * words + sb,        # x + distances in, stream out
             "dpratio_decode": sb + n,                 # stream in, x out
             "dp_find_roots": words // 8,              # the pending bitmap (the walks are data-dependent)
@@ -308,12 +311,15 @@ def run_lcf(args):
     for name, (cnt, ms) in ktimes.items():
         if name not in kbytes or ms <= 0:
             continue
+        if kbytes[name] == 0:  # data-dependent kernels: time share only
+            kernels[name] = {"launches": cnt, "avg_ms": ms / cnt, "share": 0.0, "achieved_gbs": None, "frac": None}
+            continue
         kernels[name] = {"launches": cnt, "avg_ms": ms / cnt, "share": 0.0,
                          "achieved_gbs": kbytes[name] / ms / 1e6, "frac": kbytes[name] / ms / 1e6 / hbm}
     ksum = sum(ms for _, ms in ktimes.values()) or 1.0
     for name in kernels:
         kernels[name]["share"] = ktimes[name][1] / ksum
-    own = {k: v for k, v in kernels.items() if not k.startswith("cub_")}
+    own = {k: v for k, v in kernels.items() if not k.startswith("cub_") and v["frac"] is not None}
     dom = max(own, key=lambda k: ktimes[k][1]) if own else None
     roofline = None
     traffic = kernel_traffic()

@@ -367,18 +367,17 @@ def run_lcf(args):
 
 
 def run_transfer(jobs, rank, dev, reps: int = 3):
-    """NEXT-3 (transfer.py): rank 0 → rank 1 over NCCL, the raw words
-    (dist.send) against the compressed sub-streams (send_compressed /
-    recv_compressed), per chunk-local job. GB/s = uncompressed bytes / time,
-    timed on the device (events on each rank's current stream), max over the
-    pair, median of `reps`."""
+    """NEXT-3 (transfer.py): rank 0 → rank 1, the raw words (dist.send), the
+    compressed sub-streams (send_compressed / recv_compressed, NCCL payload
+    messages) and the fused form (transfer.P2PChannel: the compress kernels
+    write the stream into rank 1's buffer over NVLink, rank 1 decompresses),
+    per job. GB/s = uncompressed bytes / time, timed on the device (events on
+    each rank's current stream), max over the pair, median of `reps`."""
     import statistics
     import torch.distributed as dist
     from paper_conf_asplos_azamifb25_b200 import transfer as tr
     out = []
     for j in jobs:
-        if j["codec"] == "DPratio":
-            continue
         x = j["x"]
         # the receiver sizes its buffer from the sender's (shards of one stream differ in length)
         nel = torch.tensor([x.numel()], dtype=torch.int64, device=dev)
@@ -387,8 +386,11 @@ def run_transfer(jobs, rank, dev, reps: int = 3):
         elif rank == 1:
             dist.recv(nel, 0)
         buf = torch.empty(int(nel.item()), dtype=x.dtype, device=dev)
+        ch = tr.P2PChannel(0, 1, j["codec"], int(nel.item()) * x.element_size()) if rank < 2 else None
         res = {}
-        for mode in ("raw", "compressed"):
+        for mode in ("raw", "compressed", "fused_p2p"):
+            if mode == "compressed" and j["codec"] == "DPratio":
+                continue
             ts = []
             for _ in range(reps):
                 dist.barrier()
@@ -398,22 +400,34 @@ def run_transfer(jobs, rank, dev, reps: int = 3):
                 if rank == 0:
                     if mode == "raw":
                         dist.send(x, 1)
-                    else:
+                    elif mode == "compressed":
                         tr.send_compressed(x, 1, j["codec"])
+                    else:
+                        ch.send(x)
                 elif rank == 1:
                     if mode == "raw":
                         dist.recv(buf, 0)
-                    else:
+                    elif mode == "compressed":
                         tr.recv_compressed(0, j["codec"], device=dev)
+                    else:
+                        ch.recv(buf)
                 e1.record()
                 torch.cuda.synchronize()
                 t = torch.tensor([e0.elapsed_time(e1) if rank < 2 else 0.0], device=dev)
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
                 ts.append(float(t.item()))
             res[mode] = j["nbytes"] / statistics.median(ts) / 1e6
+        if ch is not None:
+            ch.close()
+        dist.barrier()
         out.append({"codec": j["codec"], "field": j["field"], "bytes": j["nbytes"], "raw_gbs": res["raw"],
-                    "compressed_gbs": res["compressed"], "ratio": j["nbytes"] / j["sbytes"]})
-    return {"pair": "rank 0 -> rank 1 (NCCL)", "timing": "device events, max over the pair, median of 3",
+                    "compressed_gbs": res.get("compressed"), "fused_p2p_gbs": res["fused_p2p"],
+                    "ratio": j["nbytes"] / j["sbytes"]})
+    return {"pair": "rank 0 -> rank 1", "timing": "device events, max over the pair, median of 3",
+            "modes": {"raw": "NCCL send/recv of the words",
+                      "compressed": "slice-pipelined compressed sub-streams over NCCL send/recv",
+                      "fused_p2p": "compress kernels store into rank 1's buffer over NVLink (CUDA IPC), "
+                                   "then rank 1 decompresses"},
             "jobs": out}
 
 

@@ -199,3 +199,101 @@ def recv_compressed(src: int, algo, device=None, codec=None, group=None, out: to
         k += 1
     codec.finish()
     return out, TransferStats(n_bytes, wire, k)
+
+
+# ---- fused compress + transfer over peer memory ----------------------------------
+
+class P2PChannel:
+    """Compression fused with the NVLink transfer (NEXT-3, the one-kernel form):
+    the receiver's stream buffer is mapped into the sender by CUDA IPC
+    (lcf_ipc_export / lcf_ipc_import), and the sender's lcf_compress writes the
+    stream straight into it — every chunk's TMA bulk store crosses NVLink as
+    soon as its decoupled look-back resolves, so the transfer overlaps the
+    compression chunk by chunk, and no copy or NCCL payload message follows.
+    The receiver decompresses from its own memory once a one-word signal
+    (stream-ordered after the compress on the sender) arrives.
+
+    Both ranks construct the channel (collectively) for arrays of up to
+    `max_bytes`; `send` / `recv` then move one array each; `close` unmaps. The
+    buffer is reused: a send waits for the receiver's release of the previous
+    stream (recv releases it once its decode is enqueued, unless asked not
+    to — then `release()`). Any
+    torch.distributed backend carries the handle and the signal (NCCL: CUDA
+    tensors; gloo: CPU tensors after a device synchronisation)."""
+
+    def __init__(self, src: int, dst: int, algo, max_bytes: int, group=None):
+        from . import lcf
+        self.lcf, self.src, self.dst, self.group = lcf, src, dst, group
+        self.a = _algo_id(algo)
+        self.cap = lcf.lcf_max_compressed_size(self.a, None, max_bytes)
+        self.rank = dist.get_rank(group)
+        self.gloo = dist.get_backend(group) == "gloo"
+        self.peer = None
+        self.sent = 0  # streams sent (sender): every one after the first waits for a release
+        dev = torch.device("cuda", torch.cuda.current_device())
+        self.dev = dev
+        msg = torch.zeros(72, dtype=torch.uint8)
+        if self.rank == dst:
+            self.buf = torch.empty(self.cap, dtype=torch.uint8, device=dev)
+            h, off = lcf.lcf_ipc_export(self.buf)
+            msg[:64] = torch.frombuffer(bytearray(h), dtype=torch.uint8)
+            msg[64:] = torch.tensor([off], dtype=torch.int64).view(torch.uint8)
+            dist.send(self._wire(msg), src, group=group)
+        elif self.rank == src:
+            m = self._wire(msg)
+            dist.recv(m, dst, group=group)
+            m = m.cpu()
+            self.peer = lcf.lcf_ipc_import(bytes(m[:64].numpy()), int(m[64:].view(torch.int64)[0]))
+
+    def _wire(self, t):
+        return t if self.gloo else t.to(self.dev)
+
+    def _signal(self, send: bool, value: int = 0, to=None, frm=None) -> int:
+        t = self._wire(torch.tensor([value], dtype=torch.int64))
+        if send:
+            if self.gloo:
+                torch.cuda.synchronize()  # the kernels before it (and their peer stores) are complete
+            dist.send(t, self.dst if to is None else to, group=self.group)  # NCCL: stream-ordered
+            return value
+        dist.recv(t, self.src if frm is None else frm, group=self.group)
+        return int(t.item())
+
+    def send(self, x: torch.Tensor) -> int:
+        """Compress x's words into the receiver's buffer; returns the stream
+        bytes (read back from the local call, synchronising)."""
+        words = x.reshape(-1).view(_word_dtype(self.a))
+        nb = words.numel() * words.element_size()
+        if self.sent:
+            self._signal(False, frm=self.dst)  # the receiver has released the buffer
+        n = self.lcf.lcf_compress(self.a, None, words, nb, self.peer, self.cap, sync=True)
+        self._signal(True, n)
+        self.sent += 1
+        return n
+
+    def recv(self, out: torch.Tensor, release: bool = True) -> int:
+        """Decompress the array the sender wrote into this rank's buffer into
+        `out` (its word view); returns the stream bytes."""
+        n = self._signal(False)
+        words = out.reshape(-1).view(_word_dtype(self.a))
+        self.lcf.lcf_decompress(self.a, None, self.buf, n, words, words.numel() * words.element_size(), sync=False)
+        if release:
+            self.release()
+        return n
+
+    def release(self) -> None:
+        """(receiver) the buffer may be overwritten by the next send."""
+        self._signal(True, 0, to=self.src)
+
+    def stream(self) -> torch.Tensor:
+        """(receiver) the stream bytes of the last transfer, for checks."""
+        return self.buf
+
+    def close(self) -> None:
+        """Both ranks: the sender takes the receiver's last release (each
+        recv's release is matched here or by the next send), then unmaps."""
+        if self.rank == self.src and self.sent:
+            self._signal(False, frm=self.dst)
+            self.sent = 0
+        if self.peer is not None:
+            self.lcf.lcf_ipc_close(self.peer)
+            self.peer = None

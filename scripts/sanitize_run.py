@@ -62,3 +62,26 @@ assert sharded.dp_simulate_shards(xd, 3) == full
 assert torch.equal(sharded.dp_simulate_decode_shards(full, 3), xd)
 print("DPratio shards ok")
 torch.cuda.synchronize()
+# round 2: FCM-active DPratio (deferred candidates + verify, pending words,
+# chain-node list walk/gather, the slow one-word match), and the multi-view
+# root resolution of simulated shards
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+from test_gpu_parity import fcm_stress_input  # noqa: E402
+rt = datagen.field("miranda_256x384x384_f64", "rt_density", shape=(2, 64, 384)).numpy().reshape(-1).view(np.uint64)
+base = np.random.default_rng(3).integers(0, 2**63, size=700, dtype=np.uint64)
+for name, w in (("rt_slab", rt.copy()), ("fcm_stress", fcm_stress_input(n_const=20000)[:200000].copy()),
+                ("period700", np.resize(base, 9 * 2048 + 5))):
+    xd = torch.from_numpy(w.view(np.int64)).cuda()
+    s = lcf.compress("DPratio", xd)
+    assert torch.equal(lcf.decompress("DPratio", s), xd), name
+    full = s.cpu().numpy().tobytes()
+    assert torch.equal(sharded.dp_simulate_decode_shards(full, 3), xd), name
+    t = s.clone()
+    t[60] ^= 0x3C
+    try:
+        lcf.lcf_decompress("DPratio", None, t, t.numel(), xd.clone(), xd.numel() * 8)
+        lcf.lcf_check_stream()
+    except lcf.LcfError:
+        pass
+    print(name, "DPratio chains ok")
+torch.cuda.synchronize()

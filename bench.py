@@ -123,7 +123,7 @@ def replica_bytes(cfg):
     return n * (4 if dtype == torch.float32 else 8)
 
 
-def make_fields(world, rank, device):
+def make_fields(world, rank, device, sets=None):
     """Per-field inputs. N = 1: the config's field. N > 1 (weak scaling): the
     global input is the concatenation of N independent replicas of the field;
     chunk-local codecs get this rank's chunk-range shard of it (generated from
@@ -131,7 +131,7 @@ def make_fields(world, rank, device):
     replica `rank` whole."""
     from paper_conf_asplos_azamifb25_b200 import datagen, sharded
     fields = []
-    for cfg, names, codecs in FIELD_SETS:
+    for cfg, names, codecs in (sets or FIELD_SETS):
         rb = replica_bytes(cfg)
         for nm in names:
             own = datagen.field(cfg, nm, device=device, replica=rank).reshape(-1)

@@ -5,7 +5,8 @@ config 5 and §8(e).
 The corpus (§8(d)):
   f32 ≈ 32 GiB: 24 NYX-like 512³ fields, 12 HACC-like 280,953,867-word arrays,
                 300 CESM-like 1800×3600 fields — SPspeed and SPratio on each;
-  f64 ≈ 32 GiB: 114 Miranda-like 256×384×384 fields — DPspeed and DPratio.
+  f64 ≈ 32 GiB: 114 Miranda-like 256×384×384 fields (density, velocity and
+                the FCM-active rt_density in turn) — DPspeed and DPratio.
 Every field is its own LCF1 stream, generated on whichever rank owns it from
 its field id (replica ≥ 1: independent of the bench's fields). `scale` keeps a
 proportional prefix of each category (at least one field each).
@@ -42,7 +43,7 @@ CATEGORIES = (
     ("nyx_512x512x512_f32", ("velocity", "baryon_density"), 24, SP_CODECS),
     ("hacc_280953867_f32", ("xx", "vx"), 12, SP_CODECS),
     ("cesm_1800x3600_f32", ("T", "U"), 300, SP_CODECS),
-    ("miranda_256x384x384_f64", ("density", "velocity"), 114, DP_CODECS),
+    ("miranda_256x384x384_f64", ("density", "velocity", "rt_density"), 114, DP_CODECS),
 )
 
 

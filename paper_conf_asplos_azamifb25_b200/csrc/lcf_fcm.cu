@@ -53,14 +53,12 @@ __device__ __forceinline__ uint64_t make_rec(uint64_t xi, uint32_t hw, uint64_t 
   return (h << kRecHashShift) | ((uint64_t)fp << kRecFpShift) | i;
 }
 
-// Lanes of the warp holding the same digit as this lane (valid lanes only):
-// ten ballots, one per digit bit — ALU-pipe votes instead of __match_any_sync,
-// whose long MIO latency serialised the ranking loop.
-__device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
+// Lanes whose winner id (5 bits) equals this lane's (valid lanes only).
+__device__ __forceinline__ uint32_t winner_peers(uint32_t win, bool valid) {
   uint32_t peers = __ballot_sync(0xFFFFFFFFu, valid);
 #pragma unroll
-  for (int b = 0; b < kDigitBits; ++b) {
-    const bool bit = (d >> b) & 1;
+  for (int b = 0; b < 5; ++b) {
+    const bool bit = (win >> b) & 1;
     const uint32_t bb = __ballot_sync(0xFFFFFFFFu, bit);
     peers &= bit ? bb : ~bb;
   }
@@ -341,8 +339,13 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       // read another lane id back); only then are the peers matched exactly
       if (ok[k]) S.tag[warp][d] = (uint8_t)lane;
       __syncwarp();
-      const bool clash = __any_sync(0xFFFFFFFFu, ok[k] && S.tag[warp][d] != lane);
-      const uint32_t peers = clash ? digit_peers(d, ok[k]) : (1u << lane);
+      // every lane of a digit reads back the same winning lane id, and lanes of
+      // different digits read different ids (a lane has one digit): the peers
+      // are the lanes with my winner — five ballots on its bits instead of ten
+      // on the digit's
+      const uint32_t win = S.tag[warp][d];
+      const bool clash = __any_sync(0xFFFFFFFFu, ok[k] && win != lane);
+      const uint32_t peers = clash ? winner_peers(win, ok[k]) : (1u << lane);
       uint32_t* wc = &S.wcnt[warp][d >> 1];
       const uint32_t sh = 16 * (d & 1);
       const uint32_t rbase = ok[k] ? (*wc >> sh) & 0xFFFFu : 0u;

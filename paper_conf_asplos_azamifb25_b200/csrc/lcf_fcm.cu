@@ -222,13 +222,27 @@ constexpr int kOwners = kDigits / 2 / kP;
 static_assert(kP * 2 * kOwners == kDigits && kOwners <= kST, "digit pairs divide over the threads");
 constexpr int kRounds = kTile / kRound;
 static_assert(kRounds * kRound == kTile, "tile = whole rounds");
+// LCF_SCAT_U32: one u32 count per (warp, digit) instead of packed u16 pairs —
+// then lanes of distinct digits never share a word, and the rank update is a
+// plain store by each digit's leader instead of a shared atomic
+#ifndef LCF_SCAT_U32
+#define LCF_SCAT_U32 1
+#endif
 struct ScatterSmem {
   uint64_t stage[kRound];
+#if LCF_SCAT_U32
+  uint32_t wcnt[kSW][kDigits];      // count, then the warp's next stage slot, per digit
+#else
   uint32_t wcnt[kSW][kDigits / 2];  // packed u16 pair per word
+#endif
   uint32_t run[kDigits];                   // next output position of each digit (tile-wide)
   uint32_t rstart[kDigits];                // round: first stage slot of each digit
   uint32_t delta[kDigits];                 // round: output position − stage slot of each digit
+#if LCF_SCAT_U32
+  uint32_t rtot[kDigits];                  // round: digit totals
+#else
   uint32_t rtot[kDigits / 2];              // round: packed digit totals
+#endif
   uint32_t wsum[kSW];
   uint8_t tag[kSW][kDigits];        // per warp: last lane that claimed a digit
 };
@@ -290,7 +304,11 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
     }
     // 1. this warp's records of the round and its digit counts
 #pragma unroll
+#if LCF_SCAT_U32
+    for (int j = lane; j < kDigits; j += 32) S.wcnt[warp][j] = 0;
+#else
     for (int j = lane; j < kDigits / 2; j += 32) S.wcnt[warp][j] = 0;
+#endif
     __syncwarp();
     uint64_t rec[kSB];
     uint32_t dg[kSB];
@@ -299,10 +317,43 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
     for (int k = 0; k < kSB; ++k) {
       rec[k] = rd.rec(k, lane, ok[k]);
       dg[k] = ok[k] ? rec_digit(rec[k], PASS) : 0u;
+#if LCF_SCAT_U32
+      if (ok[k]) atomicAdd(&S.wcnt[warp][dg[k]], 1u);
+#else
       if (ok[k]) atomicAdd(&S.wcnt[warp][dg[k] >> 1], 1u << (16 * (dg[k] & 1)));
+#endif
     }
     __syncthreads();
     // 2. this thread's digit pairs: prefix over the warps (packed: sums ≤ kRound per half)
+#if LCF_SCAT_U32
+    {
+      uint32_t c[2 * kP], ex[2 * kP];
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) {
+        const uint32_t dj = 2 * kP * tid + j;
+        uint32_t tw = 0;
+        if (owner) {
+#pragma unroll
+          for (int w = 0; w < kSW; ++w) {
+            const uint32_t v = S.wcnt[w][dj];
+            S.wcnt[w][dj] = tw;
+            tw += v;
+          }
+        }
+        c[j] = tw;
+      }
+      digit_scan(c, ex);
+      if (owner)
+#pragma unroll
+        for (int j = 0; j < 2 * kP; ++j) {
+          const uint32_t dj = 2 * kP * tid + j;
+#pragma unroll
+          for (int w = 0; w < kSW; ++w) S.wcnt[w][dj] += ex[j];  // absolute stage slots
+          S.delta[dj] = S.run[dj] - ex[j];
+          S.rtot[dj] = c[j];
+        }
+    }
+#else
     {
       uint32_t c[2 * kP], ex[2 * kP];
 #pragma unroll
@@ -329,6 +380,7 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
           S.delta[2 * kP * tid + j] = S.run[2 * kP * tid + j] - ex[j];
         }
     }
+#endif
     __syncthreads();
     // 3. ranks → stage
 #pragma unroll
@@ -346,6 +398,15 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       const uint32_t win = S.tag[warp][d];
       const bool clash = __any_sync(0xFFFFFFFFu, ok[k] && win != lane);
       const uint32_t peers = clash ? winner_peers(win, ok[k]) : (1u << lane);
+#if LCF_SCAT_U32
+      uint32_t* wc = &S.wcnt[warp][d];
+      const uint32_t slot = ok[k] ? *wc : 0u;  // this warp's next stage slot of digit d
+      __syncwarp();
+      if (ok[k]) {
+        S.stage[slot + __popc(peers & lt)] = rec[k];
+        if (lane == (uint32_t)__ffs(peers) - 1) *wc = slot + __popc(peers);  // one writer per digit
+      }
+#else
       uint32_t* wc = &S.wcnt[warp][d >> 1];
       const uint32_t sh = 16 * (d & 1);
       const uint32_t rbase = ok[k] ? (*wc >> sh) & 0xFFFFu : 0u;
@@ -354,6 +415,7 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
         S.stage[S.rstart[d] + rbase + __popc(peers & lt)] = rec[k];
         if (lane == (uint32_t)__ffs(peers) - 1) atomicAdd(wc, (uint32_t)__popc(peers) << sh);
       }
+#endif
       __syncwarp();
     }
     if (LCF_SCAT_PREFETCH && r + 1 < kRounds) {
@@ -367,13 +429,19 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
       dst[S.delta[rec_digit(v, PASS)] + j] = v;
     }
     __syncthreads();
-    if (owner)
+    if (owner) {
+#if LCF_SCAT_U32
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) S.run[2 * kP * tid + j] += S.rtot[2 * kP * tid + j];
+#else
 #pragma unroll
       for (int q = 0; q < kP; ++q) {
         const uint32_t pq = kP * tid + q, t2 = S.rtot[pq];
         S.run[2 * pq] += t2 & 0xFFFFu;
         S.run[2 * pq + 1] += t2 >> 16;
       }
+#endif
+    }
     // (the next round's first barrier orders these updates before step 4)
   }
 }

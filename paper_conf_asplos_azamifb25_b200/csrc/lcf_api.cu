@@ -313,7 +313,7 @@ static lcf_status_t dpratio_decode_range(Workspace* ws, DecArgs a, const LaunchC
   v.v[0] = DpView{0, words, reinterpret_cast<uint64_t*>(a.out), ws->pend, ws->tgt};
   const uint64_t lo = a.first_tile * 2048, hi = end_tile && end_tile * 2048 < words ? end_tile * 2048 : words;
   launch_dp_nodes(v.v[0], a.nodes, cnt, words, ctx, ws->any_pend, false, stream);  // chain nodes → roots
-  launch_dp_gather_roots(v, a.stream, lo, hi, ctx, ws->any_pend, stream, 0);       // leaves, via their chain node
+  launch_dp_gather_leaves(v.v[0], a.stream, lo, hi, ctx, ws->any_pend, stream);    // leaves, via their chain node
   launch_dp_nodes(v.v[0], a.nodes, cnt, words, ctx, ws->any_pend, true, stream);   // chain nodes
   g_launches += 3;
   // both bitmaps of the range back to zero (the next launch writes its tiles' words)

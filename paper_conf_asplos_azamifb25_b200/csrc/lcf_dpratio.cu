@@ -1246,26 +1246,57 @@ __global__ void __launch_bounds__(256) dp_gather_roots_kernel(const __grid_const
 // (a few percent of the pending words on repeat-heavy data) instead of
 // scanning every bitmap word, in list order (≈ index order: tiles append as
 // they are decoded), writing back every hop.
+#ifndef LCF_WALK_U
+#define LCF_WALK_U 2
+#endif
+constexpr int kWalkU = LCF_WALK_U;  // list entries walked together per thread (their hops overlap)
 __global__ void __launch_bounds__(256) dp_walk_nodes_kernel(DpView me, const uint32_t* __restrict__ nodes,
                                                            const uint32_t* __restrict__ n_nodes, uint64_t cap,
                                                            LaunchCtx ctx, const uint32_t* any_pend) {
   if (any_pend && *any_pend != ctx.epoch) return;
   const uint64_t cnt = umin64(*n_nodes, cap);
-  for (uint64_t k = blockIdx.x * 256ull + threadIdx.x; k < cnt; k += (uint64_t)gridDim.x * 256) {
-    const uint64_t c = nodes[k];
-    if (c >= me.n || !((__ldcg(me.pend + c / 32) >> (c % 32)) & 1)) continue;  // a final word
-    uint64_t cur = c, t = __ldcg(me.out + c);
-    bool err = false;
-    for (;;) {
-      if (t >= cur) { err = true; break; }
-      const uint32_t pw = __ldcg(me.pend + t / 32);
-      const uint64_t nt = ld_relaxed_u64(me.out + t);
-      if (!((pw >> (t % 32)) & 1)) break;  // the root
-      cur = t;
-      t = nt;
-      st_relaxed_u64(me.out + c, t);
+  const uint64_t stride = (uint64_t)gridDim.x * 256;
+  for (uint64_t k0 = blockIdx.x * 256ull + threadIdx.x; k0 < cnt; k0 += stride * kWalkU) {
+    uint64_t c[kWalkU], cur[kWalkU], t[kWalkU];
+    bool on[kWalkU];
+#pragma unroll
+    for (int u = 0; u < kWalkU; ++u) {
+      const uint64_t k = k0 + stride * u;
+      c[u] = k < cnt ? nodes[k] : ~0ull;
+      on[u] = c[u] < me.n && ((__ldcg(me.pend + c[u] / 32) >> (c[u] % 32)) & 1);  // (a final word: nothing)
+      cur[u] = c[u];
+      t[u] = on[u] ? __ldcg(me.out + c[u]) : 0ull;
     }
-    if (err) record_error(ctx, DERR_CORRUPT);
+    bool any = false;
+#pragma unroll
+    for (int u = 0; u < kWalkU; ++u) any |= on[u];
+    while (any) {
+      uint32_t pw[kWalkU];
+      uint64_t nt[kWalkU];
+#pragma unroll
+      for (int u = 0; u < kWalkU; ++u) {
+        if (on[u] && t[u] >= cur[u]) {  // chains point strictly backwards
+          record_error(ctx, DERR_CORRUPT);
+          on[u] = false;
+        }
+        // the bit and the word are fetched together (one round trip per hop)
+        pw[u] = on[u] ? __ldcg(me.pend + t[u] / 32) : 0u;
+        nt[u] = on[u] ? ld_relaxed_u64(me.out + t[u]) : 0ull;
+      }
+      any = false;
+#pragma unroll
+      for (int u = 0; u < kWalkU; ++u) {
+        if (!on[u]) continue;
+        if (!((pw[u] >> (t[u] % 32)) & 1)) {  // t is final: the root (already stored)
+          on[u] = false;
+          continue;
+        }
+        cur[u] = t[u];
+        t[u] = nt[u];
+        st_relaxed_u64(me.out + c[u], t[u]);  // every hop is written back (concurrent pointer doubling)
+        any = true;
+      }
+    }
   }
 }
 
@@ -1280,6 +1311,68 @@ __global__ void __launch_bounds__(256) dp_gather_nodes_kernel(DpView me, const u
     const uint64_t r = __ldcg(me.out + c);
     if (r >= c) record_error(ctx, DERR_CORRUPT);
     else me.out[c] = __ldcg(me.out + r);
+  }
+}
+
+// The leaves of a single-view decode (pending words that are not chain
+// nodes), after the chain nodes' walk: each takes its value through its chain
+// node (or straight from a final target). A warp takes kLeafU bitmap words at
+// a time so that the five dependent loads of every leaf overlap with those of
+// the others (the pass is latency-bound on L2 round trips).
+#ifndef LCF_LEAF_U
+#define LCF_LEAF_U 4
+#endif
+constexpr int kLeafU = LCF_LEAF_U;
+__global__ void __launch_bounds__(256) dp_gather_leaves_kernel(DpView me, const uint8_t* stream, uint64_t w_lo,
+                                                              uint64_t w_hi, LaunchCtx ctx, const uint32_t* any_pend) {
+  if (any_pend && *any_pend != ctx.epoch) return;
+  uint64_t hi = w_hi < me.n ? w_hi : me.n;
+  if (stream) {
+    const uint64_t nw = reinterpret_cast<const uint64_t*>(stream)[1] / 8;
+    hi = hi < nw ? hi : nw;
+  }
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t wg = (blockIdx.x * 256ull + threadIdx.x) >> 5, nwarps = gridDim.x * 8ull;
+  for (uint64_t base = w_lo + wg * 32 * kLeafU; base < hi; base += nwarps * 32 * kLeafU) {
+    uint32_t bits[kLeafU];
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u) {
+      const uint64_t b = base + 32 * u;
+      bits[u] = b < hi ? __ldcg(me.pend + b / 32) & ~__ldcg(me.tgt + b / 32) : 0u;
+    }
+    uint64_t r[kLeafU];
+    bool act[kLeafU];
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u) {
+      const uint64_t li = base + 32 * u + lane;
+      act[u] = ((bits[u] >> lane) & 1) && li < hi;
+      r[u] = act[u] ? __ldcg(me.out + li) : 0ull;
+    }
+    uint32_t pr[kLeafU];
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u) {
+      const uint64_t li = base + 32 * u + lane;
+      if (act[u] && r[u] >= li) {  // chains point backwards
+        record_error(ctx, DERR_CORRUPT);
+        act[u] = false;
+      }
+      pr[u] = act[u] ? __ldcg(me.pend + r[u] / 32) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u)
+      if (act[u] && ((pr[u] >> (r[u] % 32)) & 1)) r[u] = __ldcg(me.out + r[u]);  // the chain node's root
+    uint64_t v[kLeafU];
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u) {
+      if (act[u] && r[u] >= me.n) {
+        record_error(ctx, DERR_CORRUPT);
+        act[u] = false;
+      }
+      v[u] = act[u] ? __ldcg(me.out + r[u]) : 0ull;
+    }
+#pragma unroll
+    for (int u = 0; u < kLeafU; ++u)
+      if (act[u]) me.out[base + 32 * u + lane] = v[u];
   }
 }
 
@@ -1300,6 +1393,14 @@ void launch_dp_find_roots(const DpViews& v, const uint8_t* stream, uint64_t w_lo
   else
     dp_find_roots_kernel<false><<<roots_grid((const void*)dp_find_roots_kernel<false>, w_hi - w_lo), 256, 0, st>>>(
         v, stream, w_lo, w_hi, ctx, any_pend, mode);
+}
+
+void launch_dp_gather_leaves(const DpView& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                             const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st) {
+  if (w_hi <= w_lo) return;
+  KTrace kt("dp_gather_leaves", st);
+  dp_gather_leaves_kernel<<<roots_grid((const void*)dp_gather_leaves_kernel, (w_hi - w_lo) / kLeafU), 256, 0, st>>>(
+      v, stream, w_lo, w_hi, ctx, any_pend);
 }
 
 void launch_dp_nodes(const DpView& v, const uint32_t* nodes, const uint32_t* n_nodes, uint64_t cap,

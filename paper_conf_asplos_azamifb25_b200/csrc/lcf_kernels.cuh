@@ -218,6 +218,8 @@ void launch_dp_gather_roots(const DpViews& v, const uint8_t* stream, uint64_t w_
 // indices): walk the chain nodes to their roots (gather = false), or give them
 // their roots' values (gather = true; after the leaves' gather). `cap` bounds
 // the list (max_words).
+void launch_dp_gather_leaves(const DpView& v, const uint8_t* stream, uint64_t w_lo, uint64_t w_hi,
+                             const LaunchCtx& ctx, const uint32_t* any_pend, cudaStream_t st);
 void launch_dp_nodes(const DpView& v, const uint32_t* nodes, const uint32_t* n_nodes, uint64_t cap,
                      const LaunchCtx& ctx, const uint32_t* any_pend, bool gather, cudaStream_t st);
 

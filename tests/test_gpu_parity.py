@@ -418,8 +418,9 @@ def test_host_pipelined_slices(L, orc, algo, monkeypatch):
 @pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_transfer_gpu_slices(L, orc, algo):
     """NEXT-3 slice coder on the B200: the sub-streams send_compressed puts on
-    the wire equal the CPU codec's, and decoding them slice by slice (the
-    receiver's path, loopback without a second GPU) restores the array."""
+    the wire equal the oracle's streams of the same slices (and the CPU
+    codec's), and decoding them slice by slice (the receiver's path, loopback
+    without a second GPU) restores the array."""
     from paper_conf_asplos_azamifb25_b200 import transfer
     dt = np.float32 if algo.startswith("SP") else np.float64
     words = datagen.smooth_1d(20 * 16384 // np.dtype(dt).itemsize + 77, dt, seed=33).view(wdt(algo)).copy()
@@ -429,10 +430,11 @@ def test_transfer_gpu_slices(L, orc, algo):
     ref = transfer.substreams(torch.from_numpy(words.view(np.int32 if dt == np.float32 else np.int64)), algo,
                               codec=transfer.CpuCodec(), slice_bytes=3 * 16384)
     assert [s.cpu().numpy().tobytes() for s in subs] == [r.numpy().tobytes() for r in ref]
-    out = torch.empty_like(x)
-    codec = transfer.GpuCodec()
     wb = words.itemsize
     bounds = list(transfer._slices(words.nbytes, wb, 3 * 16384 if algo != "DPratio" else transfer._whole(words.nbytes)))
+    assert [s.cpu().numpy().tobytes() for s in subs] == [orc.compress(algo, words[w0:w1]) for w0, w1 in bounds]
+    out = torch.empty_like(x)
+    codec = transfer.GpuCodec()
     assert len(bounds) == len(subs)
     for (w0, w1), s in zip(bounds, subs):
         codec.decompress_into(transfer._algo_id(algo), s, out[w0:w1])

@@ -25,7 +25,8 @@ namespace {
 constexpr int kRW = 4;                  // compute warps
 constexpr uint32_t kRT = kRW * 32;      // compute threads: one 32-word group each
 #ifndef LCF_SPR_STAGES
-#define LCF_SPR_STAGES 2
+#define LCF_SPR_STAGES 1  // 1 in-place stage + ≤ 56 registers: 6 CTAs/SM (NYX velocity 452 → 431 µs,
+                          // HACC xx 890 → 846 µs); 2 stages at 80 registers: 4 CTAs/SM
 #endif
 // encode: kRStages input stages, each also the chunk's output buffer (in place)
 #ifndef LCF_SPR_DSTAGES
@@ -331,7 +332,10 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
   }
 }
 
-__global__ void __launch_bounds__(kREncThreads, 4) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+#ifndef LCF_SPR_ENC_MINB
+#define LCF_SPR_ENC_MINB 6
+#endif
+__global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

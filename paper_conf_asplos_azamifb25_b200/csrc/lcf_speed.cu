@@ -30,12 +30,18 @@ constexpr int kCompWarps = 8, kSubPerWarp = 4;
 // Encoder buffering (measured on B200, NYX / Miranda / CESM): the input stage
 // is released as soon as the compute warps hold the chunk in registers, so one
 // input stage suffices, and a third output slot absorbs the storer's look-back
-// waits (2→1 input stages, 2→3 output slots: −4…8 % compress time).
+// waits (2→1 input stages, 2→3 output slots: −4…8 % compress time). Round 2:
+// 2 output slots with a 48-register bound fit 4 CTAs/SM (3 slots at 62
+// registers: 3 CTAs/SM): NYX velocity 229 → 225 µs, HACC xx 426 → 421 µs,
+// Miranda density 130 → 129 µs, CESM T 23.3 → 24.6 µs.
 #ifndef LCF_ENC_STAGES
 #define LCF_ENC_STAGES 1
 #endif
 #ifndef LCF_ENC_OUT
-#define LCF_ENC_OUT 3
+#define LCF_ENC_OUT 2
+#endif
+#ifndef LCF_ENC_MINB
+#define LCF_ENC_MINB 4
 #endif
 #ifndef LCF_ENC_STORERS
 #define LCF_ENC_STORERS 1

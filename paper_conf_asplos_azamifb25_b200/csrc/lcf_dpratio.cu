@@ -92,10 +92,24 @@ __device__ __forceinline__ void load8(const uint64_t* sv, uint32_t n, uint32_t t
 }
 
 // LSB-first bit writer for one thread's contiguous run of fields in a u32
-// buffer. The run's first and last words may be shared with the neighbouring
-// runs (atomicOr into a zeroed buffer); the words in between belong to this
-// thread alone (plain stores). The pending partial word is 32 bits wide: a
-// field of up to 64 bits completes at most two words, formed by funnel shifts.
+// shared-memory buffer. The run's first and last words may be shared with the
+// neighbouring runs (OR-ed into a zeroed buffer); the words in between belong
+// to this thread alone (plain stores). The pending partial word is 32 bits
+// wide: a field of up to 64 bits completes at most two words, formed by funnel
+// shifts. LCF_BW_PRED: put() is branch-free — both possible word writes are
+// predicated shared stores / reductions, so lanes at different bit offsets do
+// not diverge, and a field of width 0 is a no-op (callers pass w = 0 instead
+// of skipping the call).
+#ifndef LCF_BW_PRED
+#define LCF_BW_PRED 1
+#endif
+__device__ __forceinline__ void sts_or_pred(uint32_t addr, uint32_t v, bool st, bool red) {
+  asm volatile(
+      "{\n .reg .pred ps, pr;\n setp.ne.u32 ps, %2, 0;\n setp.ne.u32 pr, %3, 0;\n"
+      " @ps st.shared.u32 [%0], %1;\n @pr red.shared.or.b32 [%0], %1;\n}" ::"r"(addr),
+      "r"(v), "r"((uint32_t)st), "r"((uint32_t)red)
+      : "memory");
+}
 struct BitWriter {
   uint32_t* buf;
   uint32_t widx, w0, nb, pw;  // current word, first word, pending bits (< 32), pending word
@@ -106,13 +120,21 @@ struct BitWriter {
     else buf[widx] = w;
     ++widx;
   }
-  // append the low w bits of f (f < 2^w, 1 ≤ w ≤ 64)
+  // append the low w bits of f (f < 2^w, 0 ≤ w ≤ 64; w = 0 needs f = 0)
   __device__ __forceinline__ void put(uint64_t f, uint32_t w) {
     const uint32_t flo = (uint32_t)f, fhi = (uint32_t)(f >> 32);
     const uint32_t o0 = pw | (flo << nb);              // bits 0..31 of pw | f << nb
     const uint32_t o1 = __funnelshift_l(flo, fhi, nb);  // bits 32..63
     const uint32_t o2 = __funnelshift_l(fhi, 0u, nb);   // bits 64..95
     const uint32_t e = nb + w;
+#if LCF_BW_PRED
+    const bool c0 = e >= 32, c1 = e >= 64, first = widx == w0;
+    const uint32_t a = smem_addr(buf + widx);
+    sts_or_pred(a, o0, c0 && !first, c0 && first);
+    sts_or_pred(a + 4, o1, c1, false);
+    widx += (uint32_t)c0 + (uint32_t)c1;
+    pw = c1 ? o2 : (c0 ? o1 : o0);
+#else
     if (e >= 32) {
       out(o0);
       if (e >= 64) {
@@ -124,6 +146,7 @@ struct BitWriter {
     } else {
       pw = o0;
     }
+#endif
     nb = e & 31;
   }
   __device__ __forceinline__ void finish() {
@@ -267,16 +290,22 @@ __device__ __forceinline__ void a_emit(const uint64_t (&v)[8], const APlan& P, u
   if (P.byte) {
     BitWriter bw(dw, 24 + (uint64_t)P.rank0 * k);
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-      if ((P.byte >> j) & 1) bw.put(v[j] >> sh, k);
+    for (int j = 0; j < 8; ++j) {
+      const bool on = (P.byte >> j) & 1;
+      if (LCF_BW_PRED) bw.put(on ? v[j] >> sh : 0ull, on ? k : 0u);
+      else if (on) bw.put(v[j] >> sh, k);
+    }
     bw.finish();
   }
   if (wl && i0 < n) {
     const uint64_t lmask = (1ull << wl) - 1;  // wl ≤ 63
     BitWriter bw(dw, 8ull * (3 + P.hib) + (uint64_t)i0 * wl);
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-      if (i0 + j < n) bw.put(v[j] & lmask, wl);
+    for (int j = 0; j < 8; ++j) {
+      const bool on = i0 + j < n;
+      if (LCF_BW_PRED) bw.put(on ? v[j] & lmask : 0ull, on ? wl : 0u);
+      else if (on) bw.put(v[j] & lmask, wl);
+    }
     bw.finish();
   }
   auto put_byte = [&](uint32_t pos, uint32_t val) { atomicOr(dw + (pos >> 2), (val & 0xFFu) << (8 * (pos & 3))); };
@@ -304,8 +333,11 @@ __device__ __forceinline__ void a_emit_bypass_regs(const uint64_t (&v)[8], uint3
   if (i0 < n) {
     BitWriter bw(dw, 24 + 64ull * i0);
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-      if (i0 + j < n) bw.put(v[j], 64);
+    for (int j = 0; j < 8; ++j) {
+      const bool on = i0 + j < n;
+      if (LCF_BW_PRED) bw.put(on ? v[j] : 0ull, on ? 64u : 0u);
+      else if (on) bw.put(v[j], 64);
+    }
     bw.finish();
   }
 }
@@ -578,9 +610,19 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
       const uint32_t* gd = a.fcm_dist + t * kTileWords;  // (the stage is gone: distances from L2)
       if (part == 1) {  // DIFFMS₆₄ of the distances
         uint64_t pd = dprev;
+        uint32_t dv[8];
+        if (i0 + 8 <= m) {  // two 16-byte loads per thread (the tile's distances are 16-byte aligned)
+          const uint4 q0 = __ldcg(reinterpret_cast<const uint4*>(gd + i0));
+          const uint4 q1 = __ldcg(reinterpret_cast<const uint4*>(gd + i0) + 1);
+          dv[0] = q0.x; dv[1] = q0.y; dv[2] = q0.z; dv[3] = q0.w;
+          dv[4] = q1.x; dv[5] = q1.y; dv[6] = q1.z; dv[7] = q1.w;
+        } else {
+#pragma unroll
+          for (int j = 0; j < 8; ++j) dv[j] = i0 + j < m ? __ldcg(gd + i0 + j) : 0u;
+        }
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          const uint64_t dj = i0 + j < m ? (uint64_t)__ldcg(gd + i0 + j) : 0ull;
+          const uint64_t dj = dv[j];
           w[j] = tcms(dj - pd);
           pd = dj;
         }

@@ -182,9 +182,10 @@ def kernel_bytes(j):
         return {"spratio_encode": io, "spratio_decode": io}
     tiles = -(-words // 16384)
     # the sort kernels launch once per radix pass (two passes per job)
-    return {"fcm_sort_hist": 2 * 8 * words,           # x (pass 1) or pass-1 records (pass 2) in
-            "fcm_sort_scan": 2 * 8 * 1024 * tiles,    # the tile × digit count matrix, read and rewritten
-            "fcm_sort_scatter": 2 * 16 * words,       # 8-byte records (or x) in, records out
+    return {"fcm_sort_ghist": 8 * words,              # x in (both passes' digit totals in one read)
+            "fcm_sort_hist": 2 * 8 * words,           # (LCF_ONESWEEP=0 build) x or pass-1 records in
+            "fcm_sort_scan": 2 * 8 * 1024 * tiles,    # (LCF_ONESWEEP=0 build) the tile × digit count matrix
+            "fcm_sort_scatter": 2 * 16 * words,       # 8-byte records (or x) in, records out, per pass
             "fcm_match": 8 * words,                   # sorted records in (candidates scattered)
             "fcm_verify": 4 * words,                  # the candidate array in (x read only at candidates)
             "dp_walk_nodes": 0,                       # (data-dependent: the chain-node list)

@@ -446,6 +446,246 @@ __global__ void __launch_bounds__(kST, LCF_SCAT_MINB) sort_scatter_kernel(const 
   }
 }
 
+// ---- onesweep sort (LCF_ONESWEEP) ----------------------------------------------
+// The global digit totals of BOTH passes come from one read of x
+// (sort_ghist); each pass is then one kernel (sort_onesweep): persistent CTAs
+// take tiles of kRound records by ticket, count the tile's digits, publish the
+// counts, and find the tile's offset inside every digit run by a decoupled
+// look-back over the earlier tiles' status words — no per-tile count matrix,
+// no column scan, and no second histogram pass over the pass-0 records.
+// Status word of (tile, digit): 0 = not yet published, else (value + 1) with
+// bit 31 set once value is the inclusive prefix over tiles 0..t (else value is
+// the tile's own count). n < 2^31 keeps value + 1 below bit 31.
+// Measured slower than the hist/scan/scatter passes and kept for A/B builds
+// only: 94 µs + 2 × 350 µs against 2 × (71 + 15 + 284) µs on
+// Miranda; without the look-back (wrong offsets, a timing bound) 2 × 277 µs —
+// the 148 lock-stepped tiles of a wave resolve their inclusive prefixes in a
+// cascade, ≈ 2.3 µs per 8 Ki-record tile.
+#ifndef LCF_ONESWEEP
+#define LCF_ONESWEEP 0
+#endif
+#ifndef LCF_SWEEP_LB
+#define LCF_SWEEP_LB 32  // status words read per round trip of a look-back walk
+#endif
+constexpr uint32_t kIncl = 0x80000000u;
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// tot2[0][d], tot2[1][d]: how many records have digit d in pass 0 / pass 1
+// (tot2 pre-zeroed). Warps take kWarpRecs-record ranges grid-stride.
+__global__ void __launch_bounds__(kSortThreads) sort_ghist_kernel(const uint64_t* __restrict__ x, uint64_t n,
+                                                                  uint32_t* __restrict__ tot2, uint32_t halo) {
+  __shared__ uint32_t hist[2][kDigits];
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (uint32_t d = threadIdx.x; d < 2 * kDigits; d += kSortThreads) (&hist[0][0])[d] = 0;
+  __syncthreads();
+  const uint64_t ranges = (n + kWarpRecs - 1) / kWarpRecs;
+  for (uint64_t g = (uint64_t)blockIdx.x * kSortWarps + warp; g < ranges; g += (uint64_t)gridDim.x * kSortWarps) {
+    RecReader<0> rd(x, n, g * kWarpRecs, lane, halo);
+    for (int s = 0; s < kWarpRecs / (32 * kBatch); ++s, rd.advance()) {
+      if (rd.i0 >= n) break;  // warp-uniform
+      rd.load(lane);
+#pragma unroll
+      for (int k = 0; k < kBatch; ++k) {
+        bool valid;
+        const uint64_t rec = rd.rec(k, lane, valid);
+        if (valid) {
+          atomicAdd(&hist[0][rec_digit(rec, 0)], 1u);
+          atomicAdd(&hist[1][rec_digit(rec, 1)], 1u);
+        }
+      }
+    }
+  }
+  __syncthreads();
+  for (uint32_t d = threadIdx.x; d < 2 * kDigits; d += kSortThreads) {
+    const uint32_t c = (&hist[0][0])[d];
+    if (c) atomicAdd(tot2 + d, c);
+  }
+}
+
+struct OnesweepSmem {
+  uint64_t stage[kRound];
+  uint32_t wcnt[kSW][kDigits];  // count, then the warp's next stage slot, per digit
+  uint32_t gbase[kDigits];      // first output position of each digit (exclusive scan of the totals)
+  uint32_t delta[kDigits];      // tile: output position − stage slot of each digit
+  uint32_t wsum[kSW];
+  uint32_t tile[2];             // tickets (current, next)
+  uint8_t tag[kSW][kDigits];    // per warp: last lane that claimed a digit
+};
+
+// One LSD pass: records src[0, n) → dst, stable by digit PASS. tot: this
+// pass's global digit totals; status: ceil(n / kRound) × kDigits words, zeroed;
+// ticket: zeroed. Tiles are taken in ticket order and a tile only waits on
+// earlier tiles, whose holders are running: no deadlock.
+template <int PASS>
+__global__ void __launch_bounds__(kST, 1) sort_onesweep_kernel(const uint64_t* __restrict__ src, uint64_t n,
+                                                               const uint32_t* __restrict__ tot,
+                                                               uint32_t* __restrict__ status,
+                                                               uint32_t* __restrict__ ticket,
+                                                               uint64_t* __restrict__ dst, uint32_t halo) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  OnesweepSmem& S = *reinterpret_cast<OnesweepSmem*>(smem_raw);
+  const uint32_t tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint32_t lt = (1u << lane) - 1u;
+  const bool owner = tid < (uint32_t)kOwners;  // thread owns digits [2kP·tid, 2kP·tid + 2kP)
+  auto digit_scan = [&](const uint32_t (&c)[2 * kP], uint32_t (&ex)[2 * kP]) {
+    uint32_t own = 0;
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) own += c[j];
+    uint32_t x = own;
+#pragma unroll
+    for (int k = 1; k < 32; k <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, k);
+      if ((int)lane >= k) x += y;
+    }
+    if (lane == 31) S.wsum[warp] = x;
+    __syncthreads();
+    uint32_t base = x - own;
+    for (uint32_t w = 0; w < warp; ++w) base += S.wsum[w];
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) {
+      ex[j] = base;
+      base += c[j];
+    }
+  };
+  {  // digit bases
+    uint32_t c[2 * kP], ex[2 * kP];
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) c[j] = owner ? tot[2 * kP * tid + j] : 0u;
+    digit_scan(c, ex);
+    if (owner)
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) S.gbase[2 * kP * tid + j] = ex[j];
+  }
+  const uint32_t nT = (uint32_t)((n + kRound - 1) / kRound);
+  if (tid == 0) S.tile[0] = atomicAdd(ticket, 1u);
+  __syncthreads();  // (also orders wsum reuse)
+  uint32_t t = S.tile[0];
+  RecReader<PASS, kSB> rd(src, n, (uint64_t)t * kRound + warp * 32 * kSB, lane, halo);
+  if (t < nT) rd.load(lane);
+  for (uint32_t it = 0; t < nT; ++it) {
+    const uint64_t r0 = (uint64_t)t * kRound;
+    const uint32_t nr = (uint32_t)umin64(kRound, n - r0);
+    // 1. this warp's records of the tile and its digit counts
+    for (int j = lane; j < kDigits; j += 32) S.wcnt[warp][j] = 0;
+    __syncwarp();
+    uint64_t rec[kSB];
+    uint32_t dg[kSB];
+    bool ok[kSB];
+#pragma unroll
+    for (int k = 0; k < kSB; ++k) {
+      rec[k] = rd.rec(k, lane, ok[k]);
+      dg[k] = ok[k] ? rec_digit(rec[k], PASS) : 0u;
+      if (ok[k]) atomicAdd(&S.wcnt[warp][dg[k]], 1u);
+    }
+    __syncthreads();
+    // 2. per digit: prefix over the warps and the tile's count, published at
+    // once (successors add it up in their look-back), then the stage slots
+    uint32_t c[2 * kP], ex[2 * kP];
+#pragma unroll
+    for (int j = 0; j < 2 * kP; ++j) {
+      const uint32_t dj = 2 * kP * tid + j;
+      uint32_t tw = 0;
+      if (owner) {
+#pragma unroll
+        for (int w = 0; w < kSW; ++w) {
+          const uint32_t v = S.wcnt[w][dj];
+          S.wcnt[w][dj] = tw;
+          tw += v;
+        }
+        st_relaxed_u32(status + (uint64_t)t * kDigits + dj, (t == 0 ? kIncl : 0u) | (tw + 1));
+      }
+      c[j] = tw;
+    }
+    digit_scan(c, ex);
+    if (owner)
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j)
+#pragma unroll
+        for (int w = 0; w < kSW; ++w) S.wcnt[w][2 * kP * tid + j] += ex[j];  // absolute stage slots
+    if (tid == 0) S.tile[(it + 1) & 1] = atomicAdd(ticket, 1u);  // the next tile, for the prefetch
+    __syncthreads();
+    // 3. ranks → stage (as sort_scatter_kernel); the tile's offsets in the
+    // digit runs are not needed before step 4
+#pragma unroll
+    for (int k = 0; k < kSB; ++k) {
+      const uint32_t d = dg[k];
+      if (ok[k]) S.tag[warp][d] = (uint8_t)lane;
+      __syncwarp();
+      const uint32_t win = S.tag[warp][d];
+      const bool clash = __any_sync(0xFFFFFFFFu, ok[k] && win != lane);
+      const uint32_t peers = clash ? winner_peers(win, ok[k]) : (1u << lane);
+      uint32_t* wc = &S.wcnt[warp][d];
+      const uint32_t slot = ok[k] ? *wc : 0u;
+      __syncwarp();
+      if (ok[k]) {
+        S.stage[slot + __popc(peers & lt)] = rec[k];
+        if (lane == (uint32_t)__ffs(peers) - 1) *wc = slot + __popc(peers);
+      }
+      __syncwarp();
+    }
+    const uint32_t tn = S.tile[(it + 1) & 1];
+    if (tn < nT) {  // the next tile's loads fly during the look-back and the copy-out
+      rd = RecReader<PASS, kSB>(src, n, (uint64_t)tn * kRound + warp * 32 * kSB, lane, halo);
+      rd.load(lane);
+    }
+    // 2b. look-back: the tile's offset in each digit run = the sum of the
+    // earlier tiles' counts, down to the nearest inclusive prefix. The status
+    // words of the previous tile for all of the thread's digits are read at
+    // once (usually inclusive already: one L2 round trip); walking further
+    // reads kLB tiles per round trip
+#ifndef LCF_SWEEP_NOLB
+#define LCF_SWEEP_NOLB 0  // timing experiment only: no look-back (wrong offsets)
+#endif
+    if (owner && LCF_SWEEP_NOLB) {
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) S.delta[2 * kP * tid + j] = S.gbase[2 * kP * tid + j] - ex[j];
+    } else if (owner) {
+      uint32_t v0[2 * kP];
+      const uint32_t* sp = status + (uint64_t)(t > 0 ? t - 1 : 0) * kDigits + 2 * kP * tid;
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) v0[j] = t > 0 ? ld_relaxed_u32(sp + j) : (kIncl | 1u);
+#pragma unroll
+      for (int j = 0; j < 2 * kP; ++j) {
+        const uint32_t dj = 2 * kP * tid + j;
+        while (v0[j] == 0) v0[j] = ld_relaxed_u32(sp + j);
+        uint32_t excl = (v0[j] & ~kIncl) - 1;
+        if (!(v0[j] & kIncl)) {  // tile t − 1 not yet inclusive: walk on
+          constexpr int kLB = LCF_SWEEP_LB;
+          bool done = false;
+          for (int64_t s0 = (int64_t)t - 2; !done; s0 -= kLB) {
+            uint32_t v[kLB];
+#pragma unroll
+            for (int b = 0; b < kLB; ++b)
+              v[b] = s0 - b >= 0 ? ld_relaxed_u32(status + (uint64_t)(s0 - b) * kDigits + dj) : (kIncl | 1u);
+#pragma unroll
+            for (int b = 0; b < kLB; ++b) {
+              if (done) break;
+              while (v[b] == 0) v[b] = ld_relaxed_u32(status + (uint64_t)(s0 - b) * kDigits + dj);
+              excl += (v[b] & ~kIncl) - 1;
+              done = (v[b] & kIncl) != 0;
+            }
+          }
+        }
+        if (t > 0) st_relaxed_u32(status + (uint64_t)t * kDigits + dj, kIncl | (excl + c[j] + 1));
+        S.delta[dj] = S.gbase[dj] + excl - ex[j];
+      }
+    }
+    __syncthreads();
+    // 4. stage → dst, digit runs contiguous
+    for (uint32_t j = tid; j < nr; j += kST) {
+      const uint64_t v = S.stage[j];
+      dst[S.delta[rec_digit(v, PASS)] + j] = v;
+    }
+    t = tn;
+    // (step 1's barrier of the next tile orders these reads of stage / delta
+    // before they are rewritten)
+  }
+}
+
 // Thread t covers the kMatchItems sorted positions k = 8t … 8t+7; for each,
 // the nearest of the records k−1 … k−4 with the same hash and an equal word is
 // the match (L174, A-14, A-15). Records of one hash are contiguous, so the walk
@@ -664,7 +904,11 @@ uint64_t n_tiles_of(uint64_t n) { return (n + kTile - 1) / kTile; }
 
 }  // namespace
 
+static uint64_t n_sweep_tiles_of(uint64_t n) { return (n + kRound - 1) / kRound; }
+constexpr size_t kSweepMeta = 16384;  // tot2 (2 × kDigits u32) and the two tickets
+
 size_t fcm_dist_workspace(uint64_t n) {
+  if (LCF_ONESWEEP) return 2 * round16(8 * n) + kSweepMeta + 2 * round16(4 * n_sweep_tiles_of(n) * kDigits) + 256;
   return 2 * round16(8 * n) + round16(4 * n_tiles_of(n) * kDigits) + 4 * kDigits + 256;
 }
 
@@ -701,8 +945,40 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
     return true;
   }();
   (void)init;
-  int launches = sorted ? 0 : 6;
-  if (!sorted) {  // (sorted: rec_b still holds this shard's sorted records from the summary call)
+  int launches = sorted ? 0 : (LCF_ONESWEEP ? 3 : 6);
+  if (!sorted && LCF_ONESWEEP) {  // (sorted: rec_b still holds this shard's sorted records from the summary call)
+    static const bool init1 = [] {
+      cudaFuncSetAttribute(sort_onesweep_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)sizeof(OnesweepSmem));
+      cudaFuncSetAttribute(sort_onesweep_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)sizeof(OnesweepSmem));
+      return true;
+    }();
+    (void)init1;
+    const uint64_t T1 = n_sweep_tiles_of(n);
+    uint8_t* meta = p + 2 * round16(8 * n);
+    uint32_t* tot2 = reinterpret_cast<uint32_t*>(meta);
+    uint32_t* tick = tot2 + 2 * kDigits;
+    uint32_t* st0 = reinterpret_cast<uint32_t*>(meta + kSweepMeta);
+    uint32_t* st1 = reinterpret_cast<uint32_t*>(meta + kSweepMeta + round16(4 * T1 * kDigits));
+    cudaMemsetAsync(meta, 0, kSweepMeta + 2 * round16(4 * T1 * kDigits), st);
+    {
+      KTrace kt("fcm_sort_ghist", st);
+      const uint64_t ranges = (n + kWarpRecs - 1) / kWarpRecs;
+      const unsigned gb = (unsigned)umin64((ranges + kSortWarps - 1) / kSortWarps, 148 * 4);
+      sort_ghist_kernel<<<gb, kSortThreads, 0, st>>>(x, n, tot2, halo);
+    }
+    const int grid = persistent_grid(sort_onesweep_kernel<0>, kST, sizeof(OnesweepSmem), T1);
+    {
+      KTrace kt("fcm_sort_scatter", st);
+      sort_onesweep_kernel<0><<<grid, kST, sizeof(OnesweepSmem), st>>>(x, n, tot2, st0, tick, rec_a, halo);
+    }
+    {
+      KTrace kt("fcm_sort_scatter", st);
+      sort_onesweep_kernel<1><<<grid, kST, sizeof(OnesweepSmem), st>>>(rec_a, n, tot2 + kDigits, st1, tick + 1,
+                                                                     rec_b, 0);
+    }
+  } else if (!sorted) {
   {
     KTrace kt("fcm_sort_hist", st);
     sort_hist_kernel<0><<<(unsigned)T, kSortThreads, 0, st>>>(x, n, counts, halo);

@@ -17,7 +17,8 @@ os.makedirs("profiles", exist_ok=True)
 
 def short(name):
     for k, v in (("sort_hist_kernel", "fcm_sort_hist"), ("sort_scan_kernel", "fcm_sort_scan"),
-                 ("sort_scatter_kernel", "fcm_sort_scatter")):
+                 ("sort_scatter_kernel", "fcm_sort_scatter"), ("sort_ghist_kernel", "fcm_sort_ghist"),
+                 ("sort_onesweep_kernel", "fcm_sort_scatter")):
         if k in name:
             return v
     for k in ("speed_encode_kernel<unsigned int>", "speed_encode_kernel<unsigned long>",

@@ -1,24 +1,26 @@
 // lcf_dpratio.cu — DPratio = per chunk (RARE ∘ RAZE ∘ DIFFMS₆₄) over FCM(x)
 // (§3.2) on sm_100a.
 //
-// Compress (4 launches):
-//   fcm_hash_kernel   h(i) from x[i−1..i−3] (A-13) and the index, coalesced
-//   CUB radix sort    (h, i) pairs on the 20 key bits — stable, so equal hashes
-//                     stay in index order (L197: "we use the CUB library")
-//   fcm_match_kernel  per sorted position: the nearest of the 4 preceding pairs
-//                     with the same hash and the same 64-bit word (A-14); the
-//                     block stages its sorted window and the gathered words in
-//                     shared memory, then scatters the 32-bit distance
-//   dpratio_encode    persistent pipeline; item = 2048-word tile t → chunk 2t
-//                     (V) and 2t+1 (Dist) (A-16); per chunk DIFFMS₆₄ → RAZE →
-//                     RARE in shared memory (L201: histogram of leading-zero
-//                     counts by warp-aggregated shared atomics; k from the prefix
-//                     sums; bit fields emitted with warp segmented scans)
-// Decompress (1 launch): dpratio_decode — per tile: RARE⁻¹ → RAZE⁻¹ → DIFFMS⁻¹
-//   for V and Dist, then the FCM decode of the tile (L197) fused in: references
-//   inside the tile are resolved by pointer jumping in shared memory, references
-//   to earlier tiles read the already written output after an acquire on that
-//   tile's completion flag (tiles complete in ticket order, so no cycles).
+// Compress: the FCM distances come from lcf_fcm.cu (the repo's own two-pass
+// LSD radix sort of h | fp | i records, fcm_match's nearest same-hash
+// candidates, fcm_verify in index order — L172–176, A-13..A-15); then
+//   dpratio_encode   persistent pipeline (loader warp, storer warp, 8 compute
+//                    warps); item = 2048-word tile t → chunk 2t (V) and 2t+1
+//                    (Dist) (A-16); DIFFMS₆₄ in registers, RAZE → RARE planned
+//                    from clz histograms (L201: shared atomics; k* from the
+//                    prefix sums) and emitted by per-thread bit writers
+// Decompress:
+//   dpratio_decode   per tile: RARE⁻¹ → RAZE⁻¹ → DIFFMS⁻¹ for Dist and V, then
+//                    the FCM decode of the tile (L197): references inside the
+//                    tile by pointer jumping in shared memory, references into
+//                    a completed earlier tile read its output; everything else
+//                    is left PENDING (global target index + a bitmap bit) —
+//                    no tile ever waits for another
+//   dp_walk_nodes / dp_gather_leaves / dp_gather_nodes (one stream) or
+//   dp_find_roots / dp_gather_roots (shards, peer streams through CUDA IPC):
+//                    the pending words' roots by pointer walks with path
+//                    compression (the paper's union-find "find"), then the
+//                    values
 
 #include "lcf_persist.cuh"
 

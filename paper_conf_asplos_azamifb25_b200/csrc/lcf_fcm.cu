@@ -14,11 +14,15 @@
 //
 // Each pass is three kernels over tiles of kTile = 16 Ki records, 16 warps per
 // tile, warp w owning records [w·1024, (w+1)·1024) of the tile:
-//   sort_hist    per-tile digit counts (warp-aggregated shared atomics)
+//   sort_hist    per-tile digit counts (shared atomics)
 //   sort_scan    per-digit exclusive prefix over tiles (column scan) + totals
-//   sort_scatter per-warp digit counts → per-warp offsets inside the tile's
-//                digit run; then each warp walks its records in order and
-//                ranks equal digits with __match_any_sync → stable scatter
+//   sort_scatter in rounds of 8 Ki records: per-warp digit counts → per-warp
+//                stage slots inside the round's digit runs; each warp ranks
+//                equal digits in lane order (a tag store per digit detects
+//                clashes, five ballots on the winning lane id match the peers)
+//                → the round's records sorted in a shared stage → copied out
+//                with each digit run contiguous
+// (LCF_ONESWEEP builds a measured-slower onesweep variant: below.)
 #include "lcf_fcm.cuh"
 #include "lcf_kernels.cuh"
 

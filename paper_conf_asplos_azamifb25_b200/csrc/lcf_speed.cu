@@ -5,8 +5,10 @@
 // that running CTAs already own.
 //
 // Encode CTA (320 threads):
-//   warp 0  loader : ticket → 1-D TMA bulk load of the chunk into a 3-stage
-//                    shared-memory ring (mbarrier complete_tx)
+//   warp 0  loader : ticket → 1-D TMA bulk load of the chunk into a
+//                    shared-memory stage (1 stage: it is released as soon as
+//                    the compute warps hold the chunk in registers; mbarrier
+//                    complete_tx)
 //   warp 1  storer : decoupled look-back for the chunk's output offset →
 //                    1-D TMA bulk store of the packed chunk → size-table entry
 //   warps 2-9      : DIFFMS in registers (L110–112) → per-subchunk width by a

@@ -357,10 +357,12 @@ __device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t 
     uint32_t o[4] = {__funnelshift_r(pw, q.x, 8), __funnelshift_r(q.x, q.y, 8), __funnelshift_r(q.y, q.z, 8),
                      __funnelshift_r(q.z, q.w, 8)};
     if (w == 0) o[0] = (L & 0xFFFFu) | (q.x << 24);
+    if (w + 4 >= nw) {  // the group holding the stream's last word: mask past it
 #pragma unroll
-    for (uint32_t i = 0; i < 4; ++i) {
-      const uint32_t keep = w + i < nw ? 3 + L - 4 * (w + i) : 0;  // bytes of this word inside the output
-      if (keep < 4) o[i] &= keep ? (1u << (8 * keep)) - 1u : 0u;
+      for (uint32_t i = 0; i < 4; ++i) {
+        const uint32_t keep = w + i < nw ? 3 + L - 4 * (w + i) : 0;  // bytes of this word inside the output
+        if (keep < 4) o[i] &= keep ? (1u << (8 * keep)) - 1u : 0u;
+      }
     }
     reinterpret_cast<uint4*>(dst)[g] = make_uint4(o[0], o[1], o[2], o[3]);
   }

@@ -696,6 +696,9 @@ __global__ void __launch_bounds__(kST, 1) sort_onesweep_kernel(const uint64_t* _
 // stops at the first other hash. The 12 records a thread needs come from six
 // 16-byte loads (no shared memory, no barriers). The distance array is
 // pre-zeroed; only matches are scattered.
+#ifndef LCF_MATCH_SPLIT
+#define LCF_MATCH_SPLIT 1
+#endif
 #ifndef LCF_MATCH_ITEMS
 #define LCF_MATCH_ITEMS 8
 #endif
@@ -718,7 +721,7 @@ template <bool CARRY>
 __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                 const uint64_t* __restrict__ rec,
                                                                 uint32_t* __restrict__ dist, FcmCarry carry,
-                                                                uint64_t gbase) {
+                                                                uint64_t gbase, uint32_t ilo, uint32_t ihi) {
   constexpr bool carry_on = CARRY;
   const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
   for (uint64_t g = blockIdx.x * (uint64_t)kMatchBlock + threadIdx.x; g < groups;
@@ -783,7 +786,7 @@ __global__ void __launch_bounds__(kMatchBlock) fcm_match_kernel(const uint64_t* 
             d = i - (uint32_t)(r[4 + j - back] & kRecIdxMask);
           }
         }
-        if (d) dist[i] = d;
+        if (d && i - ilo < ihi - ilo) dist[i] = d;  // (this launch's index range only)
       } else {
 #pragma unroll
       for (int back = 1; back <= 4; ++back) {  // nearest first (pinned by Fig. 6)
@@ -1027,8 +1030,19 @@ int launch_fcm_shard(const uint64_t* x, uint64_t n, uint32_t halo, uint64_t gbas
     KTrace kt("fcm_match", st);
     const uint64_t groups = (n + kMatchItems - 1) / kMatchItems;
     const int mblocks = (int)umin64((groups + kMatchBlock - 1) / kMatchBlock, 148 * 16);
-    if (carry) fcm_match_kernel<true><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
-    else fcm_match_kernel<false><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase);
+    if (carry) {
+      fcm_match_kernel<true><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase, 0u, 0xFFFFFFFFu);
+    } else {
+      // LCF_MATCH_SPLIT launches, each writing the distances of one index range
+      // only: the scattered writes of a launch then land in an L2-sized part
+      // of the distance array
+      const uint32_t parts = LCF_MATCH_SPLIT;
+      for (uint32_t q = 0; q < parts; ++q) {
+        const uint32_t lo = (uint32_t)(n * q / parts), hi = (uint32_t)(n * (q + 1) / parts);
+        fcm_match_kernel<false><<<mblocks, kMatchBlock, 0, st>>>(x, n, rec_b, dist, c, gbase, lo, hi);
+      }
+      launches += parts - 1;
+    }
   }
   if (!carry) {  // deferred candidates → distances
     KTrace kt("fcm_verify", st);

@@ -117,11 +117,13 @@ struct BitWriter {
   uint32_t widx, w0, nb, pw;  // current word, first word, pending bits (< 32), pending word
   __device__ __forceinline__ BitWriter(uint32_t* b, uint64_t off)
       : buf(b), widx((uint32_t)(off >> 5)), w0((uint32_t)(off >> 5)), nb((uint32_t)(off & 31)), pw(0) {}
+#if !LCF_BW_PRED
   __device__ __forceinline__ void out(uint32_t w) {
     if (widx == w0) atomicOr(buf + widx, w);
     else buf[widx] = w;
     ++widx;
   }
+#endif
   // append the low w bits of f (f < 2^w, 0 ≤ w ≤ 64; w = 0 needs f = 0)
   __device__ __forceinline__ void put(uint64_t f, uint32_t w) {
     const uint32_t flo = (uint32_t)f, fhi = (uint32_t)(f >> 32);

@@ -25,6 +25,7 @@ def short(name):
               "speed_decode_kernel<unsigned int>", "speed_decode_kernel<unsigned long>",
               "spratio_encode_kernel", "spratio_decode_kernel", "dpratio_encode_kernel", "dpratio_decode_kernel",
               "fcm_hash_kernel", "fcm_match_kernel", "dp_find_roots_kernel", "dp_gather_roots_kernel", "fcm_verify_kernel",
+              "dp_walk_nodes_kernel", "dp_gather_leaves_kernel", "dp_gather_nodes_kernel",
               "fcm_carry_merge_kernel", "fcm_summary_kernel", "DeviceRadixSortOnesweepKernel", "DeviceRadixSortHistogramKernel",
               "DeviceRadixSortExclusiveSumKernel", "write_header_kernel"):
         if k in name:

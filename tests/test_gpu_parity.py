@@ -379,6 +379,45 @@ def test_host_buffer_api(L, orc):
     assert m == words.nbytes and np.array_equal(back, words)
 
 
+def test_host_api_two_threads(L, orc, monkeypatch):
+    """The host API from two threads at once, each on its own CUDA stream (the
+    bench's e2e pipeline: one thread compresses while the other decompresses):
+    per-stream workspaces keep the calls independent — every stream equals the
+    oracle's and every field comes back bit-exact, over sliced host paths."""
+    import threading
+    monkeypatch.setenv("LCF_HOST_SLICE_BYTES", str(5 * 16384))
+    fields = []
+    for k, algo in enumerate(("SPspeed", "SPratio", "DPspeed", "DPratio") * 2):
+        dt = np.float32 if algo.startswith("SP") else np.float64
+        w = datagen.smooth_1d(24 * 16384 // np.dtype(dt).itemsize + 37 * k, dt, seed=40 + k).view(wdt(algo)).copy()
+        if algo == "DPratio":
+            w[3000:] = np.resize(w[:2500], w.size - 3000)  # FCM matches across host slices
+        fields.append((algo, w, orc.compress(algo, w)))
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    errors = []
+
+    def worker(t):
+        try:
+            for rep in range(3):
+                for algo, w, ref in fields[t::2]:
+                    cap = L.lcf_max_compressed_size(algo, None, w.nbytes)
+                    hout = np.zeros(cap, np.uint8)
+                    n = L.lcf_compress_host(algo, None, w, w.nbytes, hout, cap, stream=streams[t])
+                    assert hout[:n].tobytes() == ref, (algo, rep)
+                    back = np.zeros_like(w)
+                    assert L.lcf_decompress_host(algo, None, hout, n, back, back.nbytes, stream=streams[t]) == w.nbytes
+                    assert np.array_equal(back, w), (algo, rep)
+        except BaseException as e:
+            errors.append(e)
+
+    ths = [threading.Thread(target=worker, args=(t,)) for t in range(2)]
+    for th in ths:
+        th.start()
+    for th in ths:
+        th.join()
+    assert not errors, errors
+
+
 @pytest.mark.parametrize("algo", GPU_ALGOS)
 def test_host_pipelined_slices(L, orc, algo, monkeypatch):
     """The sliced host path (3-chunk slices: 14 slices and a ragged tail; for

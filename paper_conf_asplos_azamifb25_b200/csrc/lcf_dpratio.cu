@@ -53,15 +53,14 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
 
 __device__ __forceinline__ uint32_t clz64(uint64_t v) { return __clzll(v); }
 
-// 64-bit field of width w (≤ 64) at bit position P of the little-endian word
-// stream at `base` (4-byte aligned; reads up to 12 bytes).
-__device__ __forceinline__ uint64_t get_field(const uint32_t* base, uint64_t P, uint32_t w) {
-  if (w == 0) return 0;
+// 64-bit field at bit position P of the little-endian word stream at `base`
+// (4-byte aligned; reads up to 12 bytes; P < 2^32: shared-memory streams),
+// masked by the caller's precomputed 2^w − 1 (all ones for w = 64, 0 for w = 0).
+__device__ __forceinline__ uint64_t get_field_m(const uint32_t* base, uint32_t P, uint64_t mask) {
   const uint32_t* p = base + (P >> 5);
   const uint32_t r = P & 31;
   const uint32_t lo = __funnelshift_r(p[0], p[1], r), hi = __funnelshift_r(p[1], p[2], r);
-  const uint64_t v = ((uint64_t)hi << 32) | lo;
-  return w >= 64 ? v : v & ((1ull << w) - 1);
+  return (((uint64_t)hi << 32) | lo) & mask;
 }
 
 // Words 8·tid … 8·tid+7 of sv with 16-byte shared loads; quad q of thread t is
@@ -440,8 +439,9 @@ __device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, 
   if (!bad && (int32_t)(3 + hib + lob + tl) != s1) bad = 1;
   if (bad) return -1;  // (warp-uniform, and the same in every warp)
   const uint32_t* sw = reinterpret_cast<const uint32_t*>(base);
-  const uint64_t f0 = 8ull * off;  // bit position of the stream in base
-  const uint64_t lo_base = f0 + 8ull * (3 + hib);
+  const uint32_t f0 = 8 * off;  // bit position of the stream in base (< 2^20: shared memory)
+  const uint32_t lo_base = f0 + 8 * (3 + hib);
+  const uint64_t hmask = k >= 64 ? ~0ull : (1ull << k) - 1, lmask = wl ? (1ull << wl) - 1 : 0ull;
   // word i = 32·(B1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane;
   // q's parity is the warp's (kDW even), so the source register is warp-uniform
   static_assert(kDW % 2 == 0, "B1 word parity = warp parity");
@@ -457,12 +457,12 @@ __device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, 
       uint64_t tp;
       if (rare) {
         const uint32_t ri = re + set;  // set words up to and including i
-        tp = ri ? get_field(sw, f0 + 24 + (uint64_t)(ri - 1) * k, k) : 0;
+        tp = ri ? get_field_m(sw, f0 + 24 + (ri - 1) * k, hmask) : 0;
       } else {
-        tp = set ? get_field(sw, f0 + 24 + (uint64_t)re * k, k) : 0;
+        tp = set ? get_field_m(sw, f0 + 24 + re * k, hmask) : 0;
       }
-      const uint64_t lw = get_field(sw, lo_base + (uint64_t)i * wl, wl);
-      *reinterpret_cast<uint64_t*>(dst + 8 * i) = k == 64 ? tp : ((tp << wl) | lw);
+      const uint64_t lw = get_field_m(sw, lo_base + i * wl, lmask);  // (0 for k = 64)
+      *reinterpret_cast<uint64_t*>(dst + 8 * i) = (tp << wl) | lw;
     }
   }
   if (tid < tl) dst[8 * n + tid] = base[lo_base / 8 + (n * wl + 7) / 8 + tid];

@@ -369,19 +369,50 @@ __device__ __forceinline__ void a_emit_bypass_smem(const uint8_t* src, uint32_t 
   }
 }
 
+// CTA-wide exclusive scan of u64 over the kDT compute threads. The warp sums go
+// to slot sh[sp] and sp flips, so consecutive scans need no trailing barrier.
+__device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t (*sh)[kDW], uint32_t& sp, uint32_t tid,
+                                                 uint64_t& total) {
+  const uint32_t warp = tid >> 5, lane = tid & 31;
+  uint64_t x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+    if ((int)lane >= d) x += y;
+  }
+  uint64_t* s = sh[sp];
+  sp ^= 1;
+  if (lane == 31) s[warp] = x;
+  bar_d();
+  uint64_t base = 0;
+  total = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < kDW; ++i) {
+    const uint64_t t = s[i];
+    if (i < warp) base += t;
+    total += t;
+  }
+  return base + x - v;
+}
+
 // Decode a RAZE/RARE stream of `len` bytes at src (16-byte aligned, ≥ 16 bytes
 // of readable slack) into dst (8-byte aligned, capacity cap). Returns the
 // decoded length or −1 if malformed. All kDT compute threads call it. Every
 // warp rebuilds B1 from B3 → B2 → B1 itself (lane l: B1 words 2l, 2l+1 and
 // their set-word prefixes), so the only barrier is the one after dst.
+// FUSE (RAZE⁻¹ of a DIFFMS stream, raze_diffms_inv): the words go straight
+// into DIFFMS⁻¹ (see there); −2 = a bypassed stream, left to the plain path.
+template <bool FUSE = false>
 __device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, uint8_t* dst, uint32_t cap, bool rare,
-                               uint32_t tid) {
+                               uint32_t tid, uint64_t (*scan)[kDW] = nullptr, uint32_t* sp = nullptr,
+                               uint64_t* any = nullptr) {
   const uint32_t warp = tid >> 5, lane = tid & 31;
   const uint8_t* src = base + off;  // the stream (base: 4-byte aligned)
   if (len < 3) return -1;
   const uint32_t L = src[0] | ((uint32_t)src[1] << 8), k = src[2];
   if (L > cap) return -1;
   if (k == 0) {  // bypass: dst[j] = src[3 + j], one funnel shift per word
+    if (FUSE) return -2;  // (the caller decodes it unfused)
     if (len != 3 + L) return -1;
     const uint32_t* sw = reinterpret_cast<const uint32_t*>(base) + (off + 3) / 4;
     const uint32_t fs = 8 * ((off + 3) % 4);
@@ -442,6 +473,45 @@ __device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, 
   const uint32_t f0 = 8 * off;  // bit position of the stream in base (< 2^20: shared memory)
   const uint32_t lo_base = f0 + 8 * (3 + hib);
   const uint64_t hmask = k >= 64 ? ~0ull : (1ull << k) - 1, lmask = wl ? (1ull << wl) - 1 : 0ull;
+  if constexpr (FUSE) {
+    // RAZE⁻¹ fused with DIFFMS⁻¹ (no tail, L = cap = 8m): thread t decodes
+    // words 8t … 8t+7 — B1 byte t, from lane t/8's B1 words — straight into
+    // registers, unTCMS, then the CTA scan; dst receives the final words
+    // after the scan's barrier (no round trip through dst before it)
+    if (L != cap || tl) return -1;  // (uniform)
+    const uint32_t sl = tid >> 3;
+    const uint32_t a0 = __shfl_sync(0xFFFFFFFFu, w0, sl), a1 = __shfl_sync(0xFFFFFFFFu, w1, sl);
+    const uint32_t e0 = __shfl_sync(0xFFFFFFFFu, cnt0, sl), e1 = __shfl_sync(0xFFFFFFFFu, cnt1, sl);
+    const bool odd = (tid >> 2) & 1;
+    const uint32_t bw = odd ? a1 : a0, sh8 = 8 * (tid & 3);
+    const uint32_t byte = (bw >> sh8) & 0xFFu;
+    uint32_t re = (odd ? e1 : e0) + __popc(bw & ((1u << sh8) - 1u));  // set words before word 8t
+    uint64_t v[8], run = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const uint32_t i = 8 * tid + j;
+      const bool set = (byte >> j) & 1;
+      const uint64_t tp = set ? get_field_m(sw, f0 + 24 + re * k, hmask) : 0;
+      re += set;
+      const uint64_t lw = get_field_m(sw, lo_base + i * wl, lmask);
+      v[j] = i < n ? tcms_inv((tp << wl) | lw) : 0;
+      run += v[j];
+    }
+    uint64_t tot;
+    uint64_t acc = cta_scan_u64(run, scan, *sp, tid, tot);
+    uint64_t an = 0;
+    uint64_t* arr = reinterpret_cast<uint64_t*>(dst);
+#pragma unroll
+    for (int j = 0; j < 8; j += 2) {
+      const uint64_t x0 = acc + v[j], x1 = x0 + v[j + 1];
+      acc = x1;
+      reinterpret_cast<ulonglong2*>(arr)[4 * tid + j / 2] = make_ulonglong2(x0, x1);  // words ≥ m: scratch
+      if (8 * tid + j < n) an |= x0;
+      if (8 * tid + j + 1 < n) an |= x1;
+    }
+    *any = an;
+    return (int)L;
+  }
   // word i = 32·(B1 word index) + lane: B1 word q = 8r + warp covers i = 256 r + 32 warp + lane;
   // q's parity is the warp's (kDW even), so the source register is warp-uniform
   static_assert(kDW % 2 == 0, "B1 word parity = warp parity");
@@ -468,32 +538,6 @@ __device__ int adaptive_decode(const uint8_t* base, uint32_t off, uint32_t len, 
   if (tid < tl) dst[8 * n + tid] = base[lo_base / 8 + (n * wl + 7) / 8 + tid];
   bar_d();
   return (int)L;
-}
-
-// CTA-wide exclusive scan of u64 over the kDT compute threads. The warp sums go
-// to slot sh[sp] and sp flips, so consecutive scans need no trailing barrier.
-__device__ __forceinline__ uint64_t cta_scan_u64(uint64_t v, uint64_t (*sh)[kDW], uint32_t& sp, uint32_t tid,
-                                                 uint64_t& total) {
-  const uint32_t warp = tid >> 5, lane = tid & 31;
-  uint64_t x = v;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
-    if ((int)lane >= d) x += y;
-  }
-  uint64_t* s = sh[sp];
-  sp ^= 1;
-  if (lane == 31) s[warp] = x;
-  bar_d();
-  uint64_t base = 0;
-  total = 0;
-#pragma unroll
-  for (uint32_t i = 0; i < kDW; ++i) {
-    const uint64_t t = s[i];
-    if (i < warp) base += t;
-    total += t;
-  }
-  return base + x - v;
 }
 
 // =================================== encode ======================================
@@ -874,6 +918,14 @@ __device__ __forceinline__ int fixed_zero_stream(const uint8_t* rz, int l1, uint
 // barrier after the scan; returns false if malformed.
 __device__ __forceinline__ bool raze_diffms_inv(const uint8_t* rz, uint32_t off, int l1, uint32_t m, uint64_t* arr,
                                                 uint64_t& any, DDecSmem& S, uint32_t& sp, uint32_t tid) {
+#ifndef LCF_DEC_FUSE
+#define LCF_DEC_FUSE 1
+#endif
+  if (LCF_DEC_FUSE) {
+    const int lf = adaptive_decode<true>(rz, off, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, tid,
+                                         S.scan, &sp, &any);
+    if (lf != -2) return lf == (int)(8 * m);  // else a bypassed RAZE stream: below
+  }
   const int l0 = adaptive_decode(rz, off, (uint32_t)l1, reinterpret_cast<uint8_t*>(arr), 8 * m, false, tid);
   if (l0 != (int)(8 * m)) return false;
   // DIFFMS⁻¹: thread owns words [8·tid, 8·tid+8), moved as 16-byte pairs

@@ -81,6 +81,13 @@ __device__ __forceinline__ void tma_store_1d(void* gmem_dst, const void* smem_sr
                "r"(smem_addr(smem_src)), "r"(bytes)
                : "memory");
 }
+// 2-D tensor store of the box at smem_src (laid out as the tensor map's
+// swizzle mode prescribes) to tensor coordinates (c0, c1)
+__device__ __forceinline__ void tma_store_2d(const void* tmap, const void* smem_src, int32_t c0, int32_t c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tmap), "r"(c0),
+               "r"(c1), "r"(smem_addr(smem_src))
+               : "memory");
+}
 __device__ __forceinline__ void tma_store_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void tma_store_wait_read0() {
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");

@@ -17,6 +17,8 @@
 // Decode inverts the stages from the end of the payload (B4 → B3 → B2 → B1 →
 // D), transposes back, and runs DIFFMS⁻¹ as a serial per-group scan plus a CTA
 // scan of the group totals.
+#include <cuda.h>
+
 #include "lcf_persist.cuh"
 
 namespace lcf {
@@ -131,7 +133,7 @@ struct RDecSmem {
   alignas(128) uint32_t in[kRDecStages][(kChunkBytes + 64) / 4];
   // T: decoded D (plane-major, 4096 words), then — once every thread holds its
   // group in registers — the decoded words with a 33-word row stride (X)
-  alignas(128) uint32_t T[kRT * 33];
+  alignas(1024) uint32_t T[kRT * 33];  // (1024-aligned: the 128-byte swizzle of the output box)
   alignas(16) uint8_t B1[2048 + 16];
   alignas(16) uint8_t B2[256 + 16];
   uint64_t full_in[kRDecStages], empty_in[kRDecStages];
@@ -336,7 +338,7 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
 #define LCF_SPR_ENC_MINB 6
 #endif
 __global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
-  extern __shared__ __align__(128) uint8_t smem_raw[];
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -354,8 +356,16 @@ __global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB) spratio_encode
 }
 
 // =================================== decode ======================================
+// Output of a full chunk (LCF_SPR_TMA_OUT): thread g writes its group's 32
+// decoded words as row g of a 128 × 128-byte box in S.T, 16-byte piece q at
+// q ^ (g mod 8) (the 128-byte swizzle: conflict-free, no register shuffling),
+// and one thread stores the box with a 2-D TMA tensor store that un-swizzles
+// it into 16 KiB of contiguous output. Ragged chunks keep the thread stores.
+#ifndef LCF_SPR_TMA_OUT
+#define LCF_SPR_TMA_OUT 1
+#endif
 __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, const LaunchCtx& ctx, uint32_t cw,
-                                              uint32_t lane) {
+                                              uint32_t lane, const CUtensorMap* tmap) {
   const uint32_t g = cw * 32 + lane;
   const uint4 h0 = reinterpret_cast<const uint4*>(a.stream)[0];
   const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / 4;
@@ -363,7 +373,10 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
     const uint32_t s = it % kRDecStages, ph = (it / kRDecStages) & 1;
     mbar_wait(&S.full_in[s], ph);
     const uint64_t t = S.chunk[s];
-    if (t == kNoChunk) return;
+    if (t == kNoChunk) {
+      if (g == 0) tma_store_wait_all0();  // the last box has left S.T
+      return;
+    }
     const uint32_t len = S.len[s], fl = S.flags[s];
     const uint32_t m = chunk_words(n_words, t, 4096);
     uint32_t* dst = reinterpret_cast<uint32_t*>(a.out) + t * 4096;
@@ -431,6 +444,7 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
         S.s2 = s2;
         S.bad = bad;
       }
+      if (lane == 0) tma_store_wait_read0();  // the previous chunk's box has been read out of S.T
     }
     bar_r();
     int32_t bad = S.bad;
@@ -541,6 +555,20 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
     // the scan's barrier also ends every read of T: X overwrites it below
     const uint32_t base = cta_excl_scan<uint32_t>(tot, S.sc32[1], cw, lane, all);
     uint32_t* const Xs = S.T;
+    if (tmap && m == 4096) {
+      uint8_t* row = reinterpret_cast<uint8_t*>(S.T) + 128 * g;
+#pragma unroll
+      for (uint32_t q = 0; q < 8; ++q)
+        *reinterpret_cast<uint4*>(row + 16 * (q ^ (g & 7))) =
+            make_uint4(X[4 * q] + base, X[4 * q + 1] + base, X[4 * q + 2] + base, X[4 * q + 3] + base);
+      fence_proxy_async_smem();
+      bar_r();
+      if (g == 0) {
+        tma_store_2d(tmap, S.T, 0, (int32_t)(t * 128));
+        tma_store_commit();
+      }
+      continue;
+    }
     if (g < G || (g == G && (m & 31))) {
 #pragma unroll
       for (int i = 0; i < 32; ++i) Xs[g * 33 + i] = X[i] + base;
@@ -563,8 +591,9 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
 #ifndef LCF_SPR_DEC_MINB
 #define LCF_SPR_DEC_MINB 5
 #endif
-__global__ void __launch_bounds__(kRDecThreads, LCF_SPR_DEC_MINB) spratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
-  extern __shared__ __align__(128) uint8_t smem_raw[];
+__global__ void __launch_bounds__(kRDecThreads, LCF_SPR_DEC_MINB)
+    spratio_decode_kernel(DecArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
   RDecSmem& S = *reinterpret_cast<RDecSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x < 16) {
@@ -585,7 +614,9 @@ __global__ void __launch_bounds__(kRDecThreads, LCF_SPR_DEC_MINB) spratio_decode
   }
   __syncthreads();
   if (warp == 0) dec_loader<kRDecStages, kRDecBatch>(S, a, ctx, lane, 4);
-  else r_dec_compute(S, a, ctx, warp - 1, lane);
+  // (the swizzled box needs a 1024-byte aligned S.T: otherwise thread stores)
+  const bool tma = use_tmap && (smem_addr(S.T) & 1023) == 0;
+  if (warp != 0) r_dec_compute(S, a, ctx, warp - 1, lane, tma ? &tmap : nullptr);
 }
 
 }  // namespace
@@ -610,8 +641,32 @@ void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
   }();
   (void)init;
   const int grid = persistent_grid(spratio_decode_kernel, kRDecThreads, smem, (max_chunks + kRDecBatch - 1) / kRDecBatch);
+  // the output as a [rows][32 words] tensor for the 2-D TMA stores of full chunks
+  // (cuTensorMapEncodeTiled from the driver at run time: no link-time libcuda)
+  typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                               const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                               CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static EncodeFn encode = [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      fn = nullptr;
+    return reinterpret_cast<EncodeFn>(fn);
+  }();
+  CUtensorMap tm;
+  memset(&tm, 0, sizeof(tm));
+  uint32_t use = 0;
+  const uint64_t rows = a.out_capacity / 128;
+  if (LCF_SPR_TMA_OUT && encode && rows >= 128 && rows < (1ull << 31) && ((uintptr_t)a.out & 15) == 0) {
+    const cuuint64_t dims[2] = {32, rows}, strides[1] = {128};
+    const cuuint32_t box[2] = {32, 128}, es[2] = {1, 1};
+    use = encode(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, a.out, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                 CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+  }
   KTrace kt("spratio_decode", st);
-  spratio_decode_kernel<<<grid, kRDecThreads, smem, st>>>(a, ctx);
+  spratio_decode_kernel<<<grid, kRDecThreads, smem, st>>>(a, ctx, tm, use);
 }
 
 }  // namespace lcf

@@ -117,13 +117,18 @@ __device__ __forceinline__ RZESizes rze_sizes(uint32_t L) {
 }
 
 struct REncSmem {
-  alignas(128) uint32_t in[kRStages][4096];  // raw chunk, then its encoding
+  // raw chunk, then its encoding. A full chunk arrives by a 2-D TMA tensor load
+  // as 128 rows of 128 bytes (one 32-word group per row) in the 128-byte
+  // swizzle — 16-byte piece q of row g at q ^ (g mod 8), so that every thread
+  // reads its own group conflict-free and in word order; a ragged chunk by a
+  // 1-D copy in plain order (in_swz)
+  alignas(1024) uint32_t in[kRStages][4096];
   alignas(128) uint32_t T[4096];  // BIT output = RZE input D
   alignas(16) uint8_t B1[2048 + 16];
   alignas(16) uint8_t B2[256 + 16];
   uint64_t full_in[kRStages], empty_in[kRStages], full_out[kRStages];
   uint64_t in_chunk[kRStages], out_chunk[kRStages];
-  uint32_t out_len[kRStages], out_raw[kRStages];
+  uint32_t out_len[kRStages], out_raw[kRStages], in_swz[kRStages];
   uint64_t sc64[2][kRW];
   uint32_t sc32[2][kRW];
   uint32_t b3;  // B3 bytes (≤ 32), kept by warp 0 in registers; B4 here
@@ -164,31 +169,28 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     const uint32_t G = m / 32;  // full groups; m mod 32 leftover words are copied (A-9)
     const uint32_t* in = S.in[s];
 
-    // ---- 1. DIFFMS (L110–112) in the rotated order, 2. BIT (L140–142) ----
+    // ---- 1. DIFFMS (L110–112), 2. BIT (L140–142) ----
+    const bool swz = S.in_swz[s];
     if (g < G) {
-      const uint32_t gr = g & 7, rot = 4 * gr;
       uint32_t A[32];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) {  // a'[4q..4q+3] = words 32g + 4((q+gr)&7) .. : conflict-free
-        const uint4 v = reinterpret_cast<const uint4*>(in)[8 * g + ((q + gr) & 7)];
+      for (int q = 0; q < 8; ++q) {  // words 32g + 4q …: piece q of row g (swizzled: conflict-free)
+        const uint4 v = reinterpret_cast<const uint4*>(in)[8 * g + (swz ? (q ^ (g & 7)) : q)];
         A[4 * q] = v.x; A[4 * q + 1] = v.y; A[4 * q + 2] = v.z; A[4 * q + 3] = v.w;
       }
-      const uint32_t xprev = g ? in[32 * g - 1] : 0u;
-      // word 32g sits at rotated index 4·kx, kx = (8 − gr) mod 8: its predecessor
-      // is xprev (a select per quad start, so that U stays in registers)
-      const uint32_t kx = (8 - gr) & 7;
-      uint32_t U[32];
+      const uint32_t r = g - 1;  // word 32g − 1: last word of row g − 1
+      const uint32_t xprev = g ? in[32 * r + 4 * (swz ? (7 ^ (r & 7)) : 7) + 3] : 0u;
 #pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        uint32_t pre = A[(j + 31) & 31];
-        if ((j & 3) == 0) pre = (uint32_t)(j >> 2) == kx ? xprev : pre;
-        U[j] = tcms(A[j] - pre);
+      for (int j = 31; j >= 0; --j) A[j] = tcms(A[j] - (j ? A[j - 1] : xprev));
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {  // rows reversed → planes MSB-first
+        const uint32_t tmp = A[i];
+        A[i] = A[31 - i];
+        A[31 - i] = tmp;
       }
-#pragma unroll
-      for (int i = 0; i < 32; ++i) A[i] = U[31 - i];  // rows reversed → planes MSB-first
       transpose32(A);
 #pragma unroll
-      for (int p = 0; p < 32; ++p) S.T[p * G + g] = __funnelshift_l(A[p], A[p], rot);  // undo rotation
+      for (int p = 0; p < 32; ++p) S.T[p * G + g] = A[p];
     } else if (g == G && (m & 31)) {  // leftover words: DIFFMS, copied unchanged by BIT
       for (uint32_t i = 32 * G; i < m; ++i) S.T[i] = tcms(in[i] - (i ? in[i - 1] : 0u));
     }
@@ -291,6 +293,10 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
     }
     uint8_t* ob = reinterpret_cast<uint8_t*>(S.in[s]);
     if (raw) {  // the stage still holds the raw chunk: zero its padding
+      if (swz) {  // (a full chunk, swizzled in the stage: its bytes again, from L2 / HBM)
+        const uint4* src = reinterpret_cast<const uint4*>(reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes);
+        for (uint32_t q = g; q < kChunkBytes / 16; q += kRT) reinterpret_cast<uint4*>(ob)[q] = __ldcg(src + q);
+      }
       if (g < round16(len) - len) ob[len + g] = 0;
     } else {
       // nz(D): non-zero bytes of every unit at its scanned offset
@@ -334,10 +340,85 @@ __device__ __forceinline__ void r_enc_compute(REncSmem& S, const EncArgs& a, con
   }
 }
 
+// The loader: as enc_loader (lcf_persist.cuh), but a full chunk comes as one
+// 2-D TMA tensor load of its 128 × 128-byte box into the swizzled stage.
+__device__ __forceinline__ void r_enc_loader(REncSmem& S, const EncArgs& a, const LaunchCtx& ctx, uint32_t lane,
+                                             const CUtensorMap* tmap) {
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kRStages, ph = (it / kRStages) & 1;
+    mbar_wait(&S.empty_in[s], ph ^ 1);
+    uint64_t t = 0;
+    if (lane == 0) t = atomicAdd(ctx.ticket, 1ull);
+    t = __shfl_sync(0xFFFFFFFFu, t, 0);
+    if (t >= a.n_chunks) {
+      if (lane == 0) {
+        S.in_chunk[s] = kNoChunk;
+        mbar_arrive(&S.full_in[s]);
+        ticket_retire(ctx);
+      }
+      return;
+    }
+    const uint32_t bytes = chunk_words(a.n_words_total, a.first_chunk + t, 4096) * 4;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(a.in) + t * kChunkBytes;
+    if (lane == 0) trace_stamp(a, t, 0);
+    if (tmap && bytes == kChunkBytes) {
+      if (lane == 0) {
+        S.in_chunk[s] = t;
+        S.in_swz[s] = 1;
+        mbar_arrive_expect_tx(&S.full_in[s], kChunkBytes);
+        tma_load_2d(S.in[s], tmap, 0, (int32_t)(t * 128), &S.full_in[s]);
+      }
+    } else if ((bytes & 15) == 0) {
+      if (lane == 0) {
+        S.in_chunk[s] = t;
+        S.in_swz[s] = 0;
+        mbar_arrive_expect_tx(&S.full_in[s], bytes);
+        tma_load_1d(S.in[s], src, bytes, &S.full_in[s]);
+      }
+    } else {  // ragged tail chunk: plain loads
+      for (uint32_t i = lane; i < bytes / 4; i += 32) S.in[s][i] = reinterpret_cast<const uint32_t*>(src)[i];
+      if (lane == 0) {
+        S.in_chunk[s] = t;
+        S.in_swz[s] = 0;
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&S.full_in[s]);
+    }
+  }
+}
+
+// A [rows][32 u32] tensor map over `base` for 2-D TMA boxes of 128 rows in the
+// 128-byte swizzle (cuTensorMapEncodeTiled from the driver at run time, so the
+// library needs no link-time libcuda); false if unavailable.
+static bool rows_tensor_map(CUtensorMap* tm, const void* base, uint64_t rows) {
+  typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                               const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                               CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static EncodeFn encode = [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      fn = nullptr;
+    return reinterpret_cast<EncodeFn>(fn);
+  }();
+  memset(tm, 0, sizeof(*tm));
+  if (!encode || rows < 128 || rows >= (1ull << 31) || ((uintptr_t)base & 15)) return false;
+  const cuuint64_t dims[2] = {32, rows}, strides[1] = {128};
+  const cuuint32_t box[2] = {32, 128}, es[2] = {1, 1};
+  return encode(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(base), dims, strides, box, es,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+#ifndef LCF_SPR_TMA_IN
+#define LCF_SPR_TMA_IN 1
+#endif
 #ifndef LCF_SPR_ENC_MINB
 #define LCF_SPR_ENC_MINB 6
 #endif
-__global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB) spratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
+__global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB)
+    spratio_encode_kernel(EncArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -350,7 +431,9 @@ __global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB) spratio_encode
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (warp == 0) enc_loader<kRStages>(S, a, ctx, lane, 4);
+  // (the swizzled box needs a 1024-byte aligned stage: otherwise 1-D copies)
+  const bool tma = use_tmap && (smem_addr(S.in[0]) & 1023) == 0;
+  if (warp == 0) r_enc_loader(S, a, ctx, lane, tma ? &tmap : nullptr);
   else if (warp == 1) enc_storer<kRStages, 1, REncSmem, true>(S, a, ctx, lane, 0);
   else r_enc_compute(S, a, ctx, warp - 2, lane);
 }
@@ -629,8 +712,12 @@ void launch_spratio_encode(const EncArgs& a, const LaunchCtx& ctx, cudaStream_t 
   }();
   (void)init;
   const int grid = persistent_grid(spratio_encode_kernel, kREncThreads, smem, a.n_chunks);
+  // full chunks of this launch (only the stream's last chunk can be ragged)
+  const uint64_t full = (a.first_chunk + a.n_chunks) * 4096 <= a.n_words_total ? a.n_chunks : a.n_chunks - 1;
+  CUtensorMap tm;
+  const uint32_t use = LCF_SPR_TMA_IN && rows_tensor_map(&tm, a.in, full * 128);
   KTrace kt("spratio_encode", st);
-  spratio_encode_kernel<<<grid, kREncThreads, smem, st>>>(a, ctx);
+  spratio_encode_kernel<<<grid, kREncThreads, smem, st>>>(a, ctx, tm, use);
 }
 
 void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_chunks, cudaStream_t st) {
@@ -642,29 +729,8 @@ void launch_spratio_decode(const DecArgs& a, const LaunchCtx& ctx, uint64_t max_
   (void)init;
   const int grid = persistent_grid(spratio_decode_kernel, kRDecThreads, smem, (max_chunks + kRDecBatch - 1) / kRDecBatch);
   // the output as a [rows][32 words] tensor for the 2-D TMA stores of full chunks
-  // (cuTensorMapEncodeTiled from the driver at run time: no link-time libcuda)
-  typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                               const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
-                               CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-  static EncodeFn encode = [] {
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess)
-      fn = nullptr;
-    return reinterpret_cast<EncodeFn>(fn);
-  }();
   CUtensorMap tm;
-  memset(&tm, 0, sizeof(tm));
-  uint32_t use = 0;
-  const uint64_t rows = a.out_capacity / 128;
-  if (LCF_SPR_TMA_OUT && encode && rows >= 128 && rows < (1ull << 31) && ((uintptr_t)a.out & 15) == 0) {
-    const cuuint64_t dims[2] = {32, rows}, strides[1] = {128};
-    const cuuint32_t box[2] = {32, 128}, es[2] = {1, 1};
-    use = encode(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, a.out, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                 CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-  }
+  const uint32_t use = LCF_SPR_TMA_OUT && rows_tensor_map(&tm, a.out, a.out_capacity / 128);
   KTrace kt("spratio_decode", st);
   spratio_decode_kernel<<<grid, kRDecThreads, smem, st>>>(a, ctx, tm, use);
 }

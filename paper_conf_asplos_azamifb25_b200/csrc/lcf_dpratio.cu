@@ -1122,7 +1122,10 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
           par ^= 1;
         }
         if (li < m) S.X[li] = val;  // x (or a pending target), in place
-        if (li < m && f) atomicOr(&S.pmask[li / 32], 1u << (li % 32));
+        {  // the warp's 32 consecutive words are one bitmap word (blocks start at multiples of 256)
+          const uint32_t pm = __ballot_sync(0xFFFFFFFFu, li < m && f);
+          if (lane == 0 && b + (tid & ~31u) < m) S.pmask[(b + (tid & ~31u)) / 32] = pm;
+        }
         // mark the word a pending word points at (a chain node, walked first by
         // dp_find_roots); lanes hitting the same bitmap word send one OR
         const bool mk = li < m && f && val >= gb && val - gb < n_words;

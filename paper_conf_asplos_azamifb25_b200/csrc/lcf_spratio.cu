@@ -2,21 +2,23 @@
 // on sm_100a, in the persistent warp-specialised pipeline of lcf_persist.cuh.
 //
 // Compute threads: 128 (4 warps); thread g owns the 32-word group g of a chunk.
-// Encode, per chunk:
-//   1. thread g reads its group from the TMA-loaded stage with a per-thread
-//      quad rotation (bank-conflict-free), DIFFMS in the rotated order
+// Encode, per chunk (loader warp, storer warp, one in-place stage):
+//   1. a full chunk arrives by a 2-D TMA tensor load into a 128-byte-swizzled
+//      stage (row g = group g), so thread g reads its group conflict-free and
+//      in word order; DIFFMS (L110–112) in registers
 //   2. BIT (L140–142, L162): 32×32 bit transpose in registers (5 butterfly
-//      stages); rows are fed reversed so plane p comes out MSB-first; the
-//      quad rotation becomes a bit rotation of each plane word, undone with one
-//      funnel shift → T[p·G + g] into shared memory (plane-major)
+//      stages, the 16- and 8-bit ones as byte permutes); rows are fed reversed
+//      so plane p comes out MSB-first → T[p·G + g] (plane-major)
 //   3. RZE (L144–148, L164): byte bitmap B1 of 16-byte units with a packed
 //      8-way CTA scan of the unit counts; repetition elimination B1→B2 (CTA
 //      scan), B2→B3 and B3→B4 in warp 0 (warp scan, ballot); every section
 //      size is known before a byte is written, so the aggregate is published
-//      first; then the non-zero and non-repeating bytes are scattered.
+//      first; then the non-zero and non-repeating bytes are scattered into the
+//      stage, which the storer's TMA bulk store reads out.
 // Decode inverts the stages from the end of the payload (B4 → B3 → B2 → B1 →
-// D), transposes back, and runs DIFFMS⁻¹ as a serial per-group scan plus a CTA
-// scan of the group totals.
+// D), transposes back, runs DIFFMS⁻¹ as a serial per-group scan plus a CTA
+// scan of the group totals, and writes a full chunk by a 2-D TMA tensor store
+// from a 128-byte-swizzled box.
 #include <cuda.h>
 
 #include "lcf_persist.cuh"

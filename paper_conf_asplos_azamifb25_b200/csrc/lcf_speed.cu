@@ -17,7 +17,7 @@
 //                    known → bit packing (L116) into a 2-slot output ring.
 // Decode CTA (288 threads):
 //   warp 0  loader : ticket → size entry → aggregate published at once →
-//                    look-back → TMA bulk load of the payload (4 stages)
+//                    look-back → TMA bulk load of the payload (3 stages)
 //   warps 1-8      : unpack (funnel shifts) → unTCMS → DIFFMS⁻¹ as a CTA-wide
 //                    prefix sum (L132) → 16-byte coalesced stores.
 // Each compute warp owns subchunks 4w..4w+3 (512 B, L118); a lane holds K = 4

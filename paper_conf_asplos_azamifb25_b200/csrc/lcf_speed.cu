@@ -171,6 +171,23 @@ __device__ __forceinline__ void emit_equal(uint32_t* buf, uint32_t lane, uint32_
     if (j < e || (j == e && keep_last)) buf[F + j] = T[j];
 }
 
+// LCF_ENC_OR: the same strings OR-ed into an output slot that is zero by
+// invariant (the storer re-zeroes what it stored before handing the slot back):
+// no shuffle of the partial word, no select of the last word, one predicated
+// shared reduction per touched word.
+#ifndef LCF_ENC_OR
+#define LCF_ENC_OR 1
+#endif
+__device__ __forceinline__ void emit_or(uint32_t* buf, uint32_t lane, uint32_t L, const uint32_t* S) {
+  const uint32_t P = lane * L, F = P >> 5, r = P & 31;
+  const uint32_t e = (r + L - 1) >> 5;  // index of the last word touched (0..4)
+  const uint32_t T[5] = {S[0] << r, __funnelshift_l(S[0], S[1], r), __funnelshift_l(S[1], S[2], r),
+                         __funnelshift_l(S[2], S[3], r), __funnelshift_l(S[3], 0u, r)};
+#pragma unroll
+  for (uint32_t j = 0; j < 5; ++j)
+    if (j <= e) atomicOr(buf + F + j, T[j]);
+}
+
 // ---- shared-memory field extraction (decode) ------------------------------------
 __device__ __forceinline__ void split_string(const uint32_t* U4, uint32_t w, uint32_t* v) {
   const uint32_t m = w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u);
@@ -342,7 +359,9 @@ __device__ __forceinline__ void enc_compute(EncSmem& S, const EncArgs& a, const 
         uint32_t Sg[4];
         make_string(v[q], w, Sg);
         uint32_t* buf = S.out[o] + (off >> 2);
-        if (L >= 32) {
+        if (LCF_ENC_OR) {
+          emit_or(buf, lane, L, Sg);  // (L < 32 too: a word shared by several lanes takes their ORs)
+        } else if (L >= 32) {
           emit_equal(buf, lane, L, Sg);
         } else {
           emit_bits_warp(buf, (uint64_t)lane * L, L, (uint64_t)Sg[0] | ((uint64_t)Sg[1] << 32),
@@ -385,9 +404,12 @@ __global__ void LCF_ENC_BOUNDS speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if (LCF_ENC_OR)  // the output slots start zeroed (then re-zeroed by the storer)
+    for (uint32_t i = threadIdx.x; i < sizeof(S.out) / 16; i += blockDim.x)
+      reinterpret_cast<uint4*>(&S.out[0][0])[i] = make_uint4(0, 0, 0, 0);
   __syncthreads();
   if (warp == 0) enc_loader<kEncStages>(S, a, ctx, lane, sizeof(U));
-  else if (warp <= kStorers) enc_storer<kEncOut, kStorers>(S, a, ctx, lane, warp - 1);
+  else if (warp <= kStorers) enc_storer<kEncOut, kStorers, EncSmem, false, LCF_ENC_OR>(S, a, ctx, lane, warp - 1);
   else enc_compute<U>(S, a, ctx, warp - 1 - kStorers, lane);
 }
 

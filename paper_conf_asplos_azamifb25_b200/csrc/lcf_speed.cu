@@ -172,7 +172,9 @@ __device__ __forceinline__ void emit_equal(uint32_t* buf, uint32_t lane, uint32_
 }
 
 // LCF_ENC_OR: the same strings OR-ed into an output slot that is zero by
-// invariant (the storer re-zeroes what it stored before handing the slot back):
+// invariant (the storer re-zeroes what it stored before handing the slot back;
+// zeroing by the compute warps behind one more barrier measured equal, a third
+// output slot at 3 CTAs/SM slower):
 // no shuffle of the partial word, no select of the last word, one predicated
 // shared reduction per touched word.
 #ifndef LCF_ENC_OR

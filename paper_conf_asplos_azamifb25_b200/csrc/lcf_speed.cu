@@ -180,14 +180,34 @@ __device__ __forceinline__ void emit_equal(uint32_t* buf, uint32_t lane, uint32_
 #ifndef LCF_ENC_OR
 #define LCF_ENC_OR 1
 #endif
+#ifndef LCF_ENC_OR_UNIFORM
+#define LCF_ENC_OR_UNIFORM 1
+#endif
 __device__ __forceinline__ void emit_or(uint32_t* buf, uint32_t lane, uint32_t L, const uint32_t* S) {
   const uint32_t P = lane * L, F = P >> 5, r = P & 31;
   const uint32_t e = (r + L - 1) >> 5;  // index of the last word touched (0..4)
+#if LCF_ENC_OR_UNIFORM
+  // words past emax = (L + 30) / 32 (warp-uniform: L is the subchunk's) are
+  // touched by no lane: uniform branches skip their shifts and reductions
+  const uint32_t emax = (L + 30) >> 5;
+  atomicOr(buf + F, S[0] << r);
+  if (emax >= 1) {
+    if (e >= 1) atomicOr(buf + F + 1, __funnelshift_l(S[0], S[1], r));
+    if (emax >= 2) {
+      if (e >= 2) atomicOr(buf + F + 2, __funnelshift_l(S[1], S[2], r));
+      if (emax >= 3) {
+        if (e >= 3) atomicOr(buf + F + 3, __funnelshift_l(S[2], S[3], r));
+        if (emax >= 4 && e >= 4) atomicOr(buf + F + 4, __funnelshift_l(S[3], 0u, r));
+      }
+    }
+  }
+#else
   const uint32_t T[5] = {S[0] << r, __funnelshift_l(S[0], S[1], r), __funnelshift_l(S[1], S[2], r),
                          __funnelshift_l(S[2], S[3], r), __funnelshift_l(S[3], 0u, r)};
 #pragma unroll
   for (uint32_t j = 0; j < 5; ++j)
     if (j <= e) atomicOr(buf + F + j, T[j]);
+#endif
 }
 
 // ---- shared-memory field extraction (decode) ------------------------------------

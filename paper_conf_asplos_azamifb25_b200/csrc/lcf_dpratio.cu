@@ -770,7 +770,7 @@ __device__ __forceinline__ void d_enc_compute(DEncSmem& S, const EncArgs& a, con
 __global__ void __launch_bounds__(kDEncThreads, LCF_ENC_MINB) dpratio_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DEncSmem& S = *reinterpret_cast<DEncSmem*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   // invariants: both histograms, S.rz and the output slots start zeroed
   for (uint32_t i = threadIdx.x; i < 2 * 66; i += blockDim.x) (&S.sc.hist[0][0])[i] = 0;
   for (uint32_t i = threadIdx.x; i < sizeof(S.rz) / 16; i += blockDim.x)
@@ -1181,7 +1181,7 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
 __global__ void __launch_bounds__(kDDecThreads, 3) dpratio_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DDecSmem& S = *reinterpret_cast<DDecSmem*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     mbar_init(&S.full_v[0], 1);
     mbar_init(&S.empty_v[0], kDW);

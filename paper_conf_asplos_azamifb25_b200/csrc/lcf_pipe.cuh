@@ -110,6 +110,15 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// The warp's index, broadcast from lane 0: ptxas then knows that a branch on it
+// (the warp-role dispatch of the persistent kernels) is warp-uniform, and
+// compiles the warp-synchronous code behind it (shuffles, votes, redux) without
+// WARPSYNC.COLLECTIVE / ENDCOLLECTIVE convergence wrappers. Requires the whole
+// warp to be active at the call (kernel entry).
+__device__ __forceinline__ uint32_t warp_index_uniform() {
+  return __shfl_sync(0xFFFFFFFFu, threadIdx.x >> 5, 0);
+}
+
 // ---- named barriers (id 0 is __syncthreads) ------------------------------------
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");

@@ -104,14 +104,32 @@ template <> __device__ __forceinline__ uint4 pack16<uint64_t>(const uint64_t* v)
 }
 
 // ---- MPLG width: bitlen(max) == bitlen(OR) over the subchunk --------------------
+// LCF_REDUX: 0 = __reduce_or_sync, 1 = redux.sync in inline PTX, 2 = a
+// butterfly of shuffles
+#ifndef LCF_REDUX
+#define LCF_REDUX 0
+#endif
+__device__ __forceinline__ uint32_t warp_or(uint32_t x) {
+#if LCF_REDUX == 1
+  uint32_t o;
+  asm volatile("redux.sync.or.b32 %0, %1, 0xffffffff;" : "=r"(o) : "r"(x));
+  return o;
+#elif LCF_REDUX == 2
+#pragma unroll
+  for (int d = 16; d >= 1; d >>= 1) x |= __shfl_xor_sync(0xFFFFFFFFu, x, d);
+  return x;
+#else
+  return __reduce_or_sync(0xFFFFFFFFu, x);
+#endif
+}
 __device__ __forceinline__ uint32_t warp_width(const uint32_t* v) {
-  const uint32_t o = __reduce_or_sync(0xFFFFFFFFu, v[0] | v[1] | v[2] | v[3]);
+  const uint32_t o = warp_or(v[0] | v[1] | v[2] | v[3]);
   return 32 - __clz(o);
 }
 __device__ __forceinline__ uint32_t warp_width(const uint64_t* v) {
   const uint64_t x = v[0] | v[1];
-  const uint32_t hi = __reduce_or_sync(0xFFFFFFFFu, (uint32_t)(x >> 32));
-  const uint32_t lo = __reduce_or_sync(0xFFFFFFFFu, (uint32_t)x);
+  const uint32_t hi = warp_or((uint32_t)(x >> 32));
+  const uint32_t lo = warp_or((uint32_t)x);
   return hi ? 64 - __clz(hi) : 32 - __clz(lo);
 }
 
@@ -414,7 +432,7 @@ template <typename U>
 __global__ void LCF_ENC_BOUNDS speed_encode_kernel(EncArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   EncSmem& S = *reinterpret_cast<EncSmem*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kEncStages; ++i) {
       mbar_init(&S.full_in[i], 1);
@@ -575,7 +593,7 @@ template <typename U>
 __global__ void LCF_DEC_BOUNDS speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   DecSmem<U>& S = *reinterpret_cast<DecSmem<U>*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kDecStages; ++i) {
       mbar_init(&S.full_in[i], 1);

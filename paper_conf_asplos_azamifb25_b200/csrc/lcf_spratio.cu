@@ -423,7 +423,7 @@ __global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB)
     spratio_encode_kernel(EncArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kRStages; ++i) {
       mbar_init(&S.full_in[i], 1);
@@ -680,7 +680,7 @@ __global__ void __launch_bounds__(kRDecThreads, LCF_SPR_DEC_MINB)
     spratio_decode_kernel(DecArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   RDecSmem& S = *reinterpret_cast<RDecSmem*>(smem_raw);
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x < 16) {
     const uint32_t m = threadIdx.x;
     uint32_t sel = 0, c = 0;

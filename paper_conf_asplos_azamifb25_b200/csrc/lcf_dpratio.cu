@@ -46,7 +46,7 @@ __device__ __forceinline__ bool bar_d_or(bool p) {
                : "=r"(r)
                : "r"((uint32_t)p), "r"(kBarD), "r"(kDT)
                : "memory");
-  return r != 0;
+  return warp_uniform(r) != 0;  // (CTA-uniform; broadcast so that ptxas knows it)
 }
 
 // ============================ RAZE / RARE in shared memory ============================
@@ -977,12 +977,12 @@ __device__ __forceinline__ void d_dec_compute(DDecSmem& S, const DecArgs& a, con
   FcmScratch& F = *reinterpret_cast<FcmScratch*>(S.rz);
   for (uint32_t it = 0;; ++it) {
     mbar_wait(&S.full_v[0], it & 1);
-    const uint64_t t = S.tile[0];
+    const uint64_t t = warp_uniform(S.tile[0]);
     if (t == kNoChunk) {
       finish_pending();
       return;
     }
-    const uint32_t fl = S.flags[0], lenV = S.len[0], lenD = S.len[1];
+    const uint32_t fl = warp_uniform(S.flags[0]), lenV = warp_uniform(S.len[0]), lenD = warp_uniform(S.len[1]);
     const uint32_t m = (uint32_t)umin64(kTileWords, n_words - t * kTileWords);
     if (tid == 0) trace_stamp(a, t, 2);
     bool ok = !(fl & 4);

@@ -25,6 +25,7 @@
 // (LCF_ONESWEEP builds a measured-slower onesweep variant: below.)
 #include "lcf_fcm.cuh"
 #include "lcf_kernels.cuh"
+#include "lcf_pipe.cuh"
 
 namespace lcf {
 namespace {
@@ -129,7 +130,7 @@ template <int PASS>
 __global__ void __launch_bounds__(kSortThreads) sort_hist_kernel(const uint64_t* __restrict__ src, uint64_t n,
                                                                  uint32_t* __restrict__ counts, uint32_t halo) {
   __shared__ uint32_t hist[kDigits];
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   for (uint32_t d = threadIdx.x; d < kDigits; d += kSortThreads) hist[d] = 0;
   __syncthreads();
   const uint64_t start = (uint64_t)blockIdx.x * kTile + warp * kWarpRecs;
@@ -157,7 +158,7 @@ constexpr int kScanDig = 8, kScanSub = 32 / kScanDig;
 __global__ void __launch_bounds__(kScanWarps * 32) sort_scan_kernel(uint32_t* __restrict__ counts, uint32_t n_tiles,
                                                                    uint32_t* __restrict__ tot) {
   __shared__ uint32_t part[kScanWarps][32];
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   const uint32_t dl = lane % kScanDig, sub = lane / kScanDig;
   const uint32_t d = blockIdx.x * kScanDig + dl;
   const uint32_t t0 = (uint32_t)((uint64_t)warp * n_tiles / kScanWarps);
@@ -483,7 +484,7 @@ __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
 __global__ void __launch_bounds__(kSortThreads) sort_ghist_kernel(const uint64_t* __restrict__ x, uint64_t n,
                                                                   uint32_t* __restrict__ tot2, uint32_t halo) {
   __shared__ uint32_t hist[2][kDigits];
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   for (uint32_t d = threadIdx.x; d < 2 * kDigits; d += kSortThreads) (&hist[0][0])[d] = 0;
   __syncthreads();
   const uint64_t ranges = (n + kWarpRecs - 1) / kWarpRecs;

@@ -119,6 +119,12 @@ __device__ __forceinline__ uint32_t warp_index_uniform() {
   return __shfl_sync(0xFFFFFFFFu, threadIdx.x >> 5, 0);
 }
 
+// A value the caller knows to be warp-uniform (read from shared memory by
+// every lane, or the result of a CTA-wide barrier reduction), broadcast from
+// lane 0 so that ptxas can prove it uniform too (same reason as above).
+__device__ __forceinline__ uint32_t warp_uniform(uint32_t v) { return __shfl_sync(0xFFFFFFFFu, v, 0); }
+__device__ __forceinline__ uint64_t warp_uniform(uint64_t v) { return __shfl_sync(0xFFFFFFFFu, v, 0); }
+
 // ---- named barriers (id 0 is __syncthreads) ------------------------------------
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");

@@ -416,6 +416,9 @@ static bool rows_tensor_map(CUtensorMap* tm, const void* base, uint64_t rows) {
 #ifndef LCF_SPR_TMA_IN
 #define LCF_SPR_TMA_IN 1
 #endif
+#ifndef LCF_SPR_ENC_WU
+#define LCF_SPR_ENC_WU 0  // the uniform warp index (no convergence wrappers) measured 1 % slower here
+#endif
 #ifndef LCF_SPR_ENC_MINB
 #define LCF_SPR_ENC_MINB 6
 #endif
@@ -423,7 +426,7 @@ __global__ void __launch_bounds__(kREncThreads, LCF_SPR_ENC_MINB)
     spratio_encode_kernel(EncArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   REncSmem& S = *reinterpret_cast<REncSmem*>(smem_raw);
-  const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
+  const uint32_t warp = LCF_SPR_ENC_WU ? warp_index_uniform() : threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kRStages; ++i) {
       mbar_init(&S.full_in[i], 1);

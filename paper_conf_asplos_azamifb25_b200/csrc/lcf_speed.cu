@@ -78,7 +78,19 @@ struct EncSmem {
   uint32_t hdr[2][32];
 };
 
+// Decoder payload stages per word type: the f32 decoder at 40 registers fits 5
+// CTAs per SM with 2 stages (NYX velocity 184 → 182 µs, HACC xx 341 → 334 µs);
+// the f64 decoder measured slower that way (123 → 124.5 µs) and keeps 3 stages
+// at 4 CTAs per SM.
+#ifndef LCF_DEC_STAGES_U32
+#define LCF_DEC_STAGES_U32 2
+#endif
+template <typename U> struct DecCfg {
+  static constexpr int kStages = sizeof(U) == 4 ? LCF_DEC_STAGES_U32 : kDecStages;
+  static constexpr int kMinBlocks = sizeof(U) == 4 && LCF_DEC_STAGES_U32 == 2 ? 5 : 4;
+};
 template <typename U> struct DecSmem {
+  static constexpr int kDecStages = DecCfg<U>::kStages;
   alignas(128) uint32_t in[kDecStages][(kChunkBytes + 64) / 4];
   uint64_t full_in[kDecStages], empty_in[kDecStages];
   uint64_t chunk[kDecStages];
@@ -463,6 +475,7 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
   const uint64_t n_words = (((uint64_t)h0.w << 32) | h0.z) / sizeof(U);
   uint32_t scan_it = 0;
   for (uint32_t it = 0;; ++it) {
+    constexpr int kDecStages = DecCfg<U>::kStages;
     const uint32_t s = it % kDecStages, ph = (it / kDecStages) & 1;
     mbar_wait(&S.full_in[s], ph);
     const uint64_t t = S.chunk[s];
@@ -587,7 +600,7 @@ __device__ __forceinline__ void dec_compute(DecSmem<U>& S, const DecArgs& a, con
 #ifdef LCF_DEC_MINB
 #define LCF_DEC_BOUNDS __launch_bounds__(kDecThreads, LCF_DEC_MINB)
 #else
-#define LCF_DEC_BOUNDS __launch_bounds__(kDecThreads)
+#define LCF_DEC_BOUNDS __launch_bounds__(kDecThreads, DecCfg<U>::kMinBlocks)
 #endif
 template <typename U>
 __global__ void LCF_DEC_BOUNDS speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
@@ -595,14 +608,14 @@ __global__ void LCF_DEC_BOUNDS speed_decode_kernel(DecArgs a, LaunchCtx ctx) {
   DecSmem<U>& S = *reinterpret_cast<DecSmem<U>*>(smem_raw);
   const uint32_t warp = warp_index_uniform(), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kDecStages; ++i) {
+    for (int i = 0; i < DecCfg<U>::kStages; ++i) {
       mbar_init(&S.full_in[i], 1);
       mbar_init(&S.empty_in[i], kCompWarps);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (warp == 0) dec_loader<kDecStages, kDecBatch>(S, a, ctx, lane, sizeof(U));
+  if (warp == 0) dec_loader<DecCfg<U>::kStages, kDecBatch>(S, a, ctx, lane, sizeof(U));
   else dec_compute<U>(S, a, ctx, warp - 1, lane);
 }
 

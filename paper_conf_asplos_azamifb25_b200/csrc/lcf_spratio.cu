@@ -677,7 +677,7 @@ __device__ __forceinline__ void r_dec_compute(RDecSmem& S, const DecArgs& a, con
 }
 
 #ifndef LCF_SPR_DEC_MINB
-#define LCF_SPR_DEC_MINB 5
+#define LCF_SPR_DEC_MINB 6  // 64 registers, no spills since the warp-uniform dispatch: 6 CTAs/SM (NYX velocity 324 -> 304 us)
 #endif
 __global__ void __launch_bounds__(kRDecThreads, LCF_SPR_DEC_MINB)
     spratio_decode_kernel(DecArgs a, LaunchCtx ctx, const __grid_constant__ CUtensorMap tmap, uint32_t use_tmap) {

@@ -164,7 +164,7 @@ struct BitWriter {
 // (the k choice, B2, B3, the section sizes) is computed redundantly by every
 // warp from shared data, so no warp waits on another's serial work.
 #ifndef LCF_ENC_MINB
-#define LCF_ENC_MINB 2
+#define LCF_ENC_MINB 3  // 64 registers, 48 B of spills: 3 CTAs/SM (density compress 1325 -> 1297 us, rt_density 1971 -> 1912 us)
 #endif
 struct EncScratch {
   uint32_t hist[2][66];  // clz histograms, alternating per plan; [65]: the tile has an FCM distance
